@@ -1,0 +1,87 @@
+// Device helpers shared by the crk kernels: ring access, vector I/O, byte realignment, byte swaps,
+// warp/block reductions.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "crk_internal.h"
+
+namespace crk {
+
+__device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }
+
+// Byte at ring cursor c (RFC 5531 §11 stream position), wrap at cap (reading R16).
+__device__ __forceinline__ uint8_t ring_byte(const RingDesc& R, uint64_t c) { return R.base[c & R.mask]; }
+
+// Big-endian u32 at ring cursor c (RFC 4506 §4.1), any alignment, across the wrap.
+__device__ __forceinline__ uint32_t ring_be32(const RingDesc& R, uint64_t c) {
+  uint64_t o = c & R.mask;
+  if ((o & 3) == 0) return bswap32(*reinterpret_cast<const uint32_t*>(R.base + o));
+  return ((uint32_t)R.base[o] << 24) | ((uint32_t)R.base[(c + 1) & R.mask] << 16) |
+         ((uint32_t)R.base[(c + 2) & R.mask] << 8) | (uint32_t)R.base[(c + 3) & R.mask];
+}
+
+// 16-byte streaming load of an aligned chunk (read-only for the kernel's lifetime).
+__device__ __forceinline__ uint4 ld16_stream(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st16(void* p, uint4 v) {
+  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ void st16_stream(void* p, uint4 v) {
+  asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+
+// The 16 bytes starting `sh` (0..15) bytes into the 32-byte window a:b (memory order, little-endian
+// words), i.e. a funnel shift across two aligned chunks.  sh is warp-uniform in callers.
+__device__ __forceinline__ uint4 funnel16(uint4 a, uint4 b, uint32_t sh) {
+  const uint32_t q = sh >> 2, r = (sh & 3) * 8;
+  uint32_t w0, w1, w2, w3, w4;
+  switch (q) {
+    case 0: w0 = a.x; w1 = a.y; w2 = a.z; w3 = a.w; w4 = b.x; break;
+    case 1: w0 = a.y; w1 = a.z; w2 = a.w; w3 = b.x; w4 = b.y; break;
+    case 2: w0 = a.z; w1 = a.w; w2 = b.x; w3 = b.y; w4 = b.z; break;
+    default: w0 = a.w; w1 = b.x; w2 = b.y; w3 = b.z; w4 = b.w; break;
+  }
+  uint4 o;
+  o.x = __funnelshift_r(w0, w1, r);
+  o.y = __funnelshift_r(w1, w2, r);
+  o.z = __funnelshift_r(w2, w3, r);
+  o.w = __funnelshift_r(w3, w4, r);
+  return o;
+}
+
+// Reverse the bytes of each esize-byte element of a 16-byte chunk (RFC 4506 big-endian <-> host).
+__device__ __forceinline__ uint4 swap16(uint4 v, uint32_t esize) {
+  if (esize == 4) {
+    v.x = bswap32(v.x); v.y = bswap32(v.y); v.z = bswap32(v.z); v.w = bswap32(v.w);
+  } else if (esize == 8) {
+    uint32_t x = bswap32(v.y), y = bswap32(v.x), z = bswap32(v.w), w = bswap32(v.z);
+    v.x = x; v.y = y; v.z = z; v.w = w;
+  }
+  return v;
+}
+
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+
+// Block-wide min of a u32 (all threads must call).  smem: >= 32 words.
+__device__ __forceinline__ uint32_t block_min_u32(uint32_t v, uint32_t* smem) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
+  const uint32_t w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  __syncthreads();
+  if (lane_id() == 0) smem[w] = v;
+  __syncthreads();
+  v = lane_id() < nw ? smem[lane_id()] : 0xffffffffu;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+}  // namespace crk

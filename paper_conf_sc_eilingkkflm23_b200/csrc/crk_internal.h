@@ -1,0 +1,166 @@
+// Internal structures shared by the crk kernels and the C ABI layer (not part of the public ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/crk.h"
+
+namespace crk {
+
+constexpr int kMaxItems = CRK_MAX_ITEMS;
+constexpr int kMaxProcs = CRK_MAX_PROCS;
+constexpr int kMaxRings = CRK_MAX_RINGS;
+constexpr int kScanThreads = 1024;  // K1: one CTA per ring, one candidate header per thread
+constexpr int kParseWarps = 8;      // K3: one warp per record
+constexpr int kMoveThreads = 256;   // K4/K6 mover CTA
+constexpr int kMaxPieces = 2 * kMaxItems + 2;
+
+struct Schema {
+  uint32_t proc, n_items;
+  uint32_t items[kMaxItems];
+};
+struct SchemaTable {
+  uint32_t n;
+  Schema s[kMaxProcs];
+};
+
+struct RingDesc {
+  uint8_t* base;
+  uint64_t mask;  // cap - 1
+  uint64_t head, tail;
+};
+
+// Device-resident tables of one index (pointers into one cudaMalloc block).
+struct IndexDev {
+  uint32_t max_rings, frags_per_ring, recs_per_ring, max_records;
+  uint32_t hash_mask;
+  RingDesc* rings;              // [max_rings]
+  crk_ring_result* res;         // [max_rings]
+  uint32_t* rec_prefix;         // [max_rings + 1]; [n_rings] = total
+  uint32_t* total;              // device scalar (== rec_prefix[n_rings])
+  uint32_t* ticket;             // scan finish ticket
+  uint64_t* frag_phys;
+  uint64_t* frag_lstart;
+  uint32_t* frag_hdr;
+  uint64_t* rec_begin;
+  uint64_t* rec_len;
+  uint32_t* rec_frag0;
+  uint32_t* rec_nfrags;
+  uint32_t* p_slot;
+  uint32_t* p_ring;
+  uint32_t* p_xid;
+  uint32_t* p_proc;
+  int32_t* p_status;
+  uint32_t* p_nitems;
+  uint32_t* p_kind;
+  uint64_t* p_off;
+  uint64_t* p_count;
+  uint64_t* p_value;
+  int32_t* s_status;
+  int32_t* s_reply_err;
+  uint64_t* s_reply_off;
+  uint64_t* s_reply_wire;
+  unsigned long long* xid_hash;  // (xid << 32 | dense id), empty = ~0
+};
+
+// ---- mover jobs ----------------------------------------------------------------------------------
+// Decode: dst[0..nbytes) <- logical bytes [loff, loff + nbytes) of record `rec`, element-swapped by esize.
+// Encode: the framed record whose logical bytes are the pieces is written to ring `out` from cursor.
+enum : uint32_t { JOB_NONE = 0, JOB_DEC = 1, JOB_ENC = 2 };
+enum : uint32_t { PIECE_WORDS = 0, PIECE_DATA = 1 };
+
+struct Piece {            // 64 bytes
+  uint64_t loff;          // logical offset of the piece within the record
+  uint64_t nbytes;        // WORDS: 4 * nwords; DATA: payload bytes (zero pad to 4 follows implicitly)
+  uint64_t src;           // DATA: device address of element 0
+  uint32_t esize;         // DATA: 1, 4 or 8
+  uint32_t type;          // PIECE_WORDS / PIECE_DATA
+  uint32_t words[8];      // WORDS: host-order values written big-endian
+};
+
+struct Job {              // 64 bytes
+  uint32_t type;          // JOB_*
+  uint32_t esize;         // DEC: element size
+  uint32_t rec;           // DEC: dense record id
+  uint32_t n_pieces;      // ENC
+  uint64_t out_start;     // DEC: dst address; ENC: out-ring cursor of the record's first header byte
+  uint64_t out_end;       // exclusive (DEC: dst + nbytes; ENC: out_start + wire size)
+  uint64_t loff;          // DEC: logical offset of the first byte; ENC: logical length of the record
+  uint32_t piece0;        // ENC: first piece in the piece pool
+  uint32_t F;             // ENC: fragment payload (0 -> explicit fragment table)
+  uint32_t lens0;         // ENC with explicit framing: first entry in the lens / wire-start pool
+  uint32_t n_lens;
+  uint32_t out_ring;      // ENC: index into the out-ring table
+  uint32_t pad_;
+};
+
+struct Scratch {          // ctx-owned device scratch
+  Job* jobs;              // [max_jobs]
+  Piece* pieces;          // [2 * max_jobs]
+  uint32_t* counters;     // [8]: 0 mover tile cursor, 1 n_jobs, 5 K2 block counter
+  uint64_t* lens_pool;    // explicit framing: [2 * max_lens] (lens, then wire starts)
+  uint32_t* lens32;       // [max_lens] staging for host-given fragment lengths
+  unsigned long long* scan_state;  // decoupled look-back state for K2
+  uint64_t* scan_tmp;     // [max_jobs + 2]: sizes -> prefix; [max_jobs + 1] = total
+  RingDesc* out_rings;    // [kMaxRings]
+  uint32_t max_jobs, max_lens, max_pieces;
+};
+
+struct ConfigDev {
+  uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
+  uint64_t max_record_bytes;
+};
+
+// ---- launchers (defined in the k_*.cu files) ------------------------------------------------------
+struct ScanRingsParam {
+  uint32_t n_rings;
+  RingDesc r[kMaxRings];
+};
+
+cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s);
+cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const ConfigDev& cfg, uint32_t n_rings,
+                         int sms, cudaStream_t s);
+// Exclusive scan of n u64 values in place; total (may be null) gets the sum.  n read from n_dev if
+// n_dev is non-null (device count), else n.
+cudaError_t launch_exclusive_scan_u64(uint64_t* data, uint32_t n, const uint32_t* n_dev, uint64_t* total,
+                                      Scratch& sc, cudaStream_t s);
+cudaError_t launch_exclusive_scan_u32(uint32_t* data, uint32_t n, const uint32_t* n_dev, uint32_t* total,
+                                      Scratch& sc, cudaStream_t s);
+
+// Resolving requests into jobs.
+struct H2DReq {
+  uint32_t xid;
+  void* dst;
+  uint64_t dst_bytes;
+  int32_t* status;
+  uint64_t* copied;
+};
+cudaError_t launch_resolve_h2d(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n, const uint32_t* xids,
+                               void* const* dsts, const uint64_t* dst_bytes, int32_t* statuses, uint64_t* copied,
+                               const H2DReq* single, cudaStream_t s);
+cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n,
+                                 const crk_item_req* reqs, const crk_item_req* single, cudaStream_t s);
+cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
+                              const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
+                              uint64_t region_bytes, cudaStream_t s);
+// Encode jobs built on the host (<= a few per call) are copied in by value.
+struct EncJobParam {
+  uint32_t n_jobs, n_pieces;
+  Job jobs[2];
+  Piece pieces[kMaxPieces];
+};
+cudaError_t launch_put_enc_jobs(Scratch& sc, const EncJobParam& p, const RingDesc& out, cudaStream_t s);
+cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const uint32_t* xids,
+                                  const void* const* srcs, const uint64_t* bytes, const int32_t* errs,
+                                  const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
+                                  cudaStream_t s);
+cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n, cudaStream_t s);
+// Plans tiles for jobs [0, n_jobs) (n_jobs from counters[1] <= max_jobs_bound) and runs the mover.
+cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
+                                 int sms, int move_ctas, cudaStream_t s);
+int mover_occupancy();
+
+// host-visible counter of our kernel launches
+void count_launch(int n = 1);
+
+}  // namespace crk

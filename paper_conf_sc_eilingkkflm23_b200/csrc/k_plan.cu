@@ -1,0 +1,372 @@
+// Job builders: turn requests (per-xid decode calls, encode calls) or a whole scanned batch (serve)
+// into mover jobs, applying the oracle's semantic checks in its order (oracle/oracle.c
+// or_decode_memcpy_h2d, or_decode_item, or_serve).
+#include "crk_device.cuh"
+
+namespace crk {
+
+namespace {
+
+constexpr uint32_t kNotFound = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t elem_size_k(uint32_t kind) {
+  switch (kind) {
+    case CRK_K_OPAQUE_VAR: case CRK_K_OPAQUE_FIX: return 1;
+    case CRK_K_I32_VAR: case CRK_K_U32_VAR: case CRK_K_F32_VAR:
+    case CRK_K_I32_FIX: case CRK_K_U32_FIX: case CRK_K_F32_FIX: return 4;
+    case CRK_K_I64_VAR: case CRK_K_U64_VAR: case CRK_K_F64_VAR:
+    case CRK_K_I64_FIX: case CRK_K_U64_FIX: case CRK_K_F64_FIX: return 8;
+    default: return 0;
+  }
+}
+
+// xid -> dense id of the earliest record carrying it (reading R11)
+__device__ __forceinline__ uint32_t xid_lookup(const IndexDev& ix, uint32_t xid) {
+  uint32_t h = (xid * 0x9E3779B1u) & ix.hash_mask;
+  for (;;) {
+    const unsigned long long k = ix.xid_hash[h];
+    if (k == ~0ull) return kNotFound;
+    if ((uint32_t)(k >> 32) == xid) return (uint32_t)k;
+    h = (h + 1) & ix.hash_mask;
+  }
+}
+
+__device__ __forceinline__ uint64_t pad4(uint64_t n) { return (4 - (n & 3)) & 3; }
+__device__ __forceinline__ uint64_t wire_of(uint64_t Ll, uint32_t F) {
+  const uint64_t nfr = Ll == 0 ? 1 : (Ll + F - 1) / F;  // reading R3: >= 1 fragment, no empty trailer
+  return Ll + 4 * nfr;
+}
+
+__device__ __forceinline__ Job dec_job(uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec, uint32_t es) {
+  Job j{};
+  j.type = nbytes ? JOB_DEC : JOB_NONE;
+  j.esize = es;
+  j.rec = rec;
+  j.out_start = dst;
+  j.out_end = dst + nbytes;
+  j.loff = loff;
+  return j;
+}
+
+// memcpy HtoD requests (oracle or_decode_memcpy_h2d)
+__global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint32_t n, const uint32_t* xids,
+                                   void* const* dsts, const uint64_t* dst_bytes, int32_t* statuses, uint64_t* copied,
+                                   H2DReq single, uint32_t use_single) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t xid = use_single ? single.xid : xids[i];
+    const uint64_t dst = (uint64_t)(use_single ? single.dst : dsts[i]);
+    const uint64_t cap = use_single ? single.dst_bytes : dst_bytes[i];
+    int32_t* st_out = use_single ? single.status : statuses + i;
+    uint64_t* cp_out = use_single ? single.copied : (copied ? copied + i : nullptr);
+    Job job{};
+    uint64_t m = 0;
+    int st;
+    const uint32_t d = xid_lookup(ix, xid);
+    if (d == kNotFound) {
+      st = CRK_E_XID;
+    } else if ((st = ix.p_status[d]) == CRK_OK) {
+      if (ix.p_proc[d] != cfg.proc_h2d) {
+        st = CRK_E_PROC;
+      } else {
+        const uint64_t nb = ix.p_count[(uint64_t)d * kMaxItems + 1];
+        const uint64_t size = ix.p_value[(uint64_t)d * kMaxItems + 2];
+        if (cfg.strict && nb != size) st = CRK_E_SIZE;
+        else {
+          m = (cfg.strict || nb <= size) ? nb : size;
+          if (cap < m) { st = CRK_E_PTR; m = 0; }
+          else job = dec_job(dst, m, ix.p_off[(uint64_t)d * kMaxItems + 1], d, 1);
+        }
+      }
+    }
+    if (st != CRK_OK) m = 0;
+    sc.jobs[i] = job;
+    *st_out = st;
+    if (cp_out) *cp_out = m;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+}
+
+// typed / opaque argument requests (oracle or_decode_item)
+__global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint32_t n, const crk_item_req* reqs,
+                                     crk_item_req single, uint32_t use_single) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const crk_item_req r = use_single ? single : reqs[i];
+    Job job{};
+    uint64_t cnt = 0;
+    int st;
+    const uint32_t d = xid_lookup(ix, r.xid);
+    if (d == kNotFound) {
+      st = CRK_E_XID;
+    } else if ((st = ix.p_status[d]) == CRK_OK) {
+      const uint64_t b = (uint64_t)d * kMaxItems + r.arg_no;
+      const uint32_t es = elem_size_k(r.kind);
+      if (r.arg_no >= ix.p_nitems[d] || ix.p_kind[b] != r.kind || es == 0) {
+        st = CRK_E_ARG;
+      } else if (ix.p_count[b] > r.max_count) {
+        st = CRK_E_SIZE;
+      } else {
+        cnt = ix.p_count[b];
+        job = dec_job((uint64_t)r.dst, cnt * es, ix.p_off[b], d, es);
+      }
+    }
+    sc.jobs[i] = job;
+    *r.status = st;
+    if (r.count) *r.count = cnt;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+}
+
+// ---- serve: statuses, HtoD decode jobs and reply sizes (pass 1) --------------------------------
+__device__ __forceinline__ void reply_words(Piece& p, uint32_t xid, int32_t err, bool with_len, uint64_t n) {
+  p = Piece{};
+  p.type = PIECE_WORDS;
+  p.loff = 0;
+  p.words[0] = xid;  // RFC 5531 §9: xid, REPLY, MSG_ACCEPTED, verf AUTH_NONE (0, len 0), SUCCESS
+  p.words[1] = 1;
+  p.words[2] = 0;
+  p.words[3] = 0;
+  p.words[4] = 0;
+  p.words[5] = 0;
+  p.words[6] = (uint32_t)err;  // mem_result discriminant (reading R10)
+  if (with_len) p.words[7] = (uint32_t)n;
+  p.nbytes = with_len ? 32 : 28;
+}
+
+__global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint64_t region_base,
+                                   uint64_t region_bytes) {
+  const uint32_t total = *ix.total;
+  uint64_t* wire = sc.scan_tmp;  // reply wire sizes -> prefix
+  for (uint32_t d = blockIdx.x * blockDim.x + threadIdx.x; d < total; d += gridDim.x * blockDim.x) {
+    int st = ix.p_status[d];
+    const uint32_t proc = ix.p_proc[d];
+    int32_t err = -1;
+    uint64_t Ll = 0;
+    Job job{};
+    if (st == CRK_OK && xid_lookup(ix, ix.p_xid[d]) != d) st = CRK_E_XID;
+    const uint64_t b = (uint64_t)d * kMaxItems;
+    if (st == CRK_OK && proc == cfg.proc_h2d) {
+      const uint64_t ptr = ix.p_value[b], nb = ix.p_count[b + 1], size = ix.p_value[b + 2];
+      const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
+      if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
+      else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
+      else { err = 0; job = dec_job(ptr, m, ix.p_off[b + 1], d, 1); }
+      Ll = 28;
+    } else if (st == CRK_OK && proc == cfg.proc_d2h) {
+      const uint64_t ptr = ix.p_value[b], size = ix.p_value[b + 1];
+      if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
+        st = CRK_E_PTR; err = 1; Ll = 28;
+      } else {
+        err = 0; Ll = 32 + size + pad4(size);
+      }
+    }
+    ix.s_status[d] = st;
+    ix.s_reply_err[d] = err;
+    const uint64_t w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
+    ix.s_reply_wire[d] = w;
+    wire[d] = w;
+    sc.jobs[d] = job;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = 2 * total;
+}
+
+struct SendRingsParam {
+  uint32_t n_rings;
+  RingDesc r[kMaxRings];
+  uint64_t off[kMaxRings];
+};
+
+// pass 2: reply cursors (prefix of wire sizes within each ring) and the encode jobs
+__global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendRingsParam S) {
+  const uint32_t total = *ix.total;
+  const uint64_t* pre = sc.scan_tmp;
+  if (blockIdx.x == 0)
+    for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
+  for (uint32_t d = blockIdx.x * blockDim.x + threadIdx.x; d < total; d += gridDim.x * blockDim.x) {
+    const uint32_t ring = ix.p_ring[d];
+    const uint32_t first = ix.rec_prefix[ring], end = ix.rec_prefix[ring + 1];
+    const uint64_t w = ix.s_reply_wire[d];
+    const uint64_t off = S.off[ring] + (pre[d] - pre[first]);
+    ix.s_reply_off[d] = off;
+    const int32_t err = ix.s_reply_err[d];
+    Job job{};
+    if (err >= 0) {
+      const uint64_t b = (uint64_t)d * kMaxItems;
+      const bool d2h = ix.p_proc[d] == cfg.proc_d2h && err == 0;
+      const uint64_t n = d2h ? ix.p_value[b + 1] : 0;
+      Piece* P = sc.pieces + 2ull * d;
+      reply_words(P[0], ix.p_xid[d], err, d2h, n);
+      uint32_t np = 1;
+      uint64_t Ll = P[0].nbytes;
+      if (d2h) {
+        Piece q{};
+        q.type = PIECE_DATA;
+        q.loff = 32;
+        q.nbytes = n;
+        q.src = ix.p_value[b];
+        q.esize = 1;
+        P[1] = q;
+        np = 2;
+        Ll = 32 + n + pad4(n);
+      }
+      job.type = JOB_ENC;
+      job.out_start = off;
+      job.out_end = off + w;
+      job.loff = Ll;
+      job.piece0 = 2 * d;
+      job.n_pieces = np;
+      job.F = cfg.F;
+      job.out_ring = ring;
+    }
+    sc.jobs[total + d] = job;
+    if (d + 1 == end) ix.res[ring].reply_bytes = pre[d] + w - pre[first];
+  }
+}
+
+__global__ void put_enc_jobs_kernel(Scratch sc, EncJobParam p, RingDesc out) {
+  if (threadIdx.x == 0) {
+    for (uint32_t j = 0; j < p.n_jobs; ++j) sc.jobs[j] = p.jobs[j];
+    sc.out_rings[0] = out;
+    sc.counters[1] = p.n_jobs;
+  }
+  for (uint32_t i = threadIdx.x; i < p.n_pieces; i += blockDim.x) sc.pieces[i] = p.pieces[i];
+}
+
+__global__ void d2h_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uint64_t* bytes, const int32_t* errs) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t err = errs ? errs[i] : 0;
+    const uint64_t nb = err == 0 ? bytes[i] : 0;
+    const uint64_t Ll = err == 0 ? 32 + nb + pad4(nb) : 28;
+    sc.scan_tmp[i] = wire_of(Ll, cfg.F);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+}
+
+__global__ void d2h_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uint32_t* xids, const void* const* srcs,
+                                const uint64_t* bytes, const int32_t* errs, RingDesc out, uint64_t out_off,
+                                uint64_t* wire_offs, uint64_t* total_dev, const uint64_t* total_scan) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    sc.out_rings[0] = out;
+    if (total_dev) *total_dev = *total_scan;
+  }
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t err = errs ? errs[i] : 0;
+    const uint64_t nb = err == 0 ? bytes[i] : 0;
+    const uint64_t off = out_off + sc.scan_tmp[i];
+    Piece* P = sc.pieces + 2ull * i;
+    reply_words(P[0], xids[i], err, err == 0, nb);
+    uint32_t np = 1;
+    uint64_t Ll = P[0].nbytes;
+    if (err == 0) {
+      Piece q{};
+      q.type = PIECE_DATA;
+      q.loff = 32;
+      q.nbytes = nb;
+      q.src = (uint64_t)srcs[i];
+      q.esize = 1;
+      P[1] = q;
+      np = 2;
+      Ll = 32 + nb + pad4(nb);
+    }
+    Job job{};
+    job.type = JOB_ENC;
+    job.out_start = off;
+    job.out_end = off + wire_of(Ll, cfg.F);
+    job.loff = Ll;
+    job.piece0 = 2 * i;
+    job.n_pieces = np;
+    job.F = cfg.F;
+    job.out_ring = 0;
+    sc.jobs[i] = job;
+    if (wire_offs) wire_offs[i] = off;
+  }
+}
+
+__global__ void lens_prep_kernel(Scratch sc, const uint32_t* lens32, uint32_t n) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    sc.lens_pool[i] = lens32[i];
+    sc.lens_pool[sc.max_lens + i] = (uint64_t)lens32[i] + 4;  // -> wire starts after the scan
+  }
+}
+
+inline uint32_t blocks_for(uint32_t n, uint32_t per = 256, uint32_t cap = 148 * 16) {
+  uint32_t b = (n + per - 1) / per;
+  return b == 0 ? 1 : (b > cap ? cap : b);
+}
+
+}  // namespace
+
+cudaError_t launch_resolve_h2d(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n, const uint32_t* xids,
+                               void* const* dsts, const uint64_t* dst_bytes, int32_t* statuses, uint64_t* copied,
+                               const H2DReq* single, cudaStream_t s) {
+  H2DReq one{};
+  if (single) one = *single;
+  resolve_h2d_kernel<<<blocks_for(n), 256, 0, s>>>(ix, cfg, sc, n, xids, dsts, dst_bytes, statuses, copied, one,
+                                                    single ? 1u : 0u);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n,
+                                 const crk_item_req* reqs, const crk_item_req* single, cudaStream_t s) {
+  crk_item_req one{};
+  if (single) one = *single;
+  resolve_items_kernel<<<blocks_for(n), 256, 0, s>>>(ix, cfg, sc, n, reqs, one, single ? 1u : 0u);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
+                              const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
+                              uint64_t region_bytes, cudaStream_t s) {
+  const uint32_t bound = ix.max_records;
+  serve_plan1_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, region_base, region_bytes);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  e = launch_exclusive_scan_u64(sc.scan_tmp, bound, ix.total, nullptr, sc, s);
+  if (e != cudaSuccess) return e;
+  SendRingsParam S{};
+  S.n_rings = n_rings;
+  for (uint32_t r = 0; r < n_rings; ++r) {
+    S.r[r].base = send_rings[r].base;
+    S.r[r].mask = send_rings[r].cap - 1;
+    S.r[r].head = S.r[r].tail = 0;
+    S.off[r] = send_offs[r];
+  }
+  serve_plan2_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, S);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_put_enc_jobs(Scratch& sc, const EncJobParam& p, const RingDesc& out, cudaStream_t s) {
+  put_enc_jobs_kernel<<<1, 64, 0, s>>>(sc, p, out);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const uint32_t* xids,
+                                  const void* const* srcs, const uint64_t* bytes, const int32_t* errs,
+                                  const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
+                                  cudaStream_t s) {
+  d2h_sizes_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, bytes, errs);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
+  e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
+  if (e != cudaSuccess) return e;
+  d2h_jobs_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
+                                                 tot);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n, cudaStream_t s) {
+  lens_prep_kernel<<<blocks_for(n), 256, 0, s>>>(sc, lens32_dev, n);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  return launch_exclusive_scan_u64(sc.lens_pool + sc.max_lens, n, nullptr, nullptr, sc, s);
+}
+
+}  // namespace crk

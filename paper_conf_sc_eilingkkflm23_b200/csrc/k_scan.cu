@@ -1,0 +1,174 @@
+// K1 + K2 (fragment part): speculative record-marking scan (RFC 5531 §11) with the segmented prefix
+// sum of fragment lengths that gives every fragment its logical start.
+//
+// The header chain is sequential (p[k+1] = p[k] + 4 + len[k]).  One CTA per ring walks it in rounds:
+// from a known true header at p, thread t reads the candidate header at p + t * (4 + len(h_pred)),
+// where h_pred is the predicted header value.  If headers 0..t-1 all equal h_pred their positions are
+// exact, so candidate t is a true header (induction); the first t* whose value differs is still a true
+// header.  A round therefore accepts t* + 1 headers with one memory latency, and 1024 at a time when
+// the sender frames regularly (greedy F-byte fragments, or back-to-back identical records).  Because
+// headers 0..t*-1 are identical, the fragment lengths' segmented prefix sums (logical starts) and the
+// record boundaries have closed forms in t; the checks are then the oracle's, in its order
+// (oracle/oracle.c or_frame_scan; DESIGN.md §4 readings R1, R2, R8):
+//   E_FRAG (sum > max_record_bytes)  ->  INCOMPLETE (data past tail)  ->  index capacity.
+#include "crk_device.cuh"
+
+namespace crk {
+
+namespace {
+
+enum : uint32_t { STOP_NONE = 0, STOP_FRAG = 1, STOP_INCOMPLETE = 2, STOP_CAP = 3 };
+
+struct ScanState {
+  uint64_t p, r0, sum;
+  uint32_t f0, nf, nr, hpred;
+  uint32_t done;
+  int32_t status;
+  uint64_t consumed;
+  uint32_t kept_frags;
+  uint32_t tstar, valid_star, h_star;
+  uint32_t tf, code_f;
+};
+
+__global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
+  const uint32_t ring = blockIdx.x;
+  const RingDesc R = P.r[ring];
+  const uint32_t t = threadIdx.x, T = blockDim.x;
+  const uint32_t FC = ix.frags_per_ring, RC = ix.recs_per_ring;
+  const uint64_t fbase = (uint64_t)ring * FC, rbase = (uint64_t)ring * RC;
+  __shared__ ScanState S;
+  __shared__ uint32_t red[32];
+  if (t == 0) {
+    ix.rings[ring] = R;
+    S.p = S.r0 = R.head;
+    S.sum = 0;
+    S.f0 = S.nf = S.nr = 0;
+    S.hpred = cfg.guess & 0x7fffffffu;
+    S.done = 0;
+  }
+  __syncthreads();
+  while (!S.done) {
+    const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
+    const uint32_t hpred = S.hpred, nf = S.nf, nr = S.nr, f0 = S.f0;
+    const uint64_t Lp = hpred & 0x7fffffffu;
+    const uint32_t lastp = hpred >> 31;
+    const uint64_t stride = 4 + Lp;
+    const uint64_t q = p + (uint64_t)t * stride;
+    const bool valid = q + 4 <= R.tail;
+    const uint32_t h = valid ? ring_be32(R, q) : 0u;
+    const bool ok = valid && h == hpred;
+    const uint32_t tstar = block_min_u32(ok ? T : t, red);
+    if (t == tstar) { S.valid_star = valid; S.h_star = h; }
+    __syncthreads();
+    const bool end_at_star = tstar < T && !S.valid_star;
+    const uint32_t n_hdr = tstar == T ? T : (end_at_star ? tstar : tstar + 1);
+    const uint32_t hstar = S.h_star;
+
+    // per-header closed forms (headers 0..tstar-1 equal hpred)
+    const bool is_hdr = t < n_hdr;
+    const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
+    const uint32_t last = (t < tstar) ? lastp : (hstar >> 31);
+    const bool start = (t == 0) ? (p == r0) : (lastp != 0);
+    // logical end of header t within its record (segmented inclusive prefix sum of lengths)
+    uint64_t send;
+    if (!lastp) send = sum + (uint64_t)t * Lp + len;
+    else send = (t == 0) ? (start ? len : sum + len) : len;
+    const uint32_t nrec = lastp ? nr + t : nr;  // completed records before header t
+
+    uint32_t code = STOP_NONE;
+    if (is_hdr) {
+      if (send > cfg.max_record_bytes) code = STOP_FRAG;
+      else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
+      else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
+    }
+    const uint32_t tf = block_min_u32(code != STOP_NONE ? t : 0xffffffffu, red);
+    if (t == tf) S.code_f = code;
+    __syncthreads();
+    const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
+
+    // emit fragments (and the records they complete)
+    if (t < n_emit) {
+      const uint64_t fs = fbase + nf + t;
+      ix.frag_phys[fs] = q + 4;
+      ix.frag_lstart[fs] = send - len;
+      ix.frag_hdr[fs] = (uint32_t)len | (last << 31);
+      if (last) {
+        const uint64_t rs = rbase + nrec;
+        ix.rec_begin[rs] = start ? q : r0;
+        ix.rec_len[rs] = send;
+        ix.rec_frag0[rs] = (uint32_t)(fbase + (start ? nf + t : f0));
+        ix.rec_nfrags[rs] = start ? 1u : nf + t - f0 + 1;
+      }
+    }
+    // the stopping thread (failure at tf, or no readable header at tstar) records the outcome
+    const bool stops_here = (tf < n_hdr) ? (t == tf) : (end_at_star && t == tstar);
+    if (stops_here) {
+      const uint64_t rstart = start ? q : r0;
+      S.consumed = rstart;
+      S.kept_frags = start ? nf + t : f0;
+      S.nr = nrec;
+      if (tf < n_hdr) {
+        const uint32_t c = S.code_f;
+        S.status = c == STOP_FRAG ? CRK_E_FRAG
+                 : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
+                 : (nrec > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
+      } else {
+        S.status = (start && q == R.tail) ? CRK_OK : CRK_INCOMPLETE;
+      }
+      S.done = 1;
+    }
+    // the last accepted header advances the state
+    if (!stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
+      S.p = q + 4 + len;
+      S.nf = nf + n_hdr;
+      if (last) {
+        S.nr = nrec + 1;
+        S.r0 = q + 4 + len;
+        S.sum = 0;
+        S.f0 = nf + n_hdr;
+      } else {
+        S.nr = nrec;
+        S.sum = send;
+        S.r0 = start ? q : r0;
+        S.f0 = start ? nf + t : f0;
+      }
+      // keep a fruitful prediction; switch to the observed header when the round made no progress
+      if (tstar < T && tstar == 0) S.hpred = hstar;
+    }
+    __syncthreads();
+  }
+  if (t == 0) {
+    crk_ring_result& rr = ix.res[ring];
+    rr.status = S.status;
+    rr.n_records = S.nr;
+    rr.n_frags = S.kept_frags;
+    rr.consumed = S.consumed;
+    rr.reply_bytes = 0;
+    __threadfence();
+    const uint32_t done = atomicAdd(ix.ticket, 1u);
+    if (done == gridDim.x - 1) {
+      // last ring: dense record numbering = exclusive prefix over rings
+      __threadfence();
+      uint32_t acc = 0;
+      for (uint32_t r = 0; r < gridDim.x; ++r) {
+        volatile crk_ring_result* vr = ix.res + r;
+        ix.rec_prefix[r] = acc;
+        vr->rec_base = acc;
+        acc += vr->n_records;
+      }
+      ix.rec_prefix[gridDim.x] = acc;
+      *ix.total = acc;
+      *ix.ticket = 0;
+    }
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s) {
+  frame_scan_kernel<<<p.n_rings, kScanThreads, 0, s>>>(ix, p, cfg);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace crk
