@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""Benchmark: XDR memcpy decode/encode GB/s per GPU (and aggregate over N GPUs) vs the binding roofline.
+
+Workload (BASELINE.json configs[4], the per-GPU slice of the metric's 8-GPU aggregate): one Cricket
+server endpoint per GPU serving 16 client streams, each a ring of ONC RPC memcpy CALL records (sizes
+log-uniform 4 KiB-16 MiB, 50/50 HtoD/DtoH, 64 MiB of payload per stream = 1 GiB per GPU), fragments of
+64 KiB.  One step = crk_serve over all 16 rings: record-marking scan (K1), prefix
+sums (K2), CALL parse (K3), HtoD opaque scatter into device memory (K4) and DtoH reply encode into the
+send rings (K6), i.e. every §8(a) row the memcpy path has.
+
+  value : payload GB/s (1e9 B/s) with rings and send rings resident in HBM (inputs > L2: 1 GiB of rings)
+  e2e   : the same through the C ABI with the rings in pinned host memory (zero-copy over PCIe: the
+          kernels read the CALLs from host memory and write the replies to host memory) plus a
+          device->host read of the per-ring results every step
+  roofline: the mover kernel (K4/K6) against the measured HBM copy bandwidth
+  cpu_baseline: the oracle (oracle/, plain C, one core) on a bounded sample of the same workload
+
+Launch: python bench.py [--gpus N --steps K --warmup W]; N > 1 under torch.distributed.run (one rank per
+GPU, NCCL only for the barrier and the max-over-ranks of the timings; the data path has no collective).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+MiB = 1 << 20
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=200)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="crk", choices=["crk", "reference"])
+    p.add_argument("--streams", type=int, default=16)
+    p.add_argument("--payload-mib", type=int, default=64, help="payload per stream")
+    p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=10.0)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------ clocks during the timed region
+
+class ClockSampler:
+    """NVML sampling of SM clocks and throttle reasons on a background thread."""
+
+    def __init__(self, index: int, period_s: float = 0.002):
+        self.index, self.period, self.samples, self.reasons = index, period_s, [], set()
+        self._stop = threading.Event()
+        self.max_mhz = None
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            self.N = N
+            self.h = N.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = N.nvmlDeviceGetMaxClockInfo(self.h, N.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover
+            self.N = None
+            self.err = repr(e)
+
+    def _run(self):
+        N = self.N
+        names = {getattr(N, k, None): k for k in (
+            "nvmlClocksEventReasonHwSlowdown", "nvmlClocksEventReasonHwThermalSlowdown",
+            "nvmlClocksEventReasonSwThermalSlowdown", "nvmlClocksEventReasonSwPowerCap",
+            "nvmlClocksEventReasonHwPowerBrakeSlowdown")}
+        label = {"nvmlClocksEventReasonHwSlowdown": "hw_slowdown",
+                 "nvmlClocksEventReasonHwThermalSlowdown": "hw_thermal_slowdown",
+                 "nvmlClocksEventReasonSwThermalSlowdown": "sw_thermal_slowdown",
+                 "nvmlClocksEventReasonSwPowerCap": "sw_power_cap",
+                 "nvmlClocksEventReasonHwPowerBrakeSlowdown": "hw_power_brake"}
+        while not self._stop.is_set():
+            try:
+                self.samples.append(N.nvmlDeviceGetClockInfo(self.h, N.NVML_CLOCK_SM))
+                r = N.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, k in names.items():
+                    if bit and r & bit:
+                        self.reasons.add(label[k])
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.N:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.N:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.N:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ CPU baseline (oracle)
+
+def oracle_sample(n_streams: int, payload_mib: int, rank: int = 0):
+    """Oracle-encoded rings for the first streams of endpoint `rank` (a bounded sample of the workload)."""
+    import numpy as np
+    import oracle as O
+    from paper_conf_sc_eilingkkflm23_b200 import gen
+    streams, _ = gen.c5_endpoint(rank, n_streams=16, payload_per_stream=payload_mib * MiB,
+                                 h2d_budget=payload_mib * MiB - payload_mib * MiB // 16)
+    cfg = O.Config(prog=gen.PROG, vers=gen.VERS, proc_h2d=gen.PROC_H2D, proc_d2h=gen.PROC_D2H, frag_payload=65536)
+    base = 0x7F0000000000
+    sample = streams[:n_streams]
+    top = max(r.region_off + r.size for s in sample for r in s.records)
+    region = np.zeros(top + 256, np.uint8)
+    rings, payload = [], 0
+    for s in sample:
+        wires = []
+        for r in s.records:
+            d = gen.random_bytes(r.seed & 0xFFFFFFFF, r.size)
+            payload += r.size
+            if r.kind == gen.PROC_H2D:
+                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + r.region_off), (O.K_OPAQUE_VAR, d),
+                                                           (O.K_U64, r.size)], cfg))
+            else:
+                region[r.region_off:r.region_off + r.size] = d
+                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + r.region_off), (O.K_U64, r.size)], cfg))
+        w = b"".join(wires)
+        cap = 1 << max(8, len(w).bit_length())
+        ring = np.zeros(cap, np.uint8)
+        ring[:len(w)] = np.frombuffer(w, np.uint8)
+        rings.append((ring, 0, len(w)))
+    send_caps = [1 << 28] * len(rings)
+
+    def step():
+        out = O.serve(rings, cfg, region, base, send_caps, [0] * len(rings), max_frags_per_ring=1 << 16,
+                      max_records_per_ring=1 << 12)
+        assert all(s == O.OK for s in out["scan_status"])
+        return out
+
+    return step, payload
+
+
+def cpu_baseline(args, seconds: float):
+    n_streams = 2
+    step, payload = oracle_sample(n_streams, args.payload_mib)
+    step()  # warm (page-in)
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        step()
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            break
+    return {"value": round(payload * reps / el / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"oracle or_serve (plain C, 1 thread) over streams 0-{n_streams - 1} of endpoint 0 "
+                      f"({payload / MiB:.0f} MiB payload) x{reps} reps, {el:.1f} s"}
+
+
+def run_reference(args):
+    """--impl reference: the oracle timed as the reference arm (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n_streams = 2
+    step, payload = oracle_sample(n_streams, args.payload_mib)
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    el = time.perf_counter() - t0
+    v = payload * args.steps / el / 1e9
+    sample = (f"oracle or_serve (plain C, 1 thread) over streams 0-{n_streams - 1} of endpoint 0 "
+              f"({payload / MiB:.0f} MiB payload per step)")
+    print(json.dumps({
+        "impl": "reference", "metric": "xdr_memcpy_serve_payload_GBps", "value": round(v, 4), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(el / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": workload_config(args), "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1,
+                                                           "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
+
+
+def workload_config(args):
+    return {"workload": f"C5 endpoint per GPU: {args.streams} client streams x {args.payload_mib} MiB memcpy payload "
+                        f"(ONC RPC CALLs, sizes log-uniform 4 KiB-16 MiB, 50/50 HtoD/DtoH, F=64 KiB fragments)",
+            "streams_per_gpu": args.streams, "payload_per_gpu_bytes": args.streams * args.payload_mib * MiB,
+            "frag_payload": 65536, "l2": "inputs larger than L2 (rings + region > 2 GiB per GPU)",
+            "parallelism": f"{args.gpus} independent endpoints, no collective"}
+
+
+# ------------------------------------------------------------------ main
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_eilingkkflm23_b200 import build, crk, workload
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    build.build()
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    ctx = crk.Context(local)
+    ep = workload.c5_endpoint(ctx, rank, dev, n_streams=args.streams, payload_per_stream=args.payload_mib * MiB)
+    idx = ctx.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
+    stream = torch.cuda.current_stream(dev)
+
+    # ---- device-resident timed region (value)
+    for _ in range(args.warmup):
+        workload.serve_step(idx, ep)
+    barrier()
+    check = workload.check_results(idx, ep)
+    crk.profile_enable(True)
+    l0 = crk.kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            workload.serve_step(idx, ep)
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = crk.kernel_launches() - l0
+    prof = crk.profile_read()
+    crk.profile_enable(False)
+    ms = e0.elapsed_time(e1) / args.steps
+    ms_max = max_over_ranks(ms)
+    payload_all = sum_over_ranks(ep.payload)
+    value = payload_all / (ms_max / 1e3) / 1e9
+
+    # roofline of the dominant kernel (the mover): algorithmic HBM bytes per launch / its event time
+    mv_ms, mv_n = prof["move"]
+    alg_bytes = 2 * ep.h2d_payload + ep.d2h_payload + ep.reply_wire  # read+write per HtoD byte; DtoH read + reply
+    mv_launch_ms = mv_ms / max(1, mv_n)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    achieved = alg_bytes / (mv_launch_ms / 1e3) / 1e9
+    traffic = None
+    try:
+        traffic = json.load(open(os.path.join(ROOT, "profiles", "mover_ncu.json")))["dram_bytes_per_launch"]
+    except Exception:
+        pass
+    stage_share = {k: round(v[0] / max(1e-9, sum(x[0] for x in prof.values())), 4) for k, v in prof.items()}
+
+    # ---- end to end through the C ABI with host (pinned, mapped) rings
+    e2e = None
+    if not args.no_e2e:
+        del idx
+        torch.cuda.empty_cache()
+        ep_h = workload.c5_endpoint(ctx, rank, dev, n_streams=args.streams, payload_per_stream=args.payload_mib * MiB,
+                                    host_rings=True)
+        idx_h = ctx.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
+        for _ in range(min(2, args.warmup)):
+            workload.serve_step(idx_h, ep_h)
+            idx_h.ring_results(len(ep_h.rings))
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            workload.serve_step(idx_h, ep_h)
+            res = idx_h.ring_results(len(ep_h.rings))  # device -> host read of the step's result (syncs)
+        el = time.perf_counter() - t0
+        el_max = max_over_ranks(el)
+        check_h = workload.check_results(idx_h, ep_h)
+        res_bytes = len(ep_h.rings) * 40
+        e2e_v = sum_over_ranks(ep_h.payload) * args.e2e_steps / el_max / 1e9
+        # live host-link peaks (copy engine, pinned) for the e2e roofline
+        link = host_link_peaks(dev)
+        t_link = max(ep_h.wire_in / link["ce_h2d_gbs"], ep_h.reply_wire / link["ce_d2h_gbs"],
+                     (ep_h.wire_in + ep_h.reply_wire) / link["ce_bidir_gbs"]) / 1e9
+        step_s = el_max / args.e2e_steps
+        e2e = {"value": round(e2e_v, 3), "unit": "GB/s", "h2d_bytes_per_step": ep_h.wire_in,
+               "d2h_bytes_per_step": ep_h.reply_wire + res_bytes, "ms_per_step": round(step_s * 1e3, 3),
+               "mode": "zero-copy: kernels read CALL rings from and write reply rings to pinned host memory",
+               "wire_gbs": round((ep_h.wire_in + ep_h.reply_wire) / step_s / 1e9, 3),
+               "host_link": {**link, "bound_ms": round(t_link * 1e3, 3), "frac": round(t_link / step_s, 4)},
+               "check": check_h}
+
+    out = {
+        "metric": "xdr_memcpy_serve_payload_GBps", "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic (seeded gen.c5_endpoint; CALLs encoded on the GPU by crk_rpc_encode_call)",
+        "config": workload_config(args),
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak, "unit": "GB/s",
+                     "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
+                     "kernel": "crk mover_kernel (K4 opaque scatter + K6 reply encode)",
+                     "alg_bytes_per_launch": alg_bytes, "launch_ms": round(mv_launch_ms, 4),
+                     "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, read+write)"},
+        "stages_ms_per_step": {k: round(v[0] / max(1, v[1]), 4) for k, v in prof.items()},
+        "stage_share": stage_share,
+        "payload_bytes_per_gpu": ep.payload, "wire_in_bytes_per_gpu": ep.wire_in,
+        "reply_bytes_per_gpu": ep.reply_wire, "records_per_gpu": ep.n_records,
+        "gpu_launches": launches, "check": check,
+        "clocks": clk.summary(),
+        "e2e": e2e,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu:
+        out["cpu_baseline"] = cpu_baseline(args, args.cpu_seconds)
+    if rank == 0:
+        print(json.dumps(out))
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def host_link_peaks(dev, nbytes: int = 512 * MiB) -> dict:
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    h2 = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+
+    def best(fn, bytes_):
+        ts = []
+        for _ in range(4):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            fn()
+            torch.cuda.synchronize()
+            ts.append(time.perf_counter() - t0)
+        return bytes_ / min(ts[1:]) / 1e9
+
+    def bi():
+        with torch.cuda.stream(s1):
+            d.copy_(h, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+
+    r = {"ce_h2d_gbs": round(best(lambda: d.copy_(h, non_blocking=True), nbytes), 2),
+         "ce_d2h_gbs": round(best(lambda: h2.copy_(d2, non_blocking=True), nbytes), 2),
+         "ce_bidir_gbs": round(best(bi, 2 * nbytes), 2)}
+    del h, h2, d, d2
+    return r
+
+
+if __name__ == "__main__":
+    main()

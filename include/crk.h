@@ -280,6 +280,14 @@ int crk_host_alloc(uint64_t bytes, void** out);
 void crk_host_free(void* p);
 int crk_copy_to_host(void* host_dst, const void* dev_src, uint64_t bytes);
 
+/* ---------------------------------------------------------------- profiling
+ * When enabled, CUDA events are recorded on the launching stream around each pipeline stage:
+ * 0 = frame scan (K1), 1 = CALL parse (K3), 2 = serve planning (statuses, K2 reply offsets, jobs),
+ * 3 = the bulk mover (K4-K7).  crk_profile_read waits for the events, returns the summed device time
+ * (ms[4]) and the number of timed launches (launches[4]) since the last read, and resets them. */
+int crk_profile_enable(int on);
+int crk_profile_read(double* ms, uint32_t* launches);
+
 /* ---------------------------------------------------------------- misc */
 const char* crk_strerror(int status);
 int crk_last_cuda_error(void);   /* cudaError_t of the last CRK_E_CUDA */

@@ -112,6 +112,8 @@ def lib():
             "crk_strerror": (C.c_char_p, [C.c_int]),
             "crk_last_cuda_error": (C.c_int, []),
             "crk_kernel_launches": (C.c_int, []),
+            "crk_profile_enable": (C.c_int, [C.c_int]),
+            "crk_profile_read": (C.c_int, [C.POINTER(C.c_double), C.POINTER(u32)]),
             "crk_version": (C.c_char_p, []),
         }
         for t in ("i32", "u32", "i64", "u64", "f32", "f64"):
@@ -131,6 +133,21 @@ def strerror(status: int) -> str:
 
 def kernel_launches() -> int:
     return int(lib().crk_kernel_launches())
+
+
+PROF_STAGES = ("scan", "parse", "plan", "move")
+
+
+def profile_enable(on: bool = True):
+    _check(lib().crk_profile_enable(int(on)), "crk_profile_enable")
+
+
+def profile_read() -> dict:
+    """{stage: (device ms summed over timed launches, launches)} since the last read."""
+    ms = (C.c_double * 4)()
+    n = (u32 * 4)()
+    _check(lib().crk_profile_read(ms, n), "crk_profile_read")
+    return {s: (ms[i], n[i]) for i, s in enumerate(PROF_STAGES)}
 
 
 def _check(st: int, what: str):

@@ -33,6 +33,22 @@ struct crk_index {
 namespace crk {
 static std::atomic<int> g_launches{0};
 void count_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+// Stage timing with CUDA events recorded on the launching stream (crk_profile_*).
+constexpr uint32_t kProfCap = 2048;
+struct ProfState {
+  bool on = false, created = false;
+  cudaEvent_t ev[PROF_STAGES][2][kProfCap];
+  uint32_t n[PROF_STAGES] = {0, 0, 0, 0};
+};
+static ProfState g_prof;
+void prof_mark(int stage, bool begin, cudaStream_t s) {
+  if (!g_prof.on) return;
+  const uint32_t i = g_prof.n[stage];
+  if (i >= kProfCap) return;
+  cudaEventRecord(g_prof.ev[stage][begin ? 0 : 1][i], s);
+  if (!begin) g_prof.n[stage] = i + 1;
+}
 }  // namespace crk
 
 static thread_local int g_last_cuda = 0;
@@ -658,6 +674,35 @@ const char* crk_strerror(int st) {
     default: return "unknown status";
   }
 }
+int crk_profile_enable(int on) {
+  if (on && !g_prof.created) {
+    for (int s = 0; s < PROF_STAGES; ++s)
+      for (int b = 0; b < 2; ++b)
+        for (uint32_t i = 0; i < kProfCap; ++i) CK(cudaEventCreate(&g_prof.ev[s][b][i]));
+    g_prof.created = true;
+  }
+  g_prof.on = on != 0;
+  for (int s = 0; s < PROF_STAGES; ++s) g_prof.n[s] = 0;
+  return CRK_OK;
+}
+
+int crk_profile_read(double* ms, uint32_t* launches) {
+  if (!ms || !launches) return CRK_E_ARG;
+  for (int s = 0; s < PROF_STAGES; ++s) {
+    double acc = 0;
+    for (uint32_t i = 0; i < g_prof.n[s]; ++i) {
+      float t = 0;
+      CK(cudaEventSynchronize(g_prof.ev[s][1][i]));
+      CK(cudaEventElapsedTime(&t, g_prof.ev[s][0][i], g_prof.ev[s][1][i]));
+      acc += t;
+    }
+    ms[s] = acc;
+    launches[s] = g_prof.n[s];
+    g_prof.n[s] = 0;
+  }
+  return CRK_OK;
+}
+
 int crk_last_cuda_error(void) { return g_last_cuda; }
 int crk_kernel_launches(void) { return crk::g_launches.load(); }
 const char* crk_version(void) { return "crk 0.1 (sm_100a)"; }

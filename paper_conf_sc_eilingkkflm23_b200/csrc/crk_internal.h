@@ -163,4 +163,8 @@ int mover_occupancy();
 // host-visible counter of our kernel launches
 void count_launch(int n = 1);
 
+// optional CUDA-event timing of the pipeline stages (crk_profile_*)
+enum { PROF_SCAN = 0, PROF_PARSE = 1, PROF_PLAN = 2, PROF_MOVE = 3, PROF_STAGES = 4 };
+void prof_mark(int stage, bool begin, cudaStream_t s);
+
 }  // namespace crk

@@ -359,8 +359,10 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   M.prefix = tiles;
   M.n_jobs_dev = n_jobs_dev;
   M.total_tiles = total;
+  prof_mark(PROF_MOVE, true, s);
   mover_kernel<<<move_ctas, kMoveThreads, 0, s>>>(M);
   count_launch();
+  prof_mark(PROF_MOVE, false, s);
   return cudaGetLastError();
 }
 

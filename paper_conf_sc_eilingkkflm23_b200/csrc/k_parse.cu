@@ -160,8 +160,10 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
 
 cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const ConfigDev& cfg, uint32_t n_rings,
                          int sms, cudaStream_t s) {
+  prof_mark(PROF_PARSE, true, s);
   parse_kernel<<<sms * 4, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
   count_launch();
+  prof_mark(PROF_PARSE, false, s);
   return cudaGetLastError();
 }
 

@@ -319,6 +319,7 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
                               const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
                               uint64_t region_bytes, cudaStream_t s) {
   const uint32_t bound = ix.max_records;
+  prof_mark(PROF_PLAN, true, s);
   serve_plan1_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, region_base, region_bytes);
   count_launch();
   cudaError_t e = cudaGetLastError();
@@ -335,6 +336,7 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
   }
   serve_plan2_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, S);
   count_launch();
+  prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();
 }
 

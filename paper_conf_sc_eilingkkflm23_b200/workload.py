@@ -1,0 +1,122 @@
+"""Builds the benchmark workloads on the GPU with the library's own encoder (no oracle involved).
+
+C5 endpoint (BASELINE.json configs[4], one per GPU): 16 client streams, each a ring of memcpy CALL
+records (sizes log-uniform 4 KiB-16 MiB, 50/50 HtoD/DtoH, 64 MiB of payload per stream, 1 GiB per GPU),
+framed with F = 64 KiB fragments.  The HtoD payloads and the DtoH source bytes come
+from gen's seeded streams; the CALL records are encoded into the rings by crk_rpc_encode_call (the
+client side of the same codec).  Ring filling is setup, outside every timed region.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import numpy as np
+import torch
+
+from . import crk, gen
+
+MiB = 1 << 20
+
+
+def next_pow2(x: int) -> int:
+    return 1 << max(8, (max(1, x) - 1).bit_length())
+
+
+@dataclass
+class Endpoint:
+    ctx: crk.Context
+    rank: int
+    streams: list
+    region: torch.Tensor
+    rings: list = field(default_factory=list)       # (Ring, head, tail)
+    sends: list = field(default_factory=list)       # Ring
+    offs: list = field(default_factory=list)
+    h2d_payload: int = 0
+    d2h_payload: int = 0
+    wire_in: int = 0
+    reply_wire: int = 0
+    n_records: int = 0
+    per_stream_reply: list = field(default_factory=list)
+    per_stream_records: list = field(default_factory=list)
+
+    @property
+    def base(self) -> int:
+        return self.region.data_ptr()
+
+    @property
+    def payload(self) -> int:
+        return self.h2d_payload + self.d2h_payload
+
+
+def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: int = 16,
+                payload_per_stream: int = 64 * MiB, host_rings: bool = False, misalign: bool = False) -> Endpoint:
+    streams, region_bytes = gen.c5_endpoint(rank, n_streams=n_streams, payload_per_stream=payload_per_stream,
+                                            h2d_budget=payload_per_stream - payload_per_stream // 16,
+                                            misalign=misalign)
+    region = torch.zeros(region_bytes + 256, dtype=torch.uint8, device=device)
+    ep = Endpoint(ctx, rank, streams, region)
+    F = ctx.cfg.frag_payload
+    for s in streams:
+        # wire size of every record from the library's closed forms, to size the rings
+        h2d = [r for r in s.records if r.kind == gen.PROC_H2D]
+        d2h = [r for r in s.records if r.kind == gen.PROC_D2H]
+        stage_cap = max([r.size for r in h2d] + [1])
+        stage = torch.empty(stage_cap + 16, dtype=torch.uint8, device=device)
+        ring_dev = crk.Ring.device(next_pow2(sum(r.size + 64 + 4 * (r.size // F + 2) for r in h2d) + 64 * len(d2h)
+                                             + 4096), device)
+        cur = 0
+        for r in s.records:
+            data = torch.from_numpy(gen.random_bytes(r.seed & 0xFFFFFFFF, r.size)).to(device)
+            if r.kind == gen.PROC_H2D:
+                stage[:r.size].copy_(data)
+                items = [(crk.K_U64, ep.base + r.region_off), (crk.K_OPAQUE_VAR, stage[:r.size]),
+                         (crk.K_U64, r.size)]
+                ep.h2d_payload += r.size
+            else:
+                ep.region[r.region_off:r.region_off + r.size].copy_(data)
+                items = [(crk.K_U64, ep.base + r.region_off), (crk.K_U64, r.size)]
+                ep.d2h_payload += r.size
+            cur += ctx.encode_call(r.xid, r.kind, items, ring_dev, cur)
+            torch.cuda.synchronize(device)
+        reply = sum(crk.wire_size_d2h(r.size, 0, F) for r in d2h) + sum(crk.wire_size_d2h(0, 1, F) for _ in h2d)
+        if host_rings:
+            ring = crk.Ring.host(ring_dev.cap)
+            torch.cuda.synchronize(device)
+            host = torch.from_numpy(ring.host_view())
+            host[:cur].copy_(ring_dev.tensor()[:cur].cpu())
+            send = crk.Ring.host(next_pow2(reply + 4096))
+            del ring_dev
+        else:
+            ring = ring_dev
+            send = crk.Ring.device(next_pow2(reply + 4096), device)
+        ep.rings.append((ring, 0, cur))
+        ep.sends.append(send)
+        ep.offs.append(0)
+        ep.wire_in += cur
+        ep.reply_wire += reply
+        ep.n_records += len(s.records)
+        ep.per_stream_reply.append(reply)
+        ep.per_stream_records.append(len(s.records))
+        del stage
+    torch.cuda.synchronize(device)
+    return ep
+
+
+def serve_step(idx: crk.Index, ep: Endpoint, stream=None):
+    idx.serve(ep.rings, ep.sends, ep.offs, ep.base, ep.region.numel(), stream=stream)
+
+
+def check_results(idx: crk.Index, ep: Endpoint) -> dict:
+    """Cheap end-of-run sanity on the device results: every ring consumed, every record OK, reply bytes
+    as the closed forms predict, and a sample of HtoD destinations equal to the generator's payload."""
+    res = idx.ring_results(len(ep.rings))
+    ok = all(r["status"] == crk.OK and r["consumed"] == t for r, (_, _, t) in zip(res, ep.rings))
+    ok &= all(r["n_records"] == n for r, n in zip(res, ep.per_stream_records))
+    ok &= all(r["reply_bytes"] == w for r, w in zip(res, ep.per_stream_reply))
+    sampled = 0
+    for s in ep.streams[:2]:
+        for r in [x for x in s.records if x.kind == gen.PROC_H2D][:3]:
+            want = torch.from_numpy(gen.random_bytes(r.seed & 0xFFFFFFFF, r.size)).to(ep.region.device)
+            ok &= bool(torch.equal(ep.region[r.region_off:r.region_off + r.size], want))
+            sampled += 1
+    return dict(ok=bool(ok), sampled_h2d_records=sampled)
