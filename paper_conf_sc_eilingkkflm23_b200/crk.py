@@ -14,7 +14,7 @@ import numpy as np
 import torch
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIBPATH = os.path.join(PKG, "lib", "libcrk.so")
+LIBPATH = os.environ.get("CRK_LIB") or os.path.join(PKG, "lib", "libcrk.so")
 
 OK, INCOMPLETE = 0, 1
 E_ARG, E_TRUNCATED, E_FRAG, E_RPC, E_AUTH, E_PAD, E_SIZE = -1, -2, -3, -4, -5, -6, -7
@@ -43,7 +43,8 @@ class Config(C.Structure):
     _fields_ = [("frag_payload", C.c_uint32), ("strict", C.c_int32), ("max_record_bytes", C.c_uint64),
                 ("prog", C.c_uint32), ("vers", C.c_uint32), ("proc_h2d", C.c_uint32), ("proc_d2h", C.c_uint32),
                 ("scan_stride_guess", C.c_uint32), ("tile_bytes", C.c_uint32), ("max_jobs", C.c_uint32),
-                ("ctas_per_sm", C.c_uint32)]
+                ("ctas_per_sm", C.c_uint32), ("scan_threads", C.c_uint32), ("mover_stages", C.c_uint32),
+                ("mover_run", C.c_uint32)]
 
 
 class CRing(C.Structure):

@@ -222,6 +222,9 @@ void crk_config_init(crk_config* c) {
   c->tile_bytes = 32768;
   c->max_jobs = 1u << 20;
   c->ctas_per_sm = 0;
+  c->scan_threads = 128;
+  c->mover_stages = 3;
+  c->mover_run = 8;
 }
 
 int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
@@ -230,7 +233,9 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   crk_config cfg;
   if (cfg_in) cfg = *cfg_in; else crk_config_init(&cfg);
   if (cfg.frag_payload == 0 || cfg.frag_payload > 0x7fffffffu || !pow2(cfg.tile_bytes) || cfg.tile_bytes < 1024 ||
-      cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h)
+      cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 32 ||
+      cfg.scan_threads > 1024 || (cfg.scan_threads & 31) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
+      cfg.mover_run < 1 || cfg.mover_run > 64)
     return CRK_E_ARG;
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -243,7 +248,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   c->device = device;
   c->cfg = cfg;
   CK(cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device));
-  int occ = cfg.ctas_per_sm ? (int)cfg.ctas_per_sm : mover_occupancy();
+  int occ = cfg.ctas_per_sm ? (int)cfg.ctas_per_sm : mover_occupancy(cfg.tile_bytes, cfg.mover_stages);
   c->move_ctas = c->sms * (occ > 0 ? occ : 1);
   ConfigDev& d = c->cd;
   d.F = cfg.frag_payload;
@@ -255,6 +260,9 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.guess = cfg.scan_stride_guess ? cfg.scan_stride_guess : cfg.frag_payload;
   d.tile_shift = (uint32_t)__builtin_ctz(cfg.tile_bytes);
   d.max_record_bytes = cfg.max_record_bytes;
+  d.scan_threads = cfg.scan_threads;
+  d.stages = cfg.mover_stages;
+  d.run = cfg.mover_run;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
   // scratch: one block

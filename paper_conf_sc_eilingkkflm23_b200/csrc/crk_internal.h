@@ -108,6 +108,7 @@ struct Scratch {          // ctx-owned device scratch
 
 struct ConfigDev {
   uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
+  uint32_t scan_threads, stages, run, pad_;
   uint64_t max_record_bytes;
 };
 
@@ -158,7 +159,7 @@ cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n,
 // Plans tiles for jobs [0, n_jobs) (n_jobs from counters[1] <= max_jobs_bound) and runs the mover.
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
                                  int sms, int move_ctas, cudaStream_t s);
-int mover_occupancy();
+int mover_occupancy(uint32_t tile_bytes, uint32_t stages);
 
 // host-visible counter of our kernel launches
 void count_launch(int n = 1);

@@ -1,19 +1,25 @@
 // K4 / K5 / K6 / K7: the bulk movers.
 //
 // Work is a list of jobs (scratch.jobs).  A DEC job gathers logical bytes [loff, loff + n) of an indexed
-// record from the ring into dst (opaque unpad/scatter, K4) with an optional per-element byte swap
+// record from its ring into dst (opaque unpad/scatter, K4) with an optional per-element byte swap
 // (typed arrays, K5).  An ENC job writes a whole framed record (REPLY/CALL header words, XDR items from
 // device memory with optional swap, zero pads, RFC 5531 §11 fragment headers) into an output ring
 // (K6 / K7).  Each job's output range is cut into tiles aligned to tile_bytes in OUTPUT address space,
-// so no 16-byte output chunk is shared by two tiles; tile counts are prefix-summed (K2) and persistent
-// CTAs claim tiles with an atomic cursor.
+// so no 16-byte output chunk is shared by two tiles; tile counts are prefix-summed (K2).
 //
-// Inside a tile the output is a sequence of segments, each an affine map output -> source (one
-// fragment of a record on decode; one fragment x one data piece on encode).  Interior 16-byte output
-// chunks of a segment are built from two aligned 16-byte source loads joined by a funnel shift (the
-// shift is constant per segment; the second load comes from the neighbour lane by shuffle) and
-// byte-swapped per element; the at most 30 edge bytes of a segment are computed one by one with the
-// exact logical -> physical map, which also covers elements split across fragments.
+// The mover is a persistent, warp-specialised TMA pipeline.  Warp 0 (producer) claims tiles with an
+// atomic cursor, resolves tile -> job -> fragments, splits the tile into segments (each an affine map
+// output -> source: one fragment of a record on decode; fragment x data piece, or a literal run of
+// headers / words / pad, on encode) and issues cp.async.bulk copies of every data segment's 16-byte
+// aligned source window into a shared-memory stage, completing on the stage's mbarrier.  Warps 1-8
+// (consumers) wait on the stage, build each aligned 16-byte output chunk from two shared-memory chunks
+// with a funnel shift (constant per segment) and a per-element byte swap, store it with STG.128, and
+// release the stage.  The few edge bytes of a segment (at most 30) are computed one by one from the
+// exact logical -> physical map, which also covers elements split across fragments.  Tiles with more
+// segments than a stage describes (fragments smaller than ~tile/8) run the generic path: the same
+// segment walk done by the consumers with direct 16-byte global loads and warp-shuffle realignment.
+// Two tile queues (decode jobs, encode jobs) are claimed alternately so a serve step keeps both PCIe
+// directions busy when the rings live in host memory.
 #include "crk_device.cuh"
 #include "crk_logical.cuh"
 
@@ -21,24 +27,81 @@ namespace crk {
 
 namespace {
 
-constexpr int kU = 4;  // 16-byte chunks per lane per warp-slice iteration
+constexpr int kU = 4;           // 16-byte chunks per lane per warp-slice iteration (generic path)
+constexpr int kMaxSeg = 8;      // segments a stage can describe
+constexpr int kMaxStages = 8;   // pipeline depth limit (runtime: cfg.stages)
+constexpr int kConsumerWarps = 8;
+constexpr int kMoverThreads = 32 * (1 + kConsumerWarps);
+
+enum : uint32_t { SEG_DATA = 0, SEG_LIT = 1 };
+
+struct Seg {               // 32 bytes
+  uint64_t out_a, out_b;   // output range (DEC: dst addresses; ENC: out-ring cursors)
+  uint64_t src;            // DEC: ring cursor of the byte for out_a; ENC: V-order address of the byte for out_a
+  uint32_t smem_off;       // offset in the stage buffer of the aligned source window (staged only)
+  uint32_t flags;          // bit 0 staged, bits 8-15 kind, bits 16-23 element size
+};
+
+struct StageHdr {
+  uint32_t type, fallback, nseg, k0;
+  uint64_t a, b;
+  Job job;
+  RingDesc R;              // DEC: the record's ring; ENC: the output ring
+  Seg seg[kMaxSeg];
+  Piece pieces[kMaxPieces];
+};
 
 struct MoveParams {
   IndexDev ix;
   Scratch sc;
   ConfigDev cfg;
-  const uint64_t* prefix;  // [n_jobs + 1] exclusive tile prefix
+  const uint64_t* prefix;  // [n_jobs] exclusive tile prefix
   const uint32_t* n_jobs_dev;
   const uint64_t* total_tiles;
+  uint32_t stage_bytes;    // bytes of one stage buffer (after its header)
 };
 
-// Generic chunk loop over nch aligned output chunks.  load(i) returns source chunk i of the aligned
-// source window (already element-swapped on encode); store(i, v) writes output chunk i.
+struct Team {              // the consumer warps
+  uint32_t tid, nthr, warp, nwarps;
+};
+
+// ------------------------------------------------------------------------------------------- PTX
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "WAIT_%=: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// TMA 1-D bulk copy global -> shared (16-byte aligned, multiple of 16), completes on `bar`
+__device__ __forceinline__ void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(sdst)),
+               "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ uint4 lds16(const uint8_t* p) { return *reinterpret_cast<const uint4*>(p); }
+
+// ------------------------------------------------------------------------------------------- generic path
+// Chunk loop over nch aligned output chunks with direct global loads: load(i) returns source chunk i of
+// the aligned source window; the second chunk of the funnel comes from the neighbour lane.
 template <class Load, class Store>
-__device__ __forceinline__ void chunk_loop(uint64_t nch, uint32_t sh, const Load& load, const Store& store) {
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+__device__ __forceinline__ void chunk_loop(const Team& T, uint64_t nch, uint32_t sh, const Load& load,
+                                           const Store& store) {
+  const uint32_t lane = threadIdx.x & 31;
   const uint4 z = make_uint4(0, 0, 0, 0);
-  for (uint64_t base = (uint64_t)warp * 32 * kU; base < nch; base += (uint64_t)nwarps * 32 * kU) {
+  for (uint64_t base = (uint64_t)T.warp * 32 * kU; base < nch; base += (uint64_t)T.nwarps * 32 * kU) {
     uint4 A[kU];
 #pragma unroll
     for (int u = 0; u < kU; ++u) {
@@ -77,25 +140,29 @@ __device__ __forceinline__ void chunk_loop(uint64_t nch, uint32_t sh, const Load
   }
 }
 
-// ------------------------------------------------------------------------------------------- DEC
+// ---- DEC
 struct DecCtx {
   LogicalRecord L;
   uint64_t dst, loff;
   uint32_t es;
 };
-
+__device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, const Job& j) {
+  c.L.init(ix, ix.rings[ix.p_ring[j.rec]], ix.p_slot[j.rec]);
+  c.dst = j.out_start;
+  c.loff = j.loff;
+  c.es = j.esize;
+}
 // exact source of destination byte x (element e, byte j) = logical byte loff + e*es + (es-1-j)
 __device__ __forceinline__ uint8_t dec_exact_byte(DecCtx& c, uint64_t x) {
   const uint64_t i = x - c.dst;
   const uint64_t e = i / c.es, j = i - e * c.es;
   return c.L.byte(c.loff + e * c.es + (c.es - 1 - j));
 }
-
-__device__ void dec_segment(DecCtx& c, uint64_t xa, uint64_t xb, uint64_t src_at_xa) {
+__device__ void dec_segment_direct(const Team& T, DecCtx& c, uint64_t xa, uint64_t xb, uint64_t src_at_xa) {
   const uint64_t c0 = (xa + 15) & ~15ull, c1 = xb & ~15ull;
   const RingDesc R = c.L.R;
   auto edge = [&](uint64_t ea, uint64_t eb) {
-    for (uint64_t x = ea + threadIdx.x; x < eb; x += blockDim.x) {
+    for (uint64_t x = ea + T.tid; x < eb; x += T.nthr) {
       const uint8_t v = c.es == 1 ? ring_byte(R, src_at_xa + (x - xa)) : dec_exact_byte(c, x);
       *reinterpret_cast<uint8_t*>(x) = v;
     }
@@ -107,25 +174,49 @@ __device__ void dec_segment(DecCtx& c, uint64_t xa, uint64_t xb, uint64_t src_at
   const uint32_t sh = (uint32_t)(s0 & 15);
   const uint64_t ab = s0 - sh;
   const uint32_t es = c.es;
-  chunk_loop((c1 - c0) >> 4, sh,
-             [&](uint64_t i) { return ld16_stream(R.base + ((ab + 16 * i) & R.mask)); },
+  chunk_loop(T, (c1 - c0) >> 4, sh, [&](uint64_t i) { return ld16_stream(R.base + ((ab + 16 * i) & R.mask)); },
              [&](uint64_t i, uint4 v) { st16(reinterpret_cast<void*>(c0 + 16 * i), swap16(v, es)); });
 }
+__device__ void dec_tile_generic(const Team& T, DecCtx& c, uint64_t a, uint64_t b, uint32_t k) {
+  c.L.hint = k;
+  uint64_t r = a;
+  while (r < b && k < c.L.nfrags) {
+    const uint64_t ls = c.L.lstart[k], fl = c.L.flen(k), ph = c.L.phys[k];
+    const uint64_t sb = min(b, c.dst + (ls + fl - c.loff));
+    if (sb > r) {
+      dec_segment_direct(T, c, r, sb, ph + (c.loff + (r - c.dst) - ls));
+      r = sb;
+    }
+    ++k;
+  }
+}
 
-// ------------------------------------------------------------------------------------------- ENC
+// ---- ENC
 struct EncCtx {
   RingDesc O;
   uint64_t start;   // cursor of the record's first byte
   uint64_t Ll;      // logical length
-  uint32_t F, n_lens, nfr, np;
+  uint32_t F, nfr, np;
   const uint64_t* lens;    // explicit framing: fragment lengths
   const uint64_t* wstart;  // explicit framing: fragment wire starts (exclusive prefix of len + 4)
-  const Piece* P;          // smem
+  const Piece* P;
 };
 struct Frag {
   uint64_t fw, len, lf;  // wire start (rel), data length, logical start
   uint32_t last;
 };
+__device__ __forceinline__ void enc_ctx_init(EncCtx& c, const Scratch& sc, const Job& j, const RingDesc& O,
+                                             const Piece* P) {
+  c.O = O;
+  c.start = j.out_start;
+  c.Ll = j.loff;
+  c.F = j.F;
+  c.np = j.n_pieces;
+  c.P = P;
+  c.lens = sc.lens_pool + j.lens0;
+  c.wstart = sc.lens_pool + sc.max_lens + j.lens0;
+  c.nfr = c.F ? (uint32_t)(c.Ll == 0 ? 1 : (c.Ll + c.F - 1) / c.F) : j.n_lens;
+}
 __device__ __forceinline__ Frag enc_frag(const EncCtx& c, uint32_t f) {
   Frag r;
   if (c.F) {
@@ -142,193 +233,406 @@ __device__ __forceinline__ Frag enc_frag(const EncCtx& c, uint32_t f) {
 }
 __device__ __forceinline__ uint32_t enc_frag_of(const EncCtx& c, uint64_t w) {
   if (c.F) {
-    uint64_t f = w / (c.F + 4);
+    const uint64_t f = w / (c.F + 4);
     return (uint32_t)(f < c.nfr ? f : c.nfr - 1);
   }
   uint32_t lo = 0, hi = c.nfr;  // largest f with wstart[f] <= w
   while (hi - lo > 1) {
-    uint32_t mid = (lo + hi) >> 1;
+    const uint32_t mid = (lo + hi) >> 1;
     if (c.wstart[mid] <= w) lo = mid; else hi = mid;
   }
   return lo;
+}
+__device__ __forceinline__ uint64_t piece_extent(const Piece& p) {
+  return p.type == PIECE_WORDS ? p.nbytes : p.nbytes + ((4 - (p.nbytes & 3)) & 3);
 }
 // Byte at logical offset l of the record (l < Ll): header words, data (with swap) or zero pad.
 __device__ __forceinline__ uint8_t enc_logical_byte(const EncCtx& c, uint64_t l) {
   for (uint32_t k = 0; k < c.np; ++k) {
     const Piece& p = c.P[k];
-    if (p.type == PIECE_WORDS) {
-      if (l < p.loff + p.nbytes) {
-        const uint64_t i = l - p.loff;
-        return (uint8_t)(p.words[i >> 2] >> (24 - 8 * (i & 3)));
-      }
-    } else {
-      const uint64_t ext = p.nbytes + ((4 - (p.nbytes & 3)) & 3);
-      if (l < p.loff + ext) {
-        const uint64_t i = l - p.loff;
-        if (i >= p.nbytes) return 0;  // RFC 4506 §3 zero pad
-        const uint64_t e = i / p.esize, j = i - e * p.esize;
-        return *reinterpret_cast<const uint8_t*>(p.src + e * p.esize + (p.esize - 1 - j));
-      }
+    if (l < p.loff + piece_extent(p)) {
+      const uint64_t i = l - p.loff;
+      if (p.type == PIECE_WORDS) return (uint8_t)(p.words[i >> 2] >> (24 - 8 * (i & 3)));
+      if (i >= p.nbytes) return 0;  // RFC 4506 §3 zero pad
+      const uint64_t e = i / p.esize, j = i - e * p.esize;
+      return *reinterpret_cast<const uint8_t*>(p.src + e * p.esize + (p.esize - 1 - j));
     }
   }
   return 0;
 }
-__device__ __forceinline__ void enc_put(const EncCtx& c, uint64_t w, uint8_t v) {
-  c.O.base[(c.start + w) & c.O.mask] = v;
-}
-// per-byte output of wire range [wa, wb) inside fragment fr
-__device__ void enc_bytes(const EncCtx& c, const Frag& fr, uint64_t wa, uint64_t wb) {
-  for (uint64_t w = wa + threadIdx.x; w < wb; w += blockDim.x) {
-    const uint64_t q = w - fr.fw;
-    uint8_t v;
-    if (q < 4) {
-      const uint32_t h = (uint32_t)fr.len | (fr.last << 31);  // RFC 5531 §11 record mark
-      v = (uint8_t)(h >> (24 - 8 * q));
-    } else {
-      v = enc_logical_byte(c, fr.lf + (q - 4));
-    }
-    enc_put(c, w, v);
+// Wire byte w (relative to the record start): RFC 5531 §11 record mark or logical byte.
+__device__ __forceinline__ uint8_t enc_wire_byte(const EncCtx& c, uint64_t w) {
+  const Frag fr = enc_frag(c, enc_frag_of(c, w));
+  const uint64_t q = w - fr.fw;
+  if (q < 4) {
+    const uint32_t h = (uint32_t)fr.len | (fr.last << 31);
+    return (uint8_t)(h >> (24 - 8 * q));
   }
+  return enc_logical_byte(c, fr.lf + (q - 4));
 }
-// data segment: wire [wa, wb) (inside one fragment's data, one DATA piece's payload), first source
-// byte address src_at_wa in V order (element-swapped stream of the piece)
-__device__ void enc_segment(const EncCtx& c, const Frag& fr, uint64_t wa, uint64_t wb, const Piece& p,
-                            uint64_t l_at_wa) {
-  const uint64_t ca = c.start + wa, cb = c.start + wb;  // cursors
+__device__ __forceinline__ void enc_bytes(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb) {
+  for (uint64_t w = wa + T.tid; w < wb; w += T.nthr) c.O.base[(c.start + w) & c.O.mask] = enc_wire_byte(c, w);
+}
+__device__ void enc_segment_direct(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb, uint64_t src_at_wa,
+                                   uint32_t es) {
+  const uint64_t ca = c.start + wa, cb = c.start + wb;
   const uint64_t c0 = (ca + 15) & ~15ull, c1 = cb & ~15ull;
-  if (c0 >= c1) { enc_bytes(c, fr, wa, wb); return; }
-  enc_bytes(c, fr, wa, wa + (c0 - ca));
-  enc_bytes(c, fr, wb - (cb - c1), wb);
-  const uint64_t s0 = p.src + (l_at_wa - p.loff) + (c0 - ca);
-  const uint32_t sh = (uint32_t)(s0 & 15), es = p.esize;
+  if (c0 >= c1) { enc_bytes(T, c, wa, wb); return; }
+  enc_bytes(T, c, wa, wa + (c0 - ca));
+  enc_bytes(T, c, wb - (cb - c1), wb);
+  const uint64_t s0 = src_at_wa + (c0 - ca);
+  const uint32_t sh = (uint32_t)(s0 & 15);
   const uint64_t ab = s0 - sh;
   const RingDesc O = c.O;
-  chunk_loop((c1 - c0) >> 4, sh,
+  chunk_loop(T, (c1 - c0) >> 4, sh,
              [&](uint64_t i) { return swap16(ld16_stream(reinterpret_cast<const void*>(ab + 16 * i)), es); },
              [&](uint64_t i, uint4 v) { st16(O.base + ((c0 + 16 * i) & O.mask), v); });
 }
-
-__device__ void enc_tile(EncCtx& c, uint64_t ra, uint64_t rb) {
+// Walks wire range [ra, rb) of the record as runs: fragment headers, then per fragment the pieces'
+// data / literal parts.  emit(kind, wa, wb, src_at_wa, es) is called for each run in order.
+template <class Emit>
+__device__ __forceinline__ bool enc_runs(const EncCtx& c, uint64_t ra, uint64_t rb, const Emit& emit) {
   uint32_t f = enc_frag_of(c, ra);
   uint64_t w = ra;
   while (w < rb) {
     const Frag fr = enc_frag(c, f);
-    const uint64_t fend = fr.fw + 4 + fr.len;
-    // header
-    if (w < fr.fw + 4) {
-      const uint64_t he = min(rb, fr.fw + 4);
-      enc_bytes(c, fr, w, he);
+    const uint64_t he = min(rb, fr.fw + 4), de = min(rb, fr.fw + 4 + fr.len);
+    if (w < he) {
+      if (!emit(SEG_LIT, w, he, 0ull, 1u)) return false;
       w = he;
     }
-    // data run of this fragment inside the tile, piece by piece
-    const uint64_t de = min(rb, fend);
     while (w < de) {
       const uint64_t l = fr.lf + (w - fr.fw - 4);
-      // piece holding logical l
       uint32_t k = 0;
-      for (; k + 1 < c.np; ++k) if (c.P[k + 1].loff > l) break;
+      for (; k + 1 < c.np; ++k)
+        if (c.P[k + 1].loff > l) break;
       const Piece& p = c.P[k];
-      const uint64_t pext = p.type == PIECE_WORDS ? p.nbytes : p.nbytes + ((4 - (p.nbytes & 3)) & 3);
-      const uint64_t run_end_l = min(p.loff + pext, fr.lf + fr.len);
+      const uint64_t run_end_l = min(p.loff + piece_extent(p), fr.lf + fr.len);
       const uint64_t run_end_w = min(de, fr.fw + 4 + (run_end_l - fr.lf));
       if (p.type == PIECE_DATA && l < p.loff + p.nbytes) {
         const uint64_t dend_l = min(p.loff + p.nbytes, fr.lf + fr.len);
         const uint64_t dend_w = min(de, fr.fw + 4 + (dend_l - fr.lf));
-        enc_segment(c, fr, w, dend_w, p, l);
-        enc_bytes(c, fr, dend_w, run_end_w);  // pad bytes (if in this run)
+        if (!emit(SEG_DATA, w, dend_w, p.src + (l - p.loff), p.esize)) return false;
+        if (dend_w < run_end_w && !emit(SEG_LIT, dend_w, run_end_w, 0ull, 1u)) return false;
       } else {
-        enc_bytes(c, fr, w, run_end_w);
+        if (!emit(SEG_LIT, w, run_end_w, 0ull, 1u)) return false;
       }
       w = run_end_w;
     }
     f++;
   }
+  return true;
+}
+__device__ void enc_tile_generic(const Team& T, const EncCtx& c, uint64_t ra, uint64_t rb) {
+  enc_runs(c, ra, rb, [&](uint32_t kind, uint64_t wa, uint64_t wb, uint64_t src, uint32_t es) {
+    if (kind == SEG_LIT) enc_bytes(T, c, wa, wb);
+    else enc_segment_direct(T, c, wa, wb, src, es);
+    return true;
+  });
+}
+
+// ------------------------------------------------------------------------------------------- staged path
+// Interior chunks [c0, c1) of a staged data segment.  `o0` = offset in `buf` of the source byte that
+// lands on output chunk c0; the chunk's bytes are buf[o0 + 16 i .. + 16).
+__device__ __forceinline__ void staged_chunks(const Team& T, const uint8_t* buf, uint32_t o0, uint64_t nch,
+                                              uint64_t out0, const RingDesc* O, uint32_t es, bool dec) {
+  const uint32_t r = o0 & 15;
+  const uint8_t* q0 = buf + (o0 & ~15u);
+  for (uint64_t i = T.tid; i < nch; i += T.nthr) {
+    uint4 lo = lds16(q0 + 16 * i), v;
+    if (dec) {
+      v = r ? funnel16(lo, lds16(q0 + 16 * i + 16), r) : lo;
+      v = swap16(v, es);
+      st16(reinterpret_cast<void*>(out0 + 16 * i), v);
+    } else {
+      lo = swap16(lo, es);
+      v = r ? funnel16(lo, swap16(lds16(q0 + 16 * i + 16), es), r) : lo;
+      st16(O->base + ((out0 + 16 * i) & O->mask), v);
+    }
+  }
 }
 
 // ------------------------------------------------------------------------------------------- kernel
-__global__ void __launch_bounds__(kMoveThreads) mover_kernel(MoveParams M) {
-  __shared__ Job sj;
-  __shared__ __align__(16) Piece sp[kMaxPieces];
-  __shared__ uint32_t s_tile, s_job, s_k0;
-  __shared__ uint64_t s_pj;
+__device__ __forceinline__ uint32_t find_job(const uint64_t* prefix, uint32_t n_jobs, uint64_t tile, uint32_t lane) {
+  uint32_t lo = 0, hi = n_jobs;  // last j with prefix[j] <= tile (32-ary search, one warp)
+  while (hi - lo > 1) {
+    const uint32_t step = (hi - lo + 31) / 32;
+    const uint32_t idx = lo + lane * step;
+    const bool pred = idx < hi && prefix[idx] <= tile;
+    const uint32_t m = __ballot_sync(0xffffffffu, pred);
+    lo = lo + (31 - __clz(m)) * step;
+    hi = min(hi, lo + step);
+  }
+  return lo;
+}
+
+#ifndef CRK_MOVER_MIN_BLOCKS
+#define CRK_MOVER_MIN_BLOCKS 2
+#endif
+__global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_kernel(MoveParams M) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t full[kMaxStages], empty[kMaxStages];
+  const uint32_t kStages = M.cfg.stages, kRun = M.cfg.run;
+  const uint32_t stage_stride = (sizeof(StageHdr) + 127) / 128 * 128 + M.stage_bytes;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (uint32_t s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kConsumerWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
   const uint64_t total = *M.total_tiles;
   const uint32_t n_jobs = *M.n_jobs_dev;
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (;;) {
-    if (threadIdx.x == 0) s_tile = atomicAdd(M.sc.counters, 1u);
-    __syncthreads();
-    const uint32_t tile = s_tile;
-    if (tile >= total) break;
-    if (warp == 0) {  // 32-ary search: last job j with prefix[j] <= tile
-      uint32_t lo = 0, hi = n_jobs;
-      while (hi - lo > 1) {
-        const uint32_t step = (hi - lo + 31) / 32;
-        const uint32_t idx = lo + lane * step;
-        const bool pred = idx < hi && M.prefix[idx] <= tile;
-        const uint32_t m = __ballot_sync(0xffffffffu, pred);
-        const uint32_t l = 31 - __clz(m);
-        lo = lo + l * step;
-        hi = min(hi, lo + step);
-      }
-      if (lane == 0) { s_job = lo; s_pj = M.prefix[lo]; }
-    }
-    __syncthreads();
-    if (threadIdx.x < sizeof(Job) / 4)
-      reinterpret_cast<uint32_t*>(&sj)[threadIdx.x] =
-          reinterpret_cast<const uint32_t*>(M.sc.jobs + s_job)[threadIdx.x];
-    __syncthreads();
-    const uint64_t t = tile - s_pj;
-    const uint32_t shf = M.cfg.tile_shift;
-    const uint64_t A = sj.out_start >> shf;
-    const uint64_t a = max(sj.out_start, (A + t) << shf), b = min(sj.out_end, (A + t + 1) << shf);
-    if (sj.type == JOB_DEC) {
-      DecCtx c;
-      const uint32_t rec = sj.rec;
-      const uint32_t slot = M.ix.p_slot[rec];
-      c.L.init(M.ix, M.ix.rings[M.ix.p_ring[rec]], slot);
-      c.dst = sj.out_start;
-      c.loff = sj.loff;
-      c.es = sj.esize;
-      if (threadIdx.x == 0) s_k0 = c.L.find(c.loff + (a - c.dst));
-      __syncthreads();
-      uint32_t k = s_k0;
-      c.L.hint = k;
-      uint64_t r = a;
-      while (r < b && k < c.L.nfrags) {
-        const uint64_t ls = c.L.lstart[k], fl = c.L.flen(k), ph = c.L.phys[k];
-        const uint64_t fend = c.dst + (ls + fl - c.loff);
-        const uint64_t sb = min(b, fend);
-        if (sb > r) {
-          dec_segment(c, r, sb, ph + (c.loff + (r - c.dst) - ls));
-          r = sb;
+  const uint32_t n_split = M.sc.counters[4] < n_jobs ? M.sc.counters[4] : n_jobs;
+  const uint64_t split = n_split < n_jobs ? M.prefix[n_split] : total;
+  const uint32_t shf = M.cfg.tile_shift;
+
+  if (warp == 0) {
+    // ------------------------------------------------ producer
+    // Tiles are claimed in runs of kRun consecutive tiles, so the job lookup and the record state are
+    // paid once per run and the fragment walk continues from the previous tile's fragment.
+    uint32_t k = 0, claims = 0;
+    DecCtx dc;
+    for (;;) {
+      uint64_t t0 = ~0ull, t1 = 0;
+      if (lane == 0) {
+        const uint32_t pref = (claims + blockIdx.x) & 1;
+        for (int tries = 0; tries < 2 && t0 == ~0ull; ++tries) {
+          const uint32_t q = pref ^ tries;
+          const uint64_t lo = q ? split : 0, hi = q ? total : split;
+          if (lo < hi) {
+            const uint64_t t = lo + (uint64_t)kRun * atomicAdd(M.sc.counters + (q ? 2 : 0), 1u);
+            if (t < hi) { t0 = t; t1 = min(hi, t + kRun); }
+          }
         }
-        ++k;
       }
-    } else if (sj.type == JOB_ENC) {
-      for (uint32_t i = threadIdx.x; i < sj.n_pieces * (sizeof(Piece) / 4); i += blockDim.x)
-        reinterpret_cast<uint32_t*>(sp)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + sj.piece0)[i];
-      __syncthreads();
-      EncCtx c;
-      c.O = M.sc.out_rings[sj.out_ring];
-      c.start = sj.out_start;
-      c.Ll = sj.loff;
-      c.F = sj.F;
-      c.n_lens = sj.n_lens;
-      c.np = sj.n_pieces;
-      c.P = sp;
-      c.lens = M.sc.lens_pool + sj.lens0;
-      c.wstart = M.sc.lens_pool + M.sc.max_lens + sj.lens0;
-      c.nfr = c.F ? (uint32_t)(c.Ll == 0 ? 1 : (c.Ll + c.F - 1) / c.F) : c.n_lens;
-      enc_tile(c, a - c.start, b - c.start);
+      ++claims;
+      t0 = __shfl_sync(0xffffffffu, t0, 0);
+      t1 = __shfl_sync(0xffffffffu, t1, 0);
+      if (t0 == ~0ull) {
+        const uint32_t s = k % kStages;
+        StageHdr& H = *reinterpret_cast<StageHdr*>(smem + s * stage_stride);
+        mbar_wait(&empty[s], ((k / kStages) & 1) ^ 1);
+        if (lane == 0) {
+          H.type = JOB_NONE;
+          mbar_arrive(&full[s]);
+        }
+        break;
+      }
+      uint32_t j = find_job(M.prefix, n_jobs, t0, lane);
+      uint64_t pj = M.prefix[j], pnext = j + 1 < n_jobs ? M.prefix[j + 1] : ~0ull;
+      bool fresh = true;
+      for (uint64_t tile = t0; tile < t1; ++tile, ++k) {
+        while (tile >= pnext) {  // next job (zero-tile jobs share a prefix value)
+          ++j;
+          pj = pnext;
+          pnext = j + 1 < n_jobs ? M.prefix[j + 1] : ~0ull;
+          fresh = true;
+        }
+        const uint32_t s = k % kStages;
+        StageHdr& H = *reinterpret_cast<StageHdr*>(smem + s * stage_stride);
+        uint8_t* buf = smem + s * stage_stride + (sizeof(StageHdr) + 127) / 128 * 128;
+        mbar_wait(&empty[s], ((k / kStages) & 1) ^ 1);
+        // job + pieces into the stage header
+        if (lane < sizeof(Job) / 4)
+          reinterpret_cast<uint32_t*>(&H.job)[lane] = reinterpret_cast<const uint32_t*>(M.sc.jobs + j)[lane];
+        __syncwarp();
+        const Job& J = H.job;
+        if (J.type == JOB_ENC)
+          for (uint32_t i = lane; i < J.n_pieces * (sizeof(Piece) / 4); i += 32)
+            reinterpret_cast<uint32_t*>(H.pieces)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + J.piece0)[i];
+        __syncwarp();
+        if (lane == 0) {
+        const uint64_t t = tile - pj;
+        const uint64_t A = J.out_start >> shf;
+        const uint64_t a = max(J.out_start, (A + t) << shf), b = min(J.out_end, (A + t + 1) << shf);
+        H.type = J.type;
+        H.a = a;
+        H.b = b;
+        H.fallback = 0;
+        uint32_t nseg = 0, bytes = 0;
+        const uint32_t cap = M.stage_bytes;
+        // copies are collected first and issued after expect_tx
+        const void* csrc[2 * kMaxSeg];
+        uint32_t cdst[2 * kMaxSeg], clen[2 * kMaxSeg], nc = 0;
+        auto stage_window = [&](Seg& g, const uint8_t* base, uint64_t mask, bool ring, uint64_t w0, uint64_t w1) {
+          // w0..w1: 16-aligned source window (ring cursors or addresses)
+          const uint32_t len = (uint32_t)(w1 - w0);
+          if (bytes + len > cap) return;
+          g.smem_off = bytes;
+          g.flags |= 1;
+          if (ring) {
+            const uint64_t o0 = w0 & mask, cap_r = mask + 1;
+            const uint64_t room = cap_r - o0;
+            const uint32_t first = room < len ? (uint32_t)room : len;
+            csrc[nc] = base + o0; cdst[nc] = bytes; clen[nc] = first; ++nc;
+            if (first < len) { csrc[nc] = base; cdst[nc] = bytes + first; clen[nc] = len - first; ++nc; }
+          } else {
+            csrc[nc] = reinterpret_cast<const void*>(w0); cdst[nc] = bytes; clen[nc] = len; ++nc;
+          }
+          bytes += len;
+        };
+        if (J.type == JOB_DEC) {
+          if (fresh) dec_ctx_init(dc, M.ix, J);
+          DecCtx& c = dc;
+          H.R = c.L.R;
+          uint32_t kf = c.L.find(c.loff + (a - c.dst));
+          H.k0 = kf;
+          uint64_t r = a;
+          bool ok = true;
+          while (r < b && kf < c.L.nfrags) {
+            const uint64_t ls = c.L.lstart[kf], fl = c.L.flen(kf), ph = c.L.phys[kf];
+            const uint64_t sb = min(b, c.dst + (ls + fl - c.loff));
+            if (sb > r) {
+              if (nseg == kMaxSeg) { ok = false; break; }
+              Seg& g = H.seg[nseg++];
+              g.out_a = r;
+              g.out_b = sb;
+              g.src = ph + (c.loff + (r - c.dst) - ls);
+              g.flags = (SEG_DATA << 8) | (J.esize << 16);
+              const uint64_t c0 = (r + 15) & ~15ull, c1 = sb & ~15ull;
+              if (c0 < c1) {  // stage the source window of the interior chunks
+                const uint64_t s0 = g.src + (c0 - r);
+                const uint64_t w0 = s0 & ~15ull, w1 = (s0 + (c1 - c0) + 15) & ~15ull;
+                stage_window(g, c.L.R.base, c.L.R.mask, true, w0, w1);
+              }
+              r = sb;
+            }
+            ++kf;
+          }
+          if (!ok) { H.fallback = 1; nseg = 0; nc = 0; bytes = 0; }
+        } else if (J.type == JOB_ENC) {
+          EncCtx c;
+          const RingDesc O = M.sc.out_rings[J.out_ring];
+          enc_ctx_init(c, M.sc, J, O, H.pieces);
+          H.R = O;
+          const bool ok = enc_runs(c, a - c.start, b - c.start,
+                                   [&](uint32_t kind, uint64_t wa, uint64_t wb, uint64_t src, uint32_t es) {
+            if (kind == SEG_LIT && nseg > 0 && (H.seg[nseg - 1].flags >> 8 & 0xff) == SEG_LIT &&
+                H.seg[nseg - 1].out_b == c.start + wa) {
+              H.seg[nseg - 1].out_b = c.start + wb;  // merge literal runs
+              return true;
+            }
+            if (nseg == kMaxSeg) return false;
+            Seg& g = H.seg[nseg++];
+            g.out_a = c.start + wa;
+            g.out_b = c.start + wb;
+            g.src = src;
+            g.flags = (kind << 8) | (es << 16);
+            if (kind == SEG_DATA) {
+              const uint64_t c0 = (g.out_a + 15) & ~15ull, c1 = g.out_b & ~15ull;
+              if (c0 < c1) {
+                const uint64_t s0 = src + (c0 - g.out_a);
+                const uint64_t w0 = s0 & ~15ull, w1 = (s0 + (c1 - c0) + 15) & ~15ull;
+                stage_window(g, nullptr, 0, false, w0, w1);
+              }
+            }
+            return true;
+          });
+          if (!ok) { H.fallback = 1; nseg = 0; nc = 0; bytes = 0; }
+        }
+        H.nseg = nseg;
+        if (bytes) {
+          mbar_arrive_expect_tx(&full[s], bytes);
+          for (uint32_t i = 0; i < nc; ++i) bulk_g2s(buf + cdst[i], csrc[i], clen[i], &full[s]);
+        } else {
+          mbar_arrive(&full[s]);
+        }
+        }
+        fresh = false;
+        __syncwarp();
+      }
     }
-    __syncthreads();
+  } else {
+    // ------------------------------------------------ consumers
+    Team T;
+    T.tid = threadIdx.x - 32;
+    T.nthr = 32 * kConsumerWarps;
+    T.warp = warp - 1;
+    T.nwarps = kConsumerWarps;
+    for (uint32_t k = 0;; ++k) {
+      const uint32_t s = k % kStages;
+      const StageHdr& H = *reinterpret_cast<const StageHdr*>(smem + s * stage_stride);
+      const uint8_t* buf = smem + s * stage_stride + (sizeof(StageHdr) + 127) / 128 * 128;
+      mbar_wait(&full[s], (k / kStages) & 1);
+      const uint32_t type = H.type;
+      if (type == JOB_NONE) break;
+      const Job J = H.job;
+      if (type == JOB_DEC) {
+        if (H.fallback) {
+          DecCtx c;
+          dec_ctx_init(c, M.ix, J);
+          dec_tile_generic(T, c, H.a, H.b, H.k0);
+        } else {
+          for (uint32_t g = 0; g < H.nseg; ++g) {
+            const Seg S = H.seg[g];
+            const uint32_t es = S.flags >> 16 & 0xff;
+            const uint64_t c0 = (S.out_a + 15) & ~15ull, c1 = S.out_b & ~15ull;
+            if (!(S.flags & 1)) {  // not staged (stage full): direct loads
+              DecCtx c;
+              dec_ctx_init(c, M.ix, J);
+              dec_segment_direct(T, c, S.out_a, S.out_b, S.src);
+              continue;
+            }
+            const uint64_t s0 = S.src + (c0 - S.out_a);
+            staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, nullptr, es, true);
+            // edge bytes
+            const uint64_t ea = min(S.out_b, c0), eb = max(S.out_a, c1);
+            const uint32_t ne = (uint32_t)((ea - S.out_a) + (S.out_b - eb));
+            if (T.tid < ne) {
+              const uint64_t x = T.tid < ea - S.out_a ? S.out_a + T.tid : eb + (T.tid - (ea - S.out_a));
+              uint8_t v;
+              if (es == 1) {
+                v = ring_byte(H.R, S.src + (x - S.out_a));
+              } else {
+                DecCtx c;
+                dec_ctx_init(c, M.ix, J);
+                v = dec_exact_byte(c, x);
+              }
+              *reinterpret_cast<uint8_t*>(x) = v;
+            }
+          }
+        }
+      } else {
+        EncCtx c;
+        enc_ctx_init(c, M.sc, J, H.R, H.pieces);
+        if (H.fallback) {
+          enc_tile_generic(T, c, H.a - c.start, H.b - c.start);
+        } else {
+          for (uint32_t g = 0; g < H.nseg; ++g) {
+            const Seg S = H.seg[g];
+            const uint32_t kind = S.flags >> 8 & 0xff, es = S.flags >> 16 & 0xff;
+            if (kind == SEG_LIT) {
+              enc_bytes(T, c, S.out_a - c.start, S.out_b - c.start);
+              continue;
+            }
+            if (!(S.flags & 1)) {
+              enc_segment_direct(T, c, S.out_a - c.start, S.out_b - c.start, S.src, es);
+              continue;
+            }
+            const uint64_t c0 = (S.out_a + 15) & ~15ull, c1 = S.out_b & ~15ull;
+            const uint64_t s0 = S.src + (c0 - S.out_a);
+            staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, &H.R, es, false);
+            enc_bytes(T, c, S.out_a - c.start, min(S.out_b, c0) - c.start);
+            enc_bytes(T, c, max(S.out_a, c1) - c.start, S.out_b - c.start);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);
+    }
   }
 }
 
 // tiles per job: output range cut at tile_bytes-aligned boundaries
 __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, const uint32_t* n_jobs_dev) {
   const uint32_t n = *n_jobs_dev;
-  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[0] = 0;  // mover tile cursor
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    sc.counters[0] = 0;  // decode-queue tile cursor
+    sc.counters[2] = 0;  // encode-queue tile cursor
+  }
   for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
     const Job jb = sc.jobs[j];
     uint64_t c = 0;
@@ -339,6 +643,11 @@ __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, co
 }
 
 }  // namespace
+
+uint32_t mover_smem_bytes(uint32_t tile_bytes, uint32_t kStages) {
+  const uint32_t stage_bytes = tile_bytes + 32 * kMaxSeg + 32;
+  return kStages * ((uint32_t)(sizeof(StageHdr) + 127) / 128 * 128 + stage_bytes);
+}
 
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
                                  int sms, int move_ctas, cudaStream_t s) {
@@ -359,16 +668,28 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   M.prefix = tiles;
   M.n_jobs_dev = n_jobs_dev;
   M.total_tiles = total;
+  M.stage_bytes = (1u << cfg.tile_shift) + 32 * kMaxSeg + 32;
+  const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
+  static uint32_t smem_set = 0;  // dynamic shared memory opt-in (per process, grows monotonically)
+  if (smem > smem_set) {
+    e = cudaFuncSetAttribute(mover_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    smem_set = smem;
+  }
   prof_mark(PROF_MOVE, true, s);
-  mover_kernel<<<move_ctas, kMoveThreads, 0, s>>>(M);
+  mover_kernel<<<move_ctas, kMoverThreads, smem, s>>>(M);
   count_launch();
   prof_mark(PROF_MOVE, false, s);
   return cudaGetLastError();
 }
 
-int mover_occupancy() {
+// CTAs per SM the mover can keep resident for a tile size (sets the dynamic shared memory limit).
+int mover_occupancy(uint32_t tile_bytes, uint32_t stages) {
+  const uint32_t smem = mover_smem_bytes(tile_bytes, stages);
+  if (cudaFuncSetAttribute(mover_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+    return 0;
   int n = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, mover_kernel, kMoveThreads, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, mover_kernel, kMoverThreads, smem);
   return n;
 }
 

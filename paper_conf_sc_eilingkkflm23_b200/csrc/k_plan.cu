@@ -83,7 +83,7 @@ __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint3
     *st_out = st;
     if (cp_out) *cp_out = m;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+  if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
 }
 
 // typed / opaque argument requests (oracle or_decode_item)
@@ -113,7 +113,7 @@ __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uin
     *r.status = st;
     if (r.count) *r.count = cnt;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+  if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
 }
 
 // ---- serve: statuses, HtoD decode jobs and reply sizes (pass 1) --------------------------------
@@ -166,7 +166,7 @@ __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint6
     wire[d] = w;
     sc.jobs[d] = job;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = 2 * total;
+  if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = 2 * total; sc.counters[4] = total; }
 }
 
 struct SendRingsParam {
@@ -227,6 +227,7 @@ __global__ void put_enc_jobs_kernel(Scratch sc, EncJobParam p, RingDesc out) {
     for (uint32_t j = 0; j < p.n_jobs; ++j) sc.jobs[j] = p.jobs[j];
     sc.out_rings[0] = out;
     sc.counters[1] = p.n_jobs;
+    sc.counters[4] = p.n_jobs;
   }
   for (uint32_t i = threadIdx.x; i < p.n_pieces; i += blockDim.x) sc.pieces[i] = p.pieces[i];
 }
@@ -238,7 +239,7 @@ __global__ void d2h_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const ui
     const uint64_t Ll = err == 0 ? 32 + nb + pad4(nb) : 28;
     sc.scan_tmp[i] = wire_of(Ll, cfg.F);
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) sc.counters[1] = n;
+  if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
 }
 
 __global__ void d2h_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uint32_t* xids, const void* const* srcs,

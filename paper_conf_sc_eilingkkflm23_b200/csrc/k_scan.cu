@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, S
 
 cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s) {
   prof_mark(PROF_SCAN, true, s);
-  frame_scan_kernel<<<p.n_rings, kScanThreads, 0, s>>>(ix, p, cfg);
+  frame_scan_kernel<<<p.n_rings, cfg.scan_threads, 0, s>>>(ix, p, cfg);
   count_launch();
   prof_mark(PROF_SCAN, false, s);
   return cudaGetLastError();
