@@ -209,11 +209,9 @@ def main():
         return
     import torch
     import torch.distributed as dist
-    from paper_conf_sc_eilingkkflm23_b200 import build, crk, workload
+    from paper_conf_sc_eilingkkflm23_b200 import build, crk, parallel, workload
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    world, rank, local = parallel.rank_env()
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     torch.cuda.set_device(local)
@@ -221,23 +219,13 @@ def main():
     build.build()
 
     def barrier():
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
+        parallel.barrier(dev)
 
     def max_over_ranks(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return parallel.max_over_ranks(x, dev)
 
     def sum_over_ranks(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
-        return float(t.item())
+        return parallel.sum_over_ranks(x, dev)
 
     ctx = crk.Context(local)
     ep = workload.c5_endpoint(ctx, rank, dev, n_streams=args.streams, payload_per_stream=args.payload_mib * MiB)
