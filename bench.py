@@ -43,6 +43,7 @@ def parse_args():
     p.add_argument("--streams", type=int, default=16)
     p.add_argument("--payload-mib", type=int, default=64, help="payload per stream")
     p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--pipeline", type=int, default=2, help="batches in flight (server loop slots)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -227,25 +228,44 @@ def main():
     def sum_over_ranks(x: float) -> float:
         return parallel.sum_over_ranks(x, dev)
 
-    ctx = crk.Context(local)
-    ep = workload.c5_endpoint(ctx, rank, dev, n_streams=args.streams, payload_per_stream=args.payload_mib * MiB)
-    idx = ctx.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
+    # A server loop keeps `pipeline` batches in flight: each slot is a (context, index, stream, batch
+    # buffers) set, so the front end (scan / parse / plan) of batch k+1 runs while the mover of batch k
+    # streams bytes.  Step k is served by slot k % pipeline; every step is one full pass over its batch.
+    P = max(1, args.pipeline)
     stream = torch.cuda.current_stream(dev)
+    slots = []
+    for i in range(P):
+        ctx_i = crk.Context(local)
+        ep_i = workload.c5_endpoint(ctx_i, rank, dev, n_streams=args.streams,
+                                    payload_per_stream=args.payload_mib * MiB)
+        idx_i = ctx_i.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
+        slots.append(workload.Slot(ctx_i, idx_i, ep_i, torch.cuda.Stream(dev) if P > 1 else stream))
+    ep = slots[0].ep
+
+    def run(n_steps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for s in slots:
+            s.stream.wait_event(e0)
+        for k in range(n_steps):
+            s = slots[k % P]
+            workload.serve_step(s.idx, s.ep, stream=s.stream)
+        for s in slots:
+            ev = torch.cuda.Event()
+            ev.record(s.stream)
+            stream.wait_event(ev)
+        e1.record(stream)
+        return e0, e1
 
     # ---- device-resident timed region (value)
-    for _ in range(args.warmup):
-        workload.serve_step(idx, ep)
+    run(max(args.warmup, P))
     barrier()
-    check = workload.check_results(idx, ep)
+    check = workload.check_results(slots[0].idx, slots[0].ep)
     crk.profile_enable(True)
     l0 = crk.kernel_launches()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     with ClockSampler(local) as clk:
-        e0.record(stream)
-        for _ in range(args.steps):
-            workload.serve_step(idx, ep)
-        e1.record(stream)
+        e0, e1 = run(args.steps)
         torch.cuda.synchronize()
     launches = crk.kernel_launches() - l0
     prof = crk.profile_read()
@@ -254,6 +274,17 @@ def main():
     ms_max = max_over_ranks(ms)
     payload_all = sum_over_ranks(ep.payload)
     value = payload_all / (ms_max / 1e3) / 1e9
+    # the same steps one at a time (no overlap), for reference
+    serial_ms = None
+    if P > 1:
+        s0 = slots[0]
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(min(args.steps, 50)):
+            workload.serve_step(s0.idx, s0.ep, stream=stream)
+        f1.record(stream)
+        torch.cuda.synchronize()
+        serial_ms = max_over_ranks(f0.elapsed_time(f1) / min(args.steps, 50))
 
     # roofline of the dominant kernel (the mover): algorithmic HBM bytes per launch / its event time
     mv_ms, mv_n = prof["move"]
@@ -276,7 +307,8 @@ def main():
     # ---- end to end through the C ABI with host (pinned, mapped) rings
     e2e = None
     if not args.no_e2e:
-        del idx
+        ctx = slots[0].ctx
+        del slots
         torch.cuda.empty_cache()
         ep_h = workload.c5_endpoint(ctx, rank, dev, n_streams=args.streams, payload_per_stream=args.payload_mib * MiB,
                                     host_rings=True)
@@ -317,6 +349,7 @@ def main():
                      "kernel": "crk mover_kernel (K4 opaque scatter + K6 reply encode)",
                      "alg_bytes_per_launch": alg_bytes, "launch_ms": round(mv_launch_ms, 4),
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, read+write)"},
+        "pipeline": P, "serial_ms_per_step": None if serial_ms is None else round(serial_ms, 4),
         "stages_ms_per_step": {k: round(v[0] / max(1, v[1]), 4) for k, v in prof.items()},
         "stage_share": stage_share,
         "payload_bytes_per_gpu": ep.payload, "wire_in_bytes_per_gpu": ep.wire_in,

@@ -97,7 +97,7 @@ typedef struct {
   uint32_t tile_bytes;       /* bytes per mover work tile, power of two in [1024, 1<<20] (default 32768) */
   uint32_t max_jobs;         /* decode + encode job capacity per call (default 1<<20) */
   uint32_t ctas_per_sm;      /* mover occupancy override, 0 = occupancy calculator */
-  uint32_t scan_threads;     /* K1 threads per ring = candidate headers per round, 32..1024 (default 128) */
+  uint32_t scan_threads;     /* K1 threads per ring, two predictor groups, 64..1024, multiple of 64 (default 256) */
   uint32_t mover_stages;     /* mover pipeline stages, 2..8 (default 3) */
   uint32_t mover_run;        /* tiles per mover claim, 1..64 (default 8) */
 } crk_config;

@@ -222,7 +222,7 @@ void crk_config_init(crk_config* c) {
   c->tile_bytes = 32768;
   c->max_jobs = 1u << 20;
   c->ctas_per_sm = 0;
-  c->scan_threads = 128;
+  c->scan_threads = 256;
   c->mover_stages = 3;
   c->mover_run = 8;
 }
@@ -233,8 +233,8 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   crk_config cfg;
   if (cfg_in) cfg = *cfg_in; else crk_config_init(&cfg);
   if (cfg.frag_payload == 0 || cfg.frag_payload > 0x7fffffffu || !pow2(cfg.tile_bytes) || cfg.tile_bytes < 1024 ||
-      cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 32 ||
-      cfg.scan_threads > 1024 || (cfg.scan_threads & 31) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
+      cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 64 ||
+      cfg.scan_threads > 1024 || (cfg.scan_threads & 63) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
       cfg.mover_run < 1 || cfg.mover_run > 64)
     return CRK_E_ARG;
   int ndev = 0;

@@ -11,7 +11,7 @@ constexpr int kMaxItems = CRK_MAX_ITEMS;
 constexpr int kMaxProcs = CRK_MAX_PROCS;
 constexpr int kMaxRings = CRK_MAX_RINGS;
 constexpr int kScanThreads = 1024;  // K1: one CTA per ring, one candidate header per thread
-constexpr int kParseWarps = 8;      // K3: one warp per record
+constexpr int kParseWarps = 4;      // K3: one warp per record (small CTAs co-reside with the mover)
 constexpr int kMoveThreads = 256;   // K4/K6 mover CTA
 constexpr int kMaxPieces = 2 * kMaxItems + 2;
 

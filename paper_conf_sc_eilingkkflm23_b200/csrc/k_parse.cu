@@ -26,19 +26,27 @@ __device__ __forceinline__ bool kind_is_var(uint32_t k) {
 }
 __device__ __forceinline__ uint64_t pad4(uint64_t n) { return (4 - (n & 3)) & 3; }
 
+constexpr uint32_t kHead = 64;  // record head prefetched by the warp (CALL header + memcpy args)
+
 struct Parser {
   LogicalRecord L;
   uint64_t o;
+  const uint8_t* head;  // first `nhead` logical bytes, already in shared memory
+  uint32_t nhead;
+  __device__ __forceinline__ uint8_t byte(uint64_t at) { return at < nhead ? head[at] : L.byte(at); }
   __device__ int get_u32(uint32_t& v) {
     if (o + 4 > L.len) return CRK_E_TRUNCATED;
-    v = L.be32(o);
+    if (o + 4 <= nhead)
+      v = ((uint32_t)head[o] << 24) | ((uint32_t)head[o + 1] << 16) | ((uint32_t)head[o + 2] << 8) | head[o + 3];
+    else
+      v = L.be32(o);
     o += 4;
     return CRK_OK;
   }
   // RFC 4506 §3: the pad bytes after an item must be zero (checked in strict mode)
   __device__ bool pad_is_zero(uint64_t at, uint64_t n) {
     for (uint64_t i = 0; i < n; ++i)
-      if (L.byte(at + i) != 0) return false;
+      if (byte(at + i) != 0) return false;
     return true;
   }
   __device__ int get_auth(bool strict) {
@@ -58,6 +66,7 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
                                                                   ConfigDev cfg, uint32_t n_rings) {
   __shared__ SchemaTable sch;
   __shared__ uint32_t prefix[kMaxRings + 1];
+  __shared__ __align__(16) uint8_t heads[kParseWarps][kHead];
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(tab)[i];
   const uint32_t total = *ix.total;
@@ -66,7 +75,6 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t gw = blockIdx.x * kParseWarps + warp, nw = gridDim.x * kParseWarps;
   for (uint32_t d = gw; d < total; d += nw) {
-    if (lane != 0) continue;
     // ring of dense record d: the last r < n_rings with prefix[r] <= d (empty rings share a prefix)
     uint32_t lo = 0, hi = n_rings;
     while (hi - lo > 1) {
@@ -78,6 +86,18 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
     Parser P;
     P.L.init(ix, ix.rings[ring], slot);
     P.o = 0;
+    // the warp prefetches the record head from its first fragment in one round trip
+    const uint64_t n0 = P.L.flen(0);
+    const uint64_t nh = n0 < P.L.len ? n0 : P.L.len;
+    P.nhead = nh < kHead ? (uint32_t)nh : kHead;
+    if (lane < P.nhead) heads[warp][lane] = ring_byte(P.L.R, P.L.phys[0] + lane);
+    if (lane + 32 < P.nhead) heads[warp][lane + 32] = ring_byte(P.L.R, P.L.phys[0] + lane + 32);
+    P.head = heads[warp];
+    __syncwarp();
+    if (lane != 0) {
+      __syncwarp();
+      continue;
+    }
     const bool strict = cfg.strict != 0;
     uint32_t xid = 0, proc = 0, v, nitems = 0;
     int st = CRK_OK;
@@ -153,6 +173,7 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
         h = (h + 1) & ix.hash_mask;
       }
     }
+    __syncwarp();  // pairs with the other lanes' wait: the head buffer is free for the next record
   }
 }
 
@@ -161,7 +182,7 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
 cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const ConfigDev& cfg, uint32_t n_rings,
                          int sms, cudaStream_t s) {
   prof_mark(PROF_PARSE, true, s);
-  parse_kernel<<<sms * 4, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
+  parse_kernel<<<sms * 8, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
   count_launch();
   prof_mark(PROF_PARSE, false, s);
   return cudaGetLastError();

@@ -1,16 +1,18 @@
 // K1 + K2 (fragment part): speculative record-marking scan (RFC 5531 §11) with the segmented prefix
 // sum of fragment lengths that gives every fragment its logical start.
 //
-// The header chain is sequential (p[k+1] = p[k] + 4 + len[k]).  One CTA per ring walks it in rounds:
-// from a known true header at p, thread t reads the candidate header at p + t * (4 + len(h_pred)),
-// where h_pred is the predicted header value.  If headers 0..t-1 all equal h_pred their positions are
-// exact, so candidate t is a true header (induction); the first t* whose value differs is still a true
-// header.  A round therefore accepts t* + 1 headers with one memory latency, and 1024 at a time when
-// the sender frames regularly (greedy F-byte fragments, or back-to-back identical records).  Because
-// headers 0..t*-1 are identical, the fragment lengths' segmented prefix sums (logical starts) and the
-// record boundaries have closed forms in t; the checks are then the oracle's, in its order
-// (oracle/oracle.c or_frame_scan; DESIGN.md §4 readings R1, R2, R8):
-//   E_FRAG (sum > max_record_bytes)  ->  INCOMPLETE (data past tail)  ->  index capacity.
+// The header chain is sequential (p[k+1] = p[k] + 4 + len[k]).  One CTA per ring walks it in rounds.
+// From a known true header at p, the CTA splits into two groups, one per predicted header value h_g:
+// thread u of group g reads the candidate header at p + u * (4 + len(h_g)).  If headers 0..u-1 all equal
+// h_g their positions are exact, so candidate u is a true header (induction); the first u* whose value
+// differs is still a true header.  The group with the longer run wins: a round accepts u* + 1 headers
+// with one memory latency.  Predictor 0 follows the stride of multi-fragment records (greedy F-byte
+// fragments); predictor 1 remembers the shape of the last single-fragment record, so streams that mix
+// large HtoD calls with small DtoH calls advance about one record per round, and
+// back-to-back identical records (C1) a whole group per round.  Because headers 0..u*-1 are identical,
+// the fragment lengths' segmented prefix sums (logical starts) and the record boundaries have closed
+// forms in u; the checks are then the oracle's, in its order (oracle/oracle.c or_frame_scan;
+// DESIGN.md §3 readings R1, R2, R8): E_FRAG -> INCOMPLETE (data past tail) -> index capacity.
 #include "crk_device.cuh"
 
 namespace crk {
@@ -18,54 +20,74 @@ namespace crk {
 namespace {
 
 enum : uint32_t { STOP_NONE = 0, STOP_FRAG = 1, STOP_INCOMPLETE = 2, STOP_CAP = 3 };
+constexpr uint32_t kNoPred = 0xffffffffu;  // a predictor value no header is expected to match
 
 struct ScanState {
   uint64_t p, r0, sum;
-  uint32_t f0, nf, nr, hpred;
+  uint32_t f0, nf, nr;
+  uint32_t hp[2];
   uint32_t done;
   int32_t status;
   uint64_t consumed;
   uint32_t kept_frags;
-  uint32_t tstar, valid_star, h_star;
-  uint32_t tf, code_f;
+  uint32_t valid_star, h_star;
+  uint32_t code_f;
+  uint32_t gmin[32];
 };
 
-__global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
+__global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
   const uint32_t ring = blockIdx.x;
   const RingDesc R = P.r[ring];
-  const uint32_t t = threadIdx.x, T = blockDim.x;
+  const uint32_t T = blockDim.x >> 1;                  // candidates per group
+  const uint32_t grp = threadIdx.x >= T, u = threadIdx.x - grp * T;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5, wpg = nw >> 1;
   const uint32_t FC = ix.frags_per_ring, RC = ix.recs_per_ring;
   const uint64_t fbase = (uint64_t)ring * FC, rbase = (uint64_t)ring * RC;
   __shared__ ScanState S;
-  __shared__ uint32_t red[32];
-  if (t == 0) {
+  if (threadIdx.x == 0) {
     ix.rings[ring] = R;
     S.p = S.r0 = R.head;
     S.sum = 0;
     S.f0 = S.nf = S.nr = 0;
-    S.hpred = cfg.guess & 0x7fffffffu;
+    S.hp[0] = cfg.guess & 0x7fffffffu;
+    S.hp[1] = kNoPred;
     S.done = 0;
   }
   __syncthreads();
   while (!S.done) {
     const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
-    const uint32_t hpred = S.hpred, nf = S.nf, nr = S.nr, f0 = S.f0;
-    const uint64_t Lp = hpred & 0x7fffffffu;
-    const uint32_t lastp = hpred >> 31;
-    const uint64_t stride = 4 + Lp;
-    const uint64_t q = p + (uint64_t)t * stride;
+    const uint32_t nf = S.nf, nr = S.nr, f0 = S.f0;
+    // ---- both groups speculate from the true header at p
+    uint32_t hpred = S.hp[grp];
+    const uint64_t q = p + (uint64_t)u * (4 + (uint64_t)(hpred & 0x7fffffffu));
     const bool valid = q + 4 <= R.tail;
     const uint32_t h = valid ? ring_be32(R, q) : 0u;
     const bool ok = valid && h == hpred;
-    const uint32_t tstar = block_min_u32(ok ? T : t, red);
-    if (t == tstar) { S.valid_star = valid; S.h_star = h; }
+    // per-group first mismatch (groups are whole warps)
+    uint32_t m = __ballot_sync(0xffffffffu, !ok);
+    if (lane == 0) S.gmin[warp] = m ? (warp - grp * wpg) * 32 + __ffs(m) - 1 : T;
     __syncthreads();
+    uint32_t ts0 = T, ts1 = T;
+    for (uint32_t w = 0; w < nw; ++w) {
+      if (w < wpg) ts0 = min(ts0, S.gmin[w]);
+      else ts1 = min(ts1, S.gmin[w]);
+    }
+    // the group with the longer verified run wins (ties: group 0)
+    const uint32_t win = ts1 > ts0;
+    const uint32_t tstar = win ? ts1 : ts0;
+    const bool mine = grp == win;
+    const uint32_t t = u;
+    if (mine && t == tstar) { S.valid_star = valid; S.h_star = h; }
+    __syncthreads();
+    hpred = S.hp[win];
+    const uint64_t Lp = hpred & 0x7fffffffu;
+    const uint32_t lastp = hpred >> 31;
     const bool end_at_star = tstar < T && !S.valid_star;
     const uint32_t n_hdr = tstar == T ? T : (end_at_star ? tstar : tstar + 1);
     const uint32_t hstar = S.h_star;
 
     // per-header closed forms (headers 0..tstar-1 equal hpred)
-    const bool is_hdr = t < n_hdr;
+    const bool is_hdr = mine && t < n_hdr;
     const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
     const uint32_t last = (t < tstar) ? lastp : (hstar >> 31);
     const bool start = (t == 0) ? (p == r0) : (lastp != 0);
@@ -81,13 +103,17 @@ __global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, S
       else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
       else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
     }
-    const uint32_t tf = block_min_u32(code != STOP_NONE ? t : 0xffffffffu, red);
-    if (t == tf) S.code_f = code;
+    m = __ballot_sync(0xffffffffu, code != STOP_NONE);
+    if (lane == 0) S.gmin[warp] = (m && grp == win) ? (warp - grp * wpg) * 32 + __ffs(m) - 1 : 0xffffffffu;
+    __syncthreads();
+    uint32_t tf = 0xffffffffu;
+    for (uint32_t w = 0; w < nw; ++w) tf = min(tf, S.gmin[w]);
+    if (mine && t == tf) S.code_f = code;
     __syncthreads();
     const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
 
     // emit fragments (and the records they complete)
-    if (t < n_emit) {
+    if (mine && t < n_emit) {
       const uint64_t fs = fbase + nf + t;
       ix.frag_phys[fs] = q + 4;
       ix.frag_lstart[fs] = send - len;
@@ -101,10 +127,9 @@ __global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, S
       }
     }
     // the stopping thread (failure at tf, or no readable header at tstar) records the outcome
-    const bool stops_here = (tf < n_hdr) ? (t == tf) : (end_at_star && t == tstar);
+    const bool stops_here = mine && ((tf < n_hdr) ? (t == tf) : (end_at_star && t == tstar));
     if (stops_here) {
-      const uint64_t rstart = start ? q : r0;
-      S.consumed = rstart;
+      S.consumed = start ? q : r0;
       S.kept_frags = start ? nf + t : f0;
       S.nr = nrec;
       if (tf < n_hdr) {
@@ -117,8 +142,8 @@ __global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, S
       }
       S.done = 1;
     }
-    // the last accepted header advances the state
-    if (!stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
+    // the last accepted header advances the state and the predictors
+    if (mine && !stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
       S.p = q + 4 + len;
       S.nf = nf + n_hdr;
       if (last) {
@@ -132,12 +157,16 @@ __global__ void __launch_bounds__(kScanThreads) frame_scan_kernel(IndexDev ix, S
         S.r0 = start ? q : r0;
         S.f0 = start ? nf + t : f0;
       }
-      // keep a fruitful prediction; switch to the observed header when the round made no progress
-      if (tstar < T && tstar == 0) S.hpred = hstar;
+      if (tstar < T) {
+        // a single-fragment record's shape becomes predictor 1; a non-last fragment of another length
+        // becomes predictor 0 (a new stride); the last fragment of a multi-fragment record changes nothing
+        if (start && last) S.hp[1] = hstar;
+        else if (!last) S.hp[0] = hstar;
+      }
     }
     __syncthreads();
   }
-  if (t == 0) {
+  if (threadIdx.x == 0) {
     crk_ring_result& rr = ix.res[ring];
     rr.status = S.status;
     rr.n_records = S.nr;

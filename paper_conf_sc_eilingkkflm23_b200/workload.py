@@ -102,6 +102,16 @@ def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: in
     return ep
 
 
+@dataclass
+class Slot:
+    """One in-flight batch of a pipelined server loop: its own context (scratch), index, stream and
+    batch buffers, so consecutive batches overlap without sharing state."""
+    ctx: crk.Context
+    idx: crk.Index
+    ep: Endpoint
+    stream: torch.cuda.Stream
+
+
 def serve_step(idx: crk.Index, ep: Endpoint, stream=None):
     idx.serve(ep.rings, ep.sends, ep.offs, ep.base, ep.region.numel(), stream=stream)
 

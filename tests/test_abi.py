@@ -38,7 +38,7 @@ def test_exports_every_declared_symbol(L):
 def test_config_defaults(L):
     c = crk.config()
     assert c.frag_payload == 65536 and c.strict == 1 and c.max_record_bytes == 1 << 32
-    assert c.tile_bytes == 32768 and c.max_jobs == 1 << 20 and c.scan_threads == 128
+    assert c.tile_bytes == 32768 and c.max_jobs == 1 << 20 and c.scan_threads == 256
 
 
 def test_wire_size_closed_form_matches_oracle(L):
