@@ -162,6 +162,15 @@ void crk_index_destroy(crk_index* idx);
 int crk_index_get_view(const crk_index* idx, crk_index_view* out);
 /* Copies the per-ring results of the last scan/serve to host memory and waits for `stream`. */
 int crk_index_ring_results(crk_index* idx, uint32_t n_rings, crk_ring_result* host_out, crk_stream_t stream);
+/* The same copy without waiting: `pinned_out` must be pinned host memory; valid once `stream` completes. */
+int crk_index_ring_results_async(crk_index* idx, uint32_t n_rings, crk_ring_result* pinned_out, crk_stream_t stream);
+
+/* Copies the cursor window [head, tail) of ring `src` into ring `dst` at the same cursors (each side
+ * wrapping at its own capacity) with copy-engine DMA (cudaMemcpyAsync, any direction).  This is the
+ * staging step of the copy-engine e2e mode: a pinned host receive ring is moved into a device ring that
+ * crk_serve then reads from HBM, and reply bytes are moved back out of a device send ring.
+ * tail - head must not exceed either capacity. */
+int crk_ring_copy(crk_ring dst, crk_ring src, uint64_t head, uint64_t tail, crk_stream_t stream);
 
 /* ---------------------------------------------------------------- K1-K3: frame scan + CALL parse
  * Scans ring r's window [heads[r], tails[r]) (RFC 5531 §11), fills the fragment table with each

@@ -94,6 +94,8 @@ def lib():
             "crk_index_destroy": (None, [vp]),
             "crk_index_get_view": (C.c_int, [vp, C.POINTER(IndexView)]),
             "crk_index_ring_results": (C.c_int, [vp, u32, C.POINTER(RingResult), vp]),
+            "crk_index_ring_results_async": (C.c_int, [vp, u32, vp, vp]),
+            "crk_ring_copy": (C.c_int, [CRing, CRing, u64, u64, vp]),
             "crk_rpc_frame_scan": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(u64), C.POINTER(u64), vp]),
             "crk_xdr_decode_memcpy_h2d": (C.c_int, [vp, vp, u32, vp, u64, vp, vp, vp]),
             "crk_xdr_decode_memcpy_h2d_batch": (C.c_int, [vp, vp, u32, vp, vp, vp, vp, vp, vp]),
@@ -256,6 +258,24 @@ class Ring:
             i += k
 
 
+def ring_copy(dst: Ring, src: Ring, head: int, tail: int, stream=None):
+    """Copy-engine copy of the cursor window [head, tail) from ring src to ring dst (crk_ring_copy)."""
+    _check(lib().crk_ring_copy(dst.c(), src.c(), head, tail, _stream(stream)), "crk_ring_copy")
+
+
+class PinnedResults:
+    """Pinned host slots for crk_index_ring_results_async."""
+
+    def __init__(self, n: int):
+        self.buf = HostBuffer(C.sizeof(RingResult) * max(1, n))
+        self.n = n
+
+    def rows(self) -> list[dict]:
+        arr = (RingResult * self.n).from_address(self.buf.ptr)
+        return [dict(status=r.status, n_records=r.n_records, n_frags=r.n_frags, rec_base=r.rec_base,
+                     consumed=r.consumed, reply_bytes=r.reply_bytes) for r in arr]
+
+
 def copy_to_host(dev_ptr: int, nbytes: int) -> np.ndarray:
     out = np.empty(max(1, nbytes), np.uint8)
     if nbytes:
@@ -415,6 +435,10 @@ class Index:
         _check(lib().crk_index_ring_results(self.h, n, out, _stream(stream)), "crk_index_ring_results")
         return [dict(status=r.status, n_records=r.n_records, n_frags=r.n_frags, rec_base=r.rec_base,
                      consumed=r.consumed, reply_bytes=r.reply_bytes) for r in out[:n]]
+
+    def ring_results_async(self, out: "PinnedResults", stream=None):
+        _check(lib().crk_index_ring_results_async(self.h, out.n, out.buf.ptr, _stream(stream)),
+               "crk_index_ring_results_async")
 
     def tables(self, n_rings: int | None = None) -> dict:
         """Host copies of the index tables after synchronising the device (tests / inspection)."""

@@ -448,6 +448,28 @@ int crk_index_ring_results(crk_index* x, uint32_t n_rings, crk_ring_result* host
   return CRK_OK;
 }
 
+int crk_index_ring_results_async(crk_index* x, uint32_t n_rings, crk_ring_result* pinned_out, crk_stream_t stream) {
+  if (!x || !pinned_out || n_rings > x->ix.max_rings) return CRK_E_ARG;
+  DeviceGuard g(x->ctx->device);
+  CK(cudaMemcpyAsync(pinned_out, x->ix.res, sizeof(crk_ring_result) * n_rings, cudaMemcpyDeviceToHost,
+                     (cudaStream_t)stream));
+  return CRK_OK;
+}
+
+int crk_ring_copy(crk_ring dst, crk_ring src, uint64_t head, uint64_t tail, crk_stream_t stream) {
+  if (!ring_ok(dst) || !ring_ok(src) || tail < head || tail - head > dst.cap || tail - head > src.cap)
+    return CRK_E_ARG;
+  for (uint64_t c = head; c < tail;) {  // contiguous pieces: neither side wraps inside a piece
+    const uint64_t os = c & (src.cap - 1), od = c & (dst.cap - 1);
+    uint64_t n = tail - c;
+    if (n > src.cap - os) n = src.cap - os;
+    if (n > dst.cap - od) n = dst.cap - od;
+    CK(cudaMemcpyAsync(dst.base + od, src.base + os, n, cudaMemcpyDefault, (cudaStream_t)stream));
+    c += n;
+  }
+  return CRK_OK;
+}
+
 int crk_rpc_frame_scan(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
                        const uint64_t* tails, crk_stream_t stream) {
   if (!c || !x || x->ctx != c) return CRK_E_ARG;

@@ -38,6 +38,8 @@ class Endpoint:
     n_records: int = 0
     per_stream_reply: list = field(default_factory=list)
     per_stream_records: list = field(default_factory=list)
+    dev_rings: list = field(default_factory=list)   # staged mode: device copies of the host rings
+    dev_sends: list = field(default_factory=list)
 
     @property
     def base(self) -> int:
@@ -49,7 +51,8 @@ class Endpoint:
 
 
 def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: int = 16,
-                payload_per_stream: int = 64 * MiB, host_rings: bool = False, misalign: bool = False) -> Endpoint:
+                payload_per_stream: int = 64 * MiB, host_rings: bool = False, misalign: bool = False,
+                staged: bool = False) -> Endpoint:
     streams, region_bytes = gen.c5_endpoint(rank, n_streams=n_streams, payload_per_stream=payload_per_stream,
                                             h2d_budget=payload_per_stream - payload_per_stream // 16,
                                             misalign=misalign)
@@ -85,7 +88,12 @@ def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: in
             host = torch.from_numpy(ring.host_view())
             host[:cur].copy_(ring_dev.tensor()[:cur].cpu())
             send = crk.Ring.host(next_pow2(reply + 4096))
-            del ring_dev
+            if staged:  # device rings the copy engine stages into / out of (crk_ring_copy)
+                ring_dev.tensor().zero_()
+                ep.dev_rings.append(ring_dev)
+                ep.dev_sends.append(crk.Ring.device(send.cap, device))
+            else:
+                del ring_dev
         else:
             ring = ring_dev
             send = crk.Ring.device(next_pow2(reply + 4096), device)
@@ -114,6 +122,24 @@ class Slot:
 
 def serve_step(idx: crk.Index, ep: Endpoint, stream=None):
     idx.serve(ep.rings, ep.sends, ep.offs, ep.base, ep.region.numel(), stream=stream)
+
+
+def staged_in_and_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResults", stream):
+    """Copy-engine mode, first half of a step: DMA each host receive window into its device ring,
+    serve from HBM into the device send rings, and queue the per-ring results to pinned memory."""
+    for (hr, h, t), dr in zip(ep.rings, ep.dev_rings):
+        crk.ring_copy(dr, hr, h, t, stream=stream)
+    idx.serve([(dr, h, t) for dr, (_, h, t) in zip(ep.dev_rings, ep.rings)], ep.dev_sends, ep.offs, ep.base,
+              ep.region.numel(), stream=stream)
+    idx.ring_results_async(results, stream=stream)
+
+
+def staged_out(ep: Endpoint, rows: list, stream):
+    """Second half: DMA each ring's reply bytes (now known on the host) back to the host send ring."""
+    for r, (hs, ds, off) in enumerate(zip(ep.sends, ep.dev_sends, ep.offs)):
+        n = rows[r]["reply_bytes"]
+        if n:
+            crk.ring_copy(hs, ds, off, off + n, stream=stream)
 
 
 def check_results(idx: crk.Index, ep: Endpoint) -> dict:

@@ -175,6 +175,25 @@ int main(int argc, char** argv) {
              tile, stages, per_sm, zr.best, zr.med, hb.best, hb.med);
     }
   }
+  // bidirectional: SM zero-copy reads and writes at once (two kernels on two streams), and a CE
+  // H2D copy concurrent with SM zero-copy writes
+  {
+    size_t half16 = n16 / 2;
+    Stat bi_sm = time_it([&] {
+      CK(cudaEventRecord(ev0, 0)); CK(cudaStreamWaitEvent(s1, ev0)); CK(cudaStreamWaitEvent(s2, ev0));
+      ldg_copy<4><<<sms * 2, 256, 0, s1>>>((const int4*)hd_a, (int4*)d_a, half16);
+      ldg_copy<4><<<sms * 2, 256, 0, s2>>>((const int4*)d_b, (int4*)hd_b, half16);
+      CK(cudaEventRecord(e1, s1)); CK(cudaEventRecord(e2, s2));
+      CK(cudaStreamWaitEvent(0, e1)); CK(cudaStreamWaitEvent(0, e2)); }, (double)n);
+    Stat ce_sm = time_it([&] {
+      CK(cudaEventRecord(ev0, 0)); CK(cudaStreamWaitEvent(s1, ev0)); CK(cudaStreamWaitEvent(s2, ev0));
+      CK(cudaMemcpyAsync(d_a, h_a, n / 2, cudaMemcpyHostToDevice, s1));
+      ldg_copy<4><<<sms * 2, 256, 0, s2>>>((const int4*)d_b, (int4*)hd_b, half16);
+      CK(cudaEventRecord(e1, s1)); CK(cudaEventRecord(e2, s2));
+      CK(cudaStreamWaitEvent(0, e1)); CK(cudaStreamWaitEvent(0, e2)); }, (double)n);
+    printf(" \"sm_zc_bidir_gbs\": [%.2f, %.2f], \"ce_h2d_plus_sm_zc_write_gbs\": [%.2f, %.2f],\n", bi_sm.best, bi_sm.med,
+           ce_sm.best, ce_sm.med);
+  }
   // correctness of the bulk path from sysmem
   CK(cudaMemset(d_a, 0, n));
   for (size_t i = 0; i < n; i += 4093) h_a[i] = (uint8_t)(i * 7);
