@@ -377,8 +377,8 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (uint32_t s = 0; s < kStages; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], kConsumerWarps);
+      mbar_init(&full[s], 32);  // every producer lane arrives after its own writes to the stage
+      mbar_init(&empty[s], 32 * kConsumerWarps);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -415,10 +415,8 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
         const uint32_t s = k % kStages;
         StageHdr& H = *reinterpret_cast<StageHdr*>(smem + s * stage_stride);
         mbar_wait(&empty[s], ((k / kStages) & 1) ^ 1);
-        if (lane == 0) {
-          H.type = JOB_NONE;
-          mbar_arrive(&full[s]);
-        }
+        if (lane == 0) H.type = JOB_NONE;
+        mbar_arrive(&full[s]);
         break;
       }
       uint32_t j = find_job(M.prefix, n_jobs, t0, lane);
@@ -444,6 +442,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           for (uint32_t i = lane; i < J.n_pieces * (sizeof(Piece) / 4); i += 32)
             reinterpret_cast<uint32_t*>(H.pieces)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + J.piece0)[i];
         __syncwarp();
+        if (lane != 0) mbar_arrive(&full[s]);  // lanes 1-31 are done writing this stage
         if (lane == 0) {
         const uint64_t t = tile - pj;
         const uint64_t A = J.out_start >> shf;
@@ -620,8 +619,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           }
         }
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[s]);
+      mbar_arrive(&empty[s]);  // every consumer thread releases the stage after its last read of it
     }
   }
 }

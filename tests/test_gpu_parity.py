@@ -525,3 +525,37 @@ def test_serve_matches_oracle(host):
         assert T["rings"][r]["consumed"] == want["consumed"][r]
         n = want["reply_bytes"][r]
         assert sends[r].read(offs[r], n) == bytes(want["send"][r][offs[r]:offs[r] + n])
+
+
+def test_ring_copy_and_async_results():
+    g = gen.rng(21)
+    for (cd, cs) in [(1 << 12, 1 << 12), (1 << 12, 1 << 14), (1 << 14, 1 << 12)]:
+        src = crk.Ring.host(cs)
+        src.host_view()[:] = gen.random_bytes(cs, cs)
+        dst = crk.Ring.device(cd)
+        dst.tensor().fill_(0)
+        for _ in range(5):
+            head = int(g.integers(0, 1 << 20))
+            n = int(g.integers(0, min(cd, cs) + 1))
+            crk.ring_copy(dst, src, head, head + n)
+            torch.cuda.synchronize()
+            assert dst.read(head, n) == src.read(head, n)
+            back = crk.Ring.host(cs)
+            crk.ring_copy(back, dst, head, head + n)
+            torch.cuda.synchronize()
+            assert back.read(head, n) == src.read(head, n)
+    with pytest.raises(crk.CrkError):
+        crk.ring_copy(dst, src, 0, max(cd, cs) + 1)
+    cfg = ocfg()
+    ctx = ctx_for(cfg)
+    ring = make_ring(1 << 16)
+    w = O.encode_call(1, gen.PROC_H2D, [(O.K_U64, 0), (O.K_OPAQUE_VAR, b"abc"), (O.K_U64, 3)], cfg)
+    ring.write(0, w)
+    idx = ctx.index(2, 1024, 64)
+    idx.frame_scan([(ring, 0, len(w)), (ring, 0, 3)])
+    out = crk.PinnedResults(2)
+    idx.ring_results_async(out)
+    torch.cuda.synchronize()
+    rows = out.rows()
+    assert rows == idx.ring_results(2)
+    assert rows[0]["status"] == O.OK and rows[0]["n_records"] == 1 and rows[1]["status"] == O.INCOMPLETE
