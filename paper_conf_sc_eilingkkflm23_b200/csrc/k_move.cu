@@ -640,6 +640,52 @@ __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, co
   }
 }
 
+// Small requests (<= kSmallJobs jobs): tile counts, their exclusive prefix (K2 in one block) and the
+// cursor reset in a single launch.
+constexpr uint32_t kSmallJobs = 2048;
+__global__ void __launch_bounds__(256) plan_small_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, uint64_t* total,
+                                                         const uint32_t* n_jobs_dev) {
+  __shared__ uint64_t warp_sum[8];
+  const uint32_t n = *n_jobs_dev;
+  if (threadIdx.x == 0) {
+    sc.counters[0] = 0;
+    sc.counters[2] = 0;
+  }
+  constexpr uint32_t IPT = kSmallJobs / 256;
+  uint64_t v[IPT], acc = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < IPT; ++i) {
+    const uint32_t j = threadIdx.x * IPT + i;
+    uint64_t c = 0;
+    if (j < n) {
+      const Job jb = sc.jobs[j];
+      if (jb.type != JOB_NONE && jb.out_end > jb.out_start)
+        c = ((jb.out_end - 1) >> cfg.tile_shift) - (jb.out_start >> cfg.tile_shift) + 1;
+    }
+    v[i] = c;
+    acc += c;
+  }
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint64_t x = acc;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  if (lane == 31) warp_sum[w] = x;
+  __syncthreads();
+  uint64_t base = 0;
+  for (uint32_t i = 0; i < w; ++i) base += warp_sum[i];
+  uint64_t run = base + x - acc;
+#pragma unroll
+  for (uint32_t i = 0; i < IPT; ++i) {
+    const uint32_t j = threadIdx.x * IPT + i;
+    if (j < n) tiles[j] = run;
+    run += v[i];
+  }
+  if (threadIdx.x == 255) *total = run;
+}
+
 }  // namespace
 
 uint32_t mover_smem_bytes(uint32_t tile_bytes, uint32_t kStages) {
@@ -648,21 +694,37 @@ uint32_t mover_smem_bytes(uint32_t tile_bytes, uint32_t kStages) {
 }
 
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
-                                 int sms, int move_ctas, cudaStream_t s) {
+                                 uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s) {
   uint64_t* tiles = sc.scan_tmp;  // [max_jobs + 1]
   uint64_t* total = sc.scan_tmp + sc.max_jobs + 1;
   const uint32_t* n_jobs_dev = sc.counters + 1;
-  const uint32_t cnt_blocks = max_jobs_bound ? (max_jobs_bound + 255) / 256 : 1;
-  plan_count_kernel<<<min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s>>>(sc, cfg, tiles, n_jobs_dev);
-  count_launch();
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  e = launch_exclusive_scan_u64(tiles, max_jobs_bound, n_jobs_dev, total, sc, s);
-  if (e != cudaSuccess) return e;
+  cudaError_t e;
+  if (max_jobs_bound <= kSmallJobs) {
+    plan_small_kernel<<<1, 256, 0, s>>>(sc, cfg, tiles, total, n_jobs_dev);
+    count_launch();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  } else {
+    const uint32_t cnt_blocks = (max_jobs_bound + 255) / 256;
+    plan_count_kernel<<<min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s>>>(sc, cfg, tiles, n_jobs_dev);
+    count_launch();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    e = launch_exclusive_scan_u64(tiles, max_jobs_bound, n_jobs_dev, total, sc, s);
+    if (e != cudaSuccess) return e;
+  }
+  // a known bound on the output bytes caps the grid at the tiles that can exist
+  uint32_t run = cfg.run;
+  if (out_bytes_bound) {
+    const uint64_t tiles_max = 2ull * max_jobs_bound + (out_bytes_bound >> cfg.tile_shift) + 1;
+    if (tiles_max < (uint64_t)move_ctas * run) {
+      run = 1;  // few tiles: one per claim, spread over the CTAs
+      if (tiles_max < (uint64_t)move_ctas) move_ctas = (int)tiles_max;
+    }
+  }
   MoveParams M;
   if (ix) M.ix = *ix; else memset(&M.ix, 0, sizeof(M.ix));
   M.sc = sc;
   M.cfg = cfg;
+  M.cfg.run = run;
   M.prefix = tiles;
   M.n_jobs_dev = n_jobs_dev;
   M.total_tiles = total;

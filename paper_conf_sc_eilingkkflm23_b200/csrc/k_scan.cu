@@ -21,6 +21,7 @@ namespace {
 
 enum : uint32_t { STOP_NONE = 0, STOP_FRAG = 1, STOP_INCOMPLETE = 2, STOP_CAP = 3 };
 constexpr uint32_t kNoPred = 0xffffffffu;  // a predictor value no header is expected to match
+constexpr uint32_t kJ = 4;                 // candidate headers per thread and round (independent loads)
 
 struct ScanState {
   uint64_t p, r0, sum;
@@ -30,7 +31,7 @@ struct ScanState {
   int32_t status;
   uint64_t consumed;
   uint32_t kept_frags;
-  uint32_t valid_star, h_star;
+  uint32_t valid_star, h_star, wide;
   uint32_t code_f;
   uint32_t gmin[32];
 };
@@ -38,7 +39,7 @@ struct ScanState {
 __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
   const uint32_t ring = blockIdx.x;
   const RingDesc R = P.r[ring];
-  const uint32_t T = blockDim.x >> 1;                  // candidates per group
+  const uint32_t T = blockDim.x >> 1;                  // threads per group
   const uint32_t grp = threadIdx.x >= T, u = threadIdx.x - grp * T;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5, wpg = nw >> 1;
   const uint32_t FC = ix.frags_per_ring, RC = ix.recs_per_ring;
@@ -52,22 +53,35 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     S.hp[0] = cfg.guess & 0x7fffffffu;
     S.hp[1] = kNoPred;
     S.done = 0;
+    S.wide = 0;
   }
   __syncthreads();
   while (!S.done) {
     const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
     const uint32_t nf = S.nf, nr = S.nr, f0 = S.f0;
-    // ---- both groups speculate from the true header at p
+    // ---- both groups speculate from the true header at p; thread u owns candidates u + j*T
     uint32_t hpred = S.hp[grp];
-    const uint64_t q = p + (uint64_t)u * (4 + (uint64_t)(hpred & 0x7fffffffu));
-    const bool valid = q + 4 <= R.tail;
-    const uint32_t h = valid ? ring_be32(R, q) : 0u;
-    const bool ok = valid && h == hpred;
+    const uint64_t stride = 4 + (uint64_t)(hpred & 0x7fffffffu);
+    // a round uses kJ candidates per thread only after a round that accepted every candidate (a long
+    // regular run: big records); otherwise one, which keeps the round short
+    const uint32_t jn = S.wide ? kJ : 1u, TT = T * jn;
+    uint32_t hv[kJ];
+    bool vv[kJ];
+    uint32_t first_bad = TT;
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j) {
+      const uint32_t t = u + j * T;
+      if (j >= jn) { vv[j] = false; hv[j] = 0; continue; }
+      const uint64_t q = p + (uint64_t)t * stride;
+      vv[j] = q + 4 <= R.tail;
+      hv[j] = vv[j] ? ring_be32(R, q) : 0u;
+      if (!(vv[j] && hv[j] == hpred)) first_bad = min(first_bad, t);
+    }
     // per-group first mismatch (groups are whole warps)
-    uint32_t m = __ballot_sync(0xffffffffu, !ok);
-    if (lane == 0) S.gmin[warp] = m ? (warp - grp * wpg) * 32 + __ffs(m) - 1 : T;
+    uint32_t wm = __reduce_min_sync(0xffffffffu, first_bad);
+    if (lane == 0) S.gmin[warp] = wm;
     __syncthreads();
-    uint32_t ts0 = T, ts1 = T;
+    uint32_t ts0 = TT, ts1 = TT;
     for (uint32_t w = 0; w < nw; ++w) {
       if (w < wpg) ts0 = min(ts0, S.gmin[w]);
       else ts1 = min(ts1, S.gmin[w]);
@@ -76,92 +90,114 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     const uint32_t win = ts1 > ts0;
     const uint32_t tstar = win ? ts1 : ts0;
     const bool mine = grp == win;
-    const uint32_t t = u;
-    if (mine && t == tstar) { S.valid_star = valid; S.h_star = h; }
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j)
+      if (mine && u + j * T == tstar) { S.valid_star = vv[j]; S.h_star = hv[j]; }
     __syncthreads();
     hpred = S.hp[win];
     const uint64_t Lp = hpred & 0x7fffffffu;
     const uint32_t lastp = hpred >> 31;
-    const bool end_at_star = tstar < T && !S.valid_star;
-    const uint32_t n_hdr = tstar == T ? T : (end_at_star ? tstar : tstar + 1);
+    const bool end_at_star = tstar < TT && !S.valid_star;
+    const uint32_t n_hdr = tstar == TT ? TT : (end_at_star ? tstar : tstar + 1);
     const uint32_t hstar = S.h_star;
 
-    // per-header closed forms (headers 0..tstar-1 equal hpred)
-    const bool is_hdr = mine && t < n_hdr;
-    const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
-    const uint32_t last = (t < tstar) ? lastp : (hstar >> 31);
-    const bool start = (t == 0) ? (p == r0) : (lastp != 0);
-    // logical end of header t within its record (segmented inclusive prefix sum of lengths)
-    uint64_t send;
-    if (!lastp) send = sum + (uint64_t)t * Lp + len;
-    else send = (t == 0) ? (start ? len : sum + len) : len;
-    const uint32_t nrec = lastp ? nr + t : nr;  // completed records before header t
-
-    uint32_t code = STOP_NONE;
-    if (is_hdr) {
-      if (send > cfg.max_record_bytes) code = STOP_FRAG;
-      else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
-      else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
+    // per-header closed forms (headers 0..tstar-1 equal hpred); checks in the oracle's order
+    uint32_t codes[kJ];
+    uint32_t first_fail = 0xffffffffu;
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j) {
+      const uint32_t t = u + j * T;
+      const uint64_t q = p + (uint64_t)t * stride;
+      const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
+      const bool start = (t == 0) ? (p == r0) : (lastp != 0);
+      uint64_t send;  // logical end of header t within its record (segmented prefix sum of lengths)
+      if (!lastp) send = sum + (uint64_t)t * Lp + len;
+      else send = (t == 0) ? (start ? len : sum + len) : len;
+      const uint32_t nrec = lastp ? nr + t : nr;  // completed records before header t
+      uint32_t code = STOP_NONE;
+      if (mine && j < jn && t < n_hdr) {
+        if (send > cfg.max_record_bytes) code = STOP_FRAG;
+        else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
+        else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
+      }
+      codes[j] = code;
+      if (code != STOP_NONE) first_fail = min(first_fail, t);
     }
-    m = __ballot_sync(0xffffffffu, code != STOP_NONE);
-    if (lane == 0) S.gmin[warp] = (m && grp == win) ? (warp - grp * wpg) * 32 + __ffs(m) - 1 : 0xffffffffu;
+    wm = __reduce_min_sync(0xffffffffu, first_fail);
+    if (lane == 0) S.gmin[warp] = wm;
     __syncthreads();
     uint32_t tf = 0xffffffffu;
     for (uint32_t w = 0; w < nw; ++w) tf = min(tf, S.gmin[w]);
-    if (mine && t == tf) S.code_f = code;
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j)
+      if (mine && u + j * T == tf) S.code_f = codes[j];
     __syncthreads();
     const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
 
-    // emit fragments (and the records they complete)
-    if (mine && t < n_emit) {
-      const uint64_t fs = fbase + nf + t;
-      ix.frag_phys[fs] = q + 4;
-      ix.frag_lstart[fs] = send - len;
-      ix.frag_hdr[fs] = (uint32_t)len | (last << 31);
-      if (last) {
-        const uint64_t rs = rbase + nrec;
-        ix.rec_begin[rs] = start ? q : r0;
-        ix.rec_len[rs] = send;
-        ix.rec_frag0[rs] = (uint32_t)(fbase + (start ? nf + t : f0));
-        ix.rec_nfrags[rs] = start ? 1u : nf + t - f0 + 1;
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j) {
+      const uint32_t t = u + j * T;
+      if (!mine || j >= jn) break;
+      const uint64_t q = p + (uint64_t)t * stride;
+      const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
+      const uint32_t last = (t < tstar) ? lastp : (hstar >> 31);
+      const bool start = (t == 0) ? (p == r0) : (lastp != 0);
+      uint64_t send;
+      if (!lastp) send = sum + (uint64_t)t * Lp + len;
+      else send = (t == 0) ? (start ? len : sum + len) : len;
+      const uint32_t nrec = lastp ? nr + t : nr;
+      // emit fragments (and the records they complete)
+      if (t < n_emit) {
+        const uint64_t fs = fbase + nf + t;
+        ix.frag_phys[fs] = q + 4;
+        ix.frag_lstart[fs] = send - len;
+        ix.frag_hdr[fs] = (uint32_t)len | (last << 31);
+        if (last) {
+          const uint64_t rs = rbase + nrec;
+          ix.rec_begin[rs] = start ? q : r0;
+          ix.rec_len[rs] = send;
+          ix.rec_frag0[rs] = (uint32_t)(fbase + (start ? nf + t : f0));
+          ix.rec_nfrags[rs] = start ? 1u : nf + t - f0 + 1;
+        }
       }
-    }
-    // the stopping thread (failure at tf, or no readable header at tstar) records the outcome
-    const bool stops_here = mine && ((tf < n_hdr) ? (t == tf) : (end_at_star && t == tstar));
-    if (stops_here) {
-      S.consumed = start ? q : r0;
-      S.kept_frags = start ? nf + t : f0;
-      S.nr = nrec;
-      if (tf < n_hdr) {
-        const uint32_t c = S.code_f;
-        S.status = c == STOP_FRAG ? CRK_E_FRAG
-                 : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
-                 : (nrec > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
-      } else {
-        S.status = (start && q == R.tail) ? CRK_OK : CRK_INCOMPLETE;
-      }
-      S.done = 1;
-    }
-    // the last accepted header advances the state and the predictors
-    if (mine && !stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
-      S.p = q + 4 + len;
-      S.nf = nf + n_hdr;
-      if (last) {
-        S.nr = nrec + 1;
-        S.r0 = q + 4 + len;
-        S.sum = 0;
-        S.f0 = nf + n_hdr;
-      } else {
+      // the stopping candidate (failure at tf, or no readable header at tstar) records the outcome
+      const bool stops_here = (tf < n_hdr) ? (t == tf) : (end_at_star && t == tstar);
+      if (stops_here) {
+        S.consumed = start ? q : r0;
+        S.kept_frags = start ? nf + t : f0;
         S.nr = nrec;
-        S.sum = send;
-        S.r0 = start ? q : r0;
-        S.f0 = start ? nf + t : f0;
+        if (tf < n_hdr) {
+          const uint32_t c = S.code_f;
+          S.status = c == STOP_FRAG ? CRK_E_FRAG
+                   : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
+                   : (nrec > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
+        } else {
+          S.status = (start && q == R.tail) ? CRK_OK : CRK_INCOMPLETE;
+        }
+        S.done = 1;
       }
-      if (tstar < T) {
-        // a single-fragment record's shape becomes predictor 1; a non-last fragment of another length
-        // becomes predictor 0 (a new stride); the last fragment of a multi-fragment record changes nothing
-        if (start && last) S.hp[1] = hstar;
-        else if (!last) S.hp[0] = hstar;
+      // the last accepted header advances the state and the predictors
+      if (!stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
+        S.wide = tstar == TT;
+        S.p = q + 4 + len;
+        S.nf = nf + n_hdr;
+        if (last) {
+          S.nr = nrec + 1;
+          S.r0 = q + 4 + len;
+          S.sum = 0;
+          S.f0 = nf + n_hdr;
+        } else {
+          S.nr = nrec;
+          S.sum = send;
+          S.r0 = start ? q : r0;
+          S.f0 = start ? nf + t : f0;
+        }
+        if (tstar < TT) {
+          // a single-fragment record's shape becomes predictor 1; a non-last fragment of another length
+          // becomes predictor 0 (a new stride); the last fragment of a multi-fragment record changes nothing
+          if (start && last) S.hp[1] = hstar;
+          else if (!last) S.hp[0] = hstar;
+        }
       }
     }
     __syncthreads();

@@ -1,0 +1,276 @@
+"""Per-config measurements beside the bench headline.
+
+Device-resident rings, CUDA-event timing on the launching stream after warm-up; every config checks its
+output against the generator's values.  Writes one JSON object (stdout).
+
+  C1   one CALL (4 KiB opaque + 1,024 int32): latency of scan+parse -> memcpy decode -> int32 decode, and
+       131,072 back-to-back records: records/s and GB/s of scan+parse+batch decode
+  C2   matrixMul transfers (A, B HtoD; C DtoH) served as one batch: microseconds
+  C3   bandwidth sweep: HtoD (scan+parse+decode) and DtoH (reply encode) GB/s per size, buffers rotated
+       over >= 256 MiB so repeated runs do not hit L2
+  C4   256 MiB typed-array stress: decode GB/s (all items, regular and irregular framing)
+  NEXT-1  one 1 GiB memcpy striped over 16 rings (16 CALLs of 64 MiB at ptr + offset), served as one batch
+  NEXT-2  cuSolverDn-shaped (100 x 900x900 f64 HtoD + 7.2 KB DtoH) and histogram-shaped (64 MiB HtoD, 1 KiB DtoH)
+"""
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_sc_eilingkkflm23_b200 import build, crk, gen  # noqa: E402
+
+MiB, GiB = 1 << 20, 1 << 30
+dev = torch.device("cuda:0")
+
+
+def timed(fn, reps, warm=3):
+    for _ in range(warm):
+        fn(0)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for i in range(reps):
+        fn(i)
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps  # ms
+
+
+def next_pow2(x):
+    return 1 << max(8, (x - 1).bit_length())
+
+
+def c1(ctx):
+    ctx.register_schema(gen.PROC_C1, gen.C1_SCHEMA)
+    c = gen.c1_call(xid=1)
+    data = torch.from_numpy(c.items[1][1]).to(dev)
+    ints = torch.from_numpy(c.items[3][1]).to(dev)
+    items = [(crk.K_U64, c.items[0][1]), (crk.K_OPAQUE_VAR, data), (crk.K_U64, 4096), (crk.K_I32_VAR, ints)]
+    ring = crk.Ring.device(1 << 14)
+    w = ctx.encode_call(1, gen.PROC_C1, items, ring, 0)
+    idx = ctx.index(1, 64, 16)
+    dst = torch.empty(4096, dtype=torch.uint8, device=dev)
+    out = torch.empty(1024, dtype=torch.int32, device=dev)
+    st = torch.zeros(2, dtype=torch.int32, device=dev)
+    cnt = torch.zeros(2, dtype=torch.int64, device=dev)
+
+    def one(_):
+        idx.frame_scan([(ring, 0, w)])
+        idx.decode_opaque(1, 1, dst, 4096, cnt[0:1], st[0:1])
+        idx.decode_array("i32", 1, 3, out, 1024, cnt[1:2], st[1:2])
+
+    lat_ms = timed(one, 200)
+    ok = bool(torch.equal(dst, data) and torch.equal(out, ints) and (st == 0).all())
+    # 131,072 back-to-back records
+    n = 131072
+    big = crk.Ring.device(next_pow2(n * w + 4096))
+    big.tensor()[:w].copy_(ring.tensor()[:w])
+    reps = torch.arange(n, device=dev, dtype=torch.int64)
+    body = big.tensor()[:w].clone()
+    view = big.tensor()[:n * w].view(n, w)
+    view.copy_(body.unsqueeze(0).expand(n, w))
+    xids = (torch.arange(n, dtype=torch.int64) + 0x100000).to(torch.int32)
+    xb = xids.numpy().astype(">u4").view(np.uint8).reshape(n, 4)
+    view[:, 4:8].copy_(torch.from_numpy(xb.copy()).to(dev))  # distinct xids
+    idx2 = ctx.index(1, n + 16, n + 16)
+    dsts = torch.empty((n, 4096), dtype=torch.uint8, device=dev)
+    outs = torch.empty((n, 1024), dtype=torch.int32, device=dev)
+    sts = torch.zeros(2 * n, dtype=torch.int32, device=dev)
+    reqs = []
+    for i in range(n):
+        reqs.append((int(xids[i]), 1, crk.K_OPAQUE_VAR, dsts[i].data_ptr(), 4096, None, sts.data_ptr() + 8 * i))
+        reqs.append((int(xids[i]), 3, crk.K_I32_VAR, outs[i].data_ptr(), 1024, None, sts.data_ptr() + 8 * i + 4))
+    arr = (crk.ItemReq * len(reqs))(*[crk.ItemReq(a, b, c_, 0, d, e, f, g) for a, b, c_, d, e, f, g in reqs])
+    dreq = torch.frombuffer(bytearray(arr), dtype=torch.uint8).to(dev)
+
+    def batch(_):
+        idx2.frame_scan([(big, 0, n * w)])
+        crk._check(crk.lib().crk_xdr_decode_items_batch(ctx.h, idx2.h, len(reqs), dreq.data_ptr(),
+                                                         torch.cuda.current_stream().cuda_stream), "batch")
+
+    bms = timed(batch, 5, warm=1)
+    ok2 = bool((sts == 0).all() and torch.equal(dsts[n - 1], data) and torch.equal(outs[12345], ints))
+    return {"latency_us": round(lat_ms * 1e3, 2), "ok": ok,
+            "note": "one record: crk_rpc_frame_scan (scan+parse) + crk_xdr_decode_opaque + crk_xdr_decode_array_i32",
+            "batch_records": n, "batch_ms": round(bms, 3), "records_per_s": round(n / bms * 1e3),
+            "batch_payload_gbs": round(n * 8192 / bms / 1e6, 1), "batch_ok": ok2}
+
+
+def c2(ctx):
+    A, B, C = gen.c2_matrices()
+    region = torch.zeros(4 * MiB, dtype=torch.uint8, device=dev)
+    base = region.data_ptr()
+    a = torch.from_numpy(A.view(np.uint8)).to(dev)
+    b = torch.from_numpy(B.view(np.uint8)).to(dev)
+    region[3 * MiB:3 * MiB + C.nbytes].copy_(torch.from_numpy(C.view(np.uint8)))
+    ring = crk.Ring.device(1 << 21)
+    cur = 0
+    cur += ctx.encode_call(1, gen.PROC_H2D, [(crk.K_U64, base), (crk.K_OPAQUE_VAR, a), (crk.K_U64, a.numel())], ring, cur)
+    cur += ctx.encode_call(2, gen.PROC_H2D, [(crk.K_U64, base + MiB), (crk.K_OPAQUE_VAR, b), (crk.K_U64, b.numel())],
+                           ring, cur)
+    cur += ctx.encode_call(3, gen.PROC_D2H, [(crk.K_U64, base + 3 * MiB), (crk.K_U64, C.nbytes)], ring, cur)
+    send = crk.Ring.device(1 << 21)
+    idx = ctx.index(1, 1024, 16)
+    ms = timed(lambda _: idx.serve([(ring, 0, cur)], [send], [0], base, region.numel()), 200)
+    ok = bool(torch.equal(region[:a.numel()], a) and torch.equal(region[MiB:MiB + b.numel()], b))
+    res = idx.ring_results(1)[0]
+    ok &= res["reply_bytes"] == crk.wire_size_d2h(C.nbytes, 0) + 2 * crk.wire_size_d2h(0, 1)
+    return {"us": round(ms * 1e3, 2), "bytes": int(A.nbytes + B.nbytes + C.nbytes), "wire_in": cur,
+            "reply_wire": res["reply_bytes"], "gbs": round((A.nbytes + B.nbytes + C.nbytes) / ms / 1e6, 2), "ok": ok}
+
+
+def c3(ctx, logs=(12, 14, 16, 18, 20, 22, 24, 26, 27, 28, 29, 30)):
+    out = []
+    for lg in logs:
+        n = 1 << lg
+        payload = torch.from_numpy(gen.c3_payload(lg)).to(dev)
+        one = crk.Ring.device(next_pow2(n + 4 * (n // 65536 + 2) + 64))
+        w = ctx.encode_call(lg, gen.PROC_H2D, [(crk.K_U64, 0), (crk.K_OPAQUE_VAR, payload), (crk.K_U64, n)], one, 0)
+        copies = max(1, min(64, (256 * MiB) // max(w, 1)))
+        rings = [one] + [crk.Ring.device(one.cap) for _ in range(copies - 1)]
+        for r in rings[1:]:
+            r.tensor()[:w].copy_(one.tensor()[:w])
+        dsts = [torch.empty(n, dtype=torch.uint8, device=dev) for _ in range(copies)]
+        idx = ctx.index(1, n // 65536 + 16, 4)
+        st = torch.zeros(1, dtype=torch.int32, device=dev)
+
+        def h2d(i):
+            k = i % copies
+            idx.frame_scan([(rings[k], 0, w)])
+            idx.decode_memcpy_h2d(lg, dsts[k], n, st)
+
+        reps = max(10, min(400, (GiB // n)))
+        ms = timed(h2d, reps)
+        ok = bool(torch.equal(dsts[(reps - 1) % copies], payload)) and st.item() == 0
+        outs = [crk.Ring.device(next_pow2(crk.wire_size_d2h(n, 0) + 64)) for _ in range(copies)]
+        srcs = [payload] + [payload.clone() for _ in range(copies - 1)]
+        wd = crk.wire_size_d2h(n, 0)
+        ms_d = timed(lambda i: ctx.encode_memcpy_d2h(lg, srcs[i % copies], 0, outs[i % copies], 0), reps)
+        out.append({"log2n": lg, "htod_gbs": round(n / ms / 1e6, 2), "htod_us": round(ms * 1e3, 2),
+                    "dtoh_gbs": round(n / ms_d / 1e6, 2), "dtoh_us": round(ms_d * 1e3, 2), "wire_in": w,
+                    "wire_out": wd, "ok": ok})
+        del rings, dsts, outs, srcs, payload
+        torch.cuda.empty_cache()
+    return out
+
+
+def c4(ctx, irregular):
+    for proc, items in gen.C4_SCHEMAS.items():
+        ctx.register_schema(proc, items)
+    calls = gen.c4_calls(256 * MiB)
+    ring = crk.Ring.device(1 << 29)
+    cur, keep, reqs, outs, srcs = 0, [], [], [], []
+    total = 0
+    for c in calls:
+        items = []
+        for code, v in c.items:
+            k = code & 0xFF
+            if k in (crk.K_U32, crk.K_U64):
+                items.append((code, v))
+                continue
+            t = torch.from_numpy(np.ascontiguousarray(v).view(np.uint8).copy()).to(dev)
+            if k not in (crk.K_OPAQUE_VAR, crk.K_OPAQUE_FIX):
+                t = t.view({4: torch.int32, 8: torch.int64}[crk.ELEM_SIZE[k]])
+            items.append((code, t))
+            keep.append(t)
+        lens = None
+        if irregular:
+            L = ctx.call_logical_size(items)
+            lens = gen.split_points(gen.frag_seed(c), L)
+        cur += ctx.encode_call(c.xid, c.proc, items, ring, cur, frag_lens=lens)
+        for a, (code, v) in enumerate(c.items):
+            k = code & 0xFF
+            if k in (crk.K_U32, crk.K_U64):
+                continue
+            nb = np.asarray(v).nbytes
+            o = torch.empty(nb + 16, dtype=torch.uint8, device=dev)
+            outs.append(o)
+            srcs.append(items[a][1])
+            reqs.append((c.xid, a, k, o.data_ptr(), len(v), None, None))
+            total += nb
+    torch.cuda.synchronize()
+    idx = ctx.index(1, 1 << 16, 1 << 12)
+    st = torch.zeros(len(reqs), dtype=torch.int32, device=dev)
+    arr = (crk.ItemReq * len(reqs))(*[crk.ItemReq(a, b, k, 0, d, m, None, st.data_ptr() + 4 * i)
+                                     for i, (a, b, k, d, m, _, _) in enumerate(reqs)])
+    dreq = torch.frombuffer(bytearray(arr), dtype=torch.uint8).to(dev)
+
+    def dec(_):
+        idx.frame_scan([(ring, 0, cur)])
+        crk._check(crk.lib().crk_xdr_decode_items_batch(ctx.h, idx.h, len(reqs), dreq.data_ptr(),
+                                                         torch.cuda.current_stream().cuda_stream), "batch")
+
+    ms = timed(dec, 10)
+    ok = bool((st == 0).all()) and all(torch.equal(o[:s.numel() * s.element_size()], s.view(torch.uint8).reshape(-1))
+                                       for o, s in zip(outs, srcs))
+    return {"records": len(calls), "items": len(reqs), "payload_bytes": total, "wire": cur, "ms": round(ms, 3),
+            "decode_gbs": round(total / ms / 1e6, 1), "ok": ok}
+
+
+def served(ctx, sizes_h2d, sizes_d2h, streams=1, reps=20):
+    """Serve a batch of HtoD records (sizes_h2d) and DtoH records over `streams` rings; GB/s of payload."""
+    total_h = sum(sizes_h2d)
+    region = torch.zeros(total_h + sum(sizes_d2h) + 4096 * (len(sizes_h2d) + len(sizes_d2h)), dtype=torch.uint8,
+                         device=dev)
+    base = region.data_ptr()
+    per = [[] for _ in range(streams)]
+    off = 0
+    srcs = []
+    for i, n in enumerate(sizes_h2d):
+        per[i % streams].append(("h", i, n, off))
+        off += (n + 255) // 256 * 256
+    for i, n in enumerate(sizes_d2h):
+        per[i % streams].append(("d", i, n, off))
+        region[off:off + n].copy_(torch.from_numpy(gen.random_bytes(7000 + i, n)))
+        off += (n + 255) // 256 * 256
+    rings, sends = [], []
+    for s in range(streams):
+        cap = next_pow2(sum(n + 64 + 4 * (n // 65536 + 2) for k, _, n, _ in per[s] if k == "h") + 64 * len(per[s]) + 4096)
+        ring = crk.Ring.device(cap)
+        cur = 0
+        for k, i, n, o in per[s]:
+            if k == "h":
+                p = torch.from_numpy(gen.random_bytes(9000 + i, n)).to(dev)
+                srcs.append((o, p))
+                cur += ctx.encode_call(0x1000 * s + i + 1, gen.PROC_H2D,
+                                       [(crk.K_U64, base + o), (crk.K_OPAQUE_VAR, p), (crk.K_U64, n)], ring, cur)
+            else:
+                cur += ctx.encode_call(0x800000 + 0x1000 * s + i, gen.PROC_D2H, [(crk.K_U64, base + o), (crk.K_U64, n)],
+                                       ring, cur)
+        rings.append((ring, 0, cur))
+        sends.append(crk.Ring.device(next_pow2(sum(crk.wire_size_d2h(n, 0) for k, _, n, _ in per[s] if k == "d")
+                                               + 64 * len(per[s]) + 4096)))
+    idx = ctx.index(streams, 1 << 20, 1 << 14)
+    ms = timed(lambda _: idx.serve(rings, sends, [0] * streams, base, region.numel()), reps)
+    ok = all(r["status"] == 0 for r in idx.ring_results(streams))
+    ok &= all(bool(torch.equal(region[o:o + p.numel()], p)) for o, p in srcs[:4])
+    pay = total_h + sum(sizes_d2h)
+    return {"ms": round(ms, 4), "payload_bytes": pay, "gbs": round(pay / ms / 1e6, 1), "ok": bool(ok)}
+
+
+def main():
+    build.build()
+    out = {}
+    ctx = crk.Context(0)
+    t0 = time.time()
+    out["C1"] = c1(ctx)
+    out["C2_matrixMul"] = c2(crk.Context(0))
+    out["C3_sweep"] = c3(crk.Context(0))
+    out["C4_typed_regular"] = c4(crk.Context(0), False)
+    out["C4_typed_irregular"] = c4(crk.Context(0), True)
+    out["NEXT1_striped_1GiB_16_rings"] = served(crk.Context(0), [64 * MiB] * 16, [], streams=16)
+    out["NEXT1_single_1GiB_1_ring"] = served(crk.Context(0), [GiB], [], streams=1)
+    out["NEXT2_cusolver_100_iters"] = served(crk.Context(0), [900 * 900 * 8] * 100, [900 * 8] * 100, streams=1, reps=10)
+    out["NEXT2_histogram"] = served(crk.Context(0), [64 * MiB], [256 * 4], streams=1)
+    out["wall_s"] = round(time.time() - t0, 1)
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()
