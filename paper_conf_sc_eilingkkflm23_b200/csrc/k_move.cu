@@ -352,6 +352,107 @@ __device__ __forceinline__ void staged_chunks(const Team& T, const uint8_t* buf,
   }
 }
 
+
+// ------------------------------------------------------------------------------------------- producer state
+constexpr uint32_t kWin = 64;  // fragment entries cached per producer
+struct ProdCache {
+  Job job;
+  Piece pieces[kMaxPieces];
+  RingDesc R;                 // DEC: the record's ring; ENC: the output ring
+  uint64_t rec_len, F0;
+  uint32_t frag0, nfrags;     // absolute index of the record's first fragment, fragment count
+  uint32_t wk0, wn;           // window: fragments [wk0, wk0 + wn) of the record
+  uint32_t hint;
+  uint64_t lstart[kWin], phys[kWin];
+  uint32_t hdr[kWin];
+};
+
+// Loads job j (and its pieces / ring / record) into the producer cache; the whole warp calls it.
+__device__ __forceinline__ void producer_load_job(ProdCache& pc, const MoveParams& M, uint32_t j, uint32_t lane) {
+  if (lane < sizeof(Job) / 4)
+    reinterpret_cast<uint32_t*>(&pc.job)[lane] = reinterpret_cast<const uint32_t*>(M.sc.jobs + j)[lane];
+  __syncwarp();
+  const Job& J = pc.job;
+  if (J.type == JOB_ENC) {
+    for (uint32_t i = lane; i < J.n_pieces * (sizeof(Piece) / 4); i += 32)
+      reinterpret_cast<uint32_t*>(pc.pieces)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + J.piece0)[i];
+    if (lane == 0) pc.R = M.sc.out_rings[J.out_ring];
+  } else if (J.type == JOB_DEC && lane == 0) {
+    const uint32_t slot = M.ix.p_slot[J.rec], ring = M.ix.p_ring[J.rec];
+    pc.R = M.ix.rings[ring];
+    pc.frag0 = M.ix.rec_frag0[slot];
+    pc.nfrags = M.ix.rec_nfrags[slot];
+    pc.rec_len = M.ix.rec_len[slot];
+    pc.F0 = M.ix.frag_hdr[pc.frag0] & 0x7fffffffu;
+    pc.wn = 0;
+    pc.hint = 0;
+  }
+  __syncwarp();
+}
+
+__device__ __forceinline__ void producer_frag(const ProdCache& pc, const MoveParams& M, uint32_t k, uint64_t& ls,
+                                              uint64_t& ph, uint32_t& hd) {
+  if (k >= pc.wk0 && k < pc.wk0 + pc.wn) {
+    const uint32_t i = k - pc.wk0;
+    ls = pc.lstart[i]; ph = pc.phys[i]; hd = pc.hdr[i];
+  } else {
+    const uint64_t g = (uint64_t)pc.frag0 + k;
+    ls = M.ix.frag_lstart[g]; ph = M.ix.frag_phys[g]; hd = M.ix.frag_hdr[g];
+  }
+}
+
+// Fragment holding logical offset `off` of the current record; makes sure the window covers it and
+// the next kMaxSeg fragments.  The whole warp calls it; lane 0's answer is returned to every lane.
+__device__ uint32_t producer_frag_window(ProdCache& pc, const MoveParams& M, uint64_t off, uint32_t lane) {
+  uint32_t k0 = 0;
+  if (lane == 0) {
+    auto holds = [&](uint32_t k) {
+      uint64_t ls, ph;
+      uint32_t hd;
+      producer_frag(pc, M, k, ls, ph, hd);
+      return off >= ls && off < ls + (hd & 0x7fffffffu);
+    };
+    const uint32_t n = pc.nfrags;
+    uint32_t k = pc.hint;
+    bool found = k < n && holds(k);
+    for (uint32_t i = 1; !found && i <= 2 && k + i < n; ++i)
+      if (holds(k + i)) { k += i; found = true; }
+    if (!found && pc.F0) {
+      const uint64_t g = off / pc.F0;
+      if (g < n && holds((uint32_t)g)) { k = (uint32_t)g; found = true; }
+    }
+    if (!found) {  // binary search over the record's fragments: largest k with lstart[k] <= off
+      uint32_t lo = 0, hi = n;
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        uint64_t ls, ph;
+        uint32_t hd;
+        producer_frag(pc, M, mid, ls, ph, hd);
+        if (ls <= off) lo = mid; else hi = mid;
+      }
+      k = lo;
+    }
+    pc.hint = k;
+    k0 = k;
+  }
+  k0 = __shfl_sync(0xffffffffu, k0, 0);
+  const uint32_t n = pc.nfrags;
+  const uint32_t want_end = min(n, k0 + kMaxSeg + 1);
+  if (!(k0 >= pc.wk0 && want_end <= pc.wk0 + pc.wn)) {
+    __syncwarp();
+    const uint32_t base = k0, cnt = min(kWin, n - base);
+    for (uint32_t i = lane; i < cnt; i += 32) {
+      const uint64_t g = (uint64_t)pc.frag0 + base + i;
+      pc.lstart[i] = M.ix.frag_lstart[g];
+      pc.phys[i] = M.ix.frag_phys[g];
+      pc.hdr[i] = M.ix.frag_hdr[g];
+    }
+    if (lane == 0) { pc.wk0 = base; pc.wn = cnt; }
+    __syncwarp();
+  }
+  return k0;
+}
+
 // ------------------------------------------------------------------------------------------- kernel
 __device__ __forceinline__ uint32_t find_job(const uint64_t* prefix, uint32_t n_jobs, uint64_t tile, uint32_t lane) {
   uint32_t lo = 0, hi = n_jobs;  // last j with prefix[j] <= tile (32-ary search, one warp)
@@ -391,10 +492,12 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
 
   if (warp == 0) {
     // ------------------------------------------------ producer
-    // Tiles are claimed in runs of kRun consecutive tiles, so the job lookup and the record state are
-    // paid once per run and the fragment walk continues from the previous tile's fragment.
+    // Tiles are claimed in runs of kRun consecutive tiles.  The job, its pieces / ring and (decode) the
+    // record's fragment table window live in producer-private shared memory: a job is loaded once, and
+    // a window of kWin fragment entries is refilled by the whole warp in one round trip, so a tile's
+    // descriptor costs no dependent global loads in the common case.
+    __shared__ ProdCache pc;
     uint32_t k = 0, claims = 0;
-    DecCtx dc;
     for (;;) {
       uint64_t t0 = ~0ull, t1 = 0;
       if (lane == 0) {
@@ -429,28 +532,30 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           pnext = j + 1 < n_jobs ? M.prefix[j + 1] : ~0ull;
           fresh = true;
         }
+        if (fresh) producer_load_job(pc, M, j, lane);
+        const Job& J = pc.job;
+        const uint64_t t = tile - pj;
+        const uint64_t A = J.out_start >> shf;
+        const uint64_t a = max(J.out_start, (A + t) << shf), b = min(J.out_end, (A + t + 1) << shf);
+        uint32_t k0 = 0;
+        if (J.type == JOB_DEC) k0 = producer_frag_window(pc, M, J.loff + (a - J.out_start), lane);
         const uint32_t s = k % kStages;
         StageHdr& H = *reinterpret_cast<StageHdr*>(smem + s * stage_stride);
         uint8_t* buf = smem + s * stage_stride + (sizeof(StageHdr) + 127) / 128 * 128;
         mbar_wait(&empty[s], ((k / kStages) & 1) ^ 1);
-        // job + pieces into the stage header
-        if (lane < sizeof(Job) / 4)
-          reinterpret_cast<uint32_t*>(&H.job)[lane] = reinterpret_cast<const uint32_t*>(M.sc.jobs + j)[lane];
-        __syncwarp();
-        const Job& J = H.job;
+        // job + pieces into the stage header (shared -> shared)
+        if (lane < sizeof(Job) / 4) reinterpret_cast<uint32_t*>(&H.job)[lane] = reinterpret_cast<const uint32_t*>(&J)[lane];
         if (J.type == JOB_ENC)
           for (uint32_t i = lane; i < J.n_pieces * (sizeof(Piece) / 4); i += 32)
-            reinterpret_cast<uint32_t*>(H.pieces)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + J.piece0)[i];
+            reinterpret_cast<uint32_t*>(H.pieces)[i] = reinterpret_cast<const uint32_t*>(pc.pieces)[i];
         __syncwarp();
         if (lane != 0) mbar_arrive(&full[s]);  // lanes 1-31 are done writing this stage
         if (lane == 0) {
-        const uint64_t t = tile - pj;
-        const uint64_t A = J.out_start >> shf;
-        const uint64_t a = max(J.out_start, (A + t) << shf), b = min(J.out_end, (A + t + 1) << shf);
         H.type = J.type;
         H.a = a;
         H.b = b;
         H.fallback = 0;
+        H.R = pc.R;
         uint32_t nseg = 0, bytes = 0;
         const uint32_t cap = M.stage_bytes;
         // copies are collected first and issued after expect_tx
@@ -474,28 +579,29 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           bytes += len;
         };
         if (J.type == JOB_DEC) {
-          if (fresh) dec_ctx_init(dc, M.ix, J);
-          DecCtx& c = dc;
-          H.R = c.L.R;
-          uint32_t kf = c.L.find(c.loff + (a - c.dst));
-          H.k0 = kf;
+          H.k0 = k0;
+          const uint64_t dst = J.out_start, loff = J.loff;
           uint64_t r = a;
+          uint32_t kf = k0;
           bool ok = true;
-          while (r < b && kf < c.L.nfrags) {
-            const uint64_t ls = c.L.lstart[kf], fl = c.L.flen(kf), ph = c.L.phys[kf];
-            const uint64_t sb = min(b, c.dst + (ls + fl - c.loff));
+          while (r < b && kf < pc.nfrags) {
+            uint64_t ls, ph;
+            uint32_t hd;
+            producer_frag(pc, M, kf, ls, ph, hd);
+            const uint64_t fl = hd & 0x7fffffffu;
+            const uint64_t sb = min(b, dst + (ls + fl - loff));
             if (sb > r) {
               if (nseg == kMaxSeg) { ok = false; break; }
               Seg& g = H.seg[nseg++];
               g.out_a = r;
               g.out_b = sb;
-              g.src = ph + (c.loff + (r - c.dst) - ls);
+              g.src = ph + (loff + (r - dst) - ls);
               g.flags = (SEG_DATA << 8) | (J.esize << 16);
               const uint64_t c0 = (r + 15) & ~15ull, c1 = sb & ~15ull;
               if (c0 < c1) {  // stage the source window of the interior chunks
                 const uint64_t s0 = g.src + (c0 - r);
                 const uint64_t w0 = s0 & ~15ull, w1 = (s0 + (c1 - c0) + 15) & ~15ull;
-                stage_window(g, c.L.R.base, c.L.R.mask, true, w0, w1);
+                stage_window(g, pc.R.base, pc.R.mask, true, w0, w1);
               }
               r = sb;
             }
@@ -504,9 +610,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           if (!ok) { H.fallback = 1; nseg = 0; nc = 0; bytes = 0; }
         } else if (J.type == JOB_ENC) {
           EncCtx c;
-          const RingDesc O = M.sc.out_rings[J.out_ring];
-          enc_ctx_init(c, M.sc, J, O, H.pieces);
-          H.R = O;
+          enc_ctx_init(c, M.sc, J, pc.R, pc.pieces);
           const bool ok = enc_runs(c, a - c.start, b - c.start,
                                    [&](uint32_t kind, uint64_t wa, uint64_t wb, uint64_t src, uint32_t es) {
             if (kind == SEG_LIT && nseg > 0 && (H.seg[nseg - 1].flags >> 8 & 0xff) == SEG_LIT &&
