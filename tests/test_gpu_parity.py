@@ -559,3 +559,93 @@ def test_ring_copy_and_async_results():
     rows = out.rows()
     assert rows == idx.ring_results(2)
     assert rows[0]["status"] == O.OK and rows[0]["n_records"] == 1 and rows[1]["status"] == O.INCOMPLETE
+
+
+@pytest.mark.parametrize("strict", [True, False])
+def test_serve_cred_bodies_lenient_and_duplicates_match_oracle(strict):
+    """Non-empty cred/verf bodies (args start past the prefetched head), odd pads, lenient mode."""
+    cfg = ocfg(strict=strict, F=3000)
+    ctx = ctx_for(cfg)
+    region = torch.zeros(1 << 20, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    host_region = np.zeros(1 << 20, np.uint8)
+    host_region[500000:600000] = gen.random_bytes(4, 100000)
+    region.copy_(torch.from_numpy(host_region))
+    g = gen.rng(31)
+    wires = []
+    for i in range(40):
+        cl, vl = int(g.integers(0, 401)), int(g.integers(0, 401))
+        cred = (1, gen.random_bytes(i, cl).tobytes())
+        verf = (6, gen.random_bytes(i + 99, vl).tobytes())
+        if i % 3 == 0:
+            L = O.call_header(100 + i, gen.PROG, gen.VERS, gen.PROC_D2H, cred, verf) + O.put_u64(base + 500000 + i) + \
+                O.put_u64(int(g.integers(0, 90000)))
+        else:
+            n = int(g.integers(0, 5000))
+            size = n if i % 5 else n + 3          # strict: E_SIZE; lenient: copies min(n, size)
+            L = O.call_header(100 + i, gen.PROG, gen.VERS, gen.PROC_H2D, cred, verf) + O.put_u64(base + 7000 * i) + \
+                O.put_opaque_var(gen.random_bytes(i + 7, n).tobytes()) + O.put_u64(size)
+            if i % 7 == 0:
+                L += b"\0" * 8                     # trailing bytes: strict E_TRAILING, lenient ignored
+        wires.append(O.frame(L, int(g.integers(7, 3000))))
+    wires.append(wires[5])                         # duplicate xid (reading R11)
+    ring = make_ring(1 << 21)
+    tail = 0
+    for w in wires:
+        tail = place(ring, w, tail)
+    send = make_ring(1 << 22)
+    idx = ctx.index(1, 1 << 14, 256)
+    idx.serve([(ring, 0, tail)], [send], [40], base, region.numel())
+    torch.cuda.synchronize()
+    T = idx.tables(1)
+    want = O.serve([(ring_np(ring), 0, tail)], cfg, host_region, base, [1 << 22], [40], max_frags_per_ring=1 << 14,
+                   max_records_per_ring=256)
+    assert [r["status"] for r in want["records"]] == list(T["parsed"]["serve_status"])
+    assert [r["reply_err"] for r in want["records"]] == list(T["parsed"]["serve_reply_err"])
+    assert np.array_equal(region.cpu().numpy(), host_region)
+    n = want["reply_bytes"][0]
+    assert T["rings"][0]["reply_bytes"] == n
+    assert send.read(40, n) == bytes(want["send"][0][40:40 + n])
+
+
+def test_serve_rejects_index_larger_than_job_scratch():
+    ctx = crk.Context(0, max_jobs=64)
+    idx = ctx.index(1, 256, 64)  # serve needs 2 jobs per record
+    ring = make_ring(1 << 12)
+    with pytest.raises(crk.CrkError) as e:
+        idx.serve([(ring, 0, 0)], [make_ring(1 << 12)], [0], 0, 0)
+    assert e.value.status == crk.E_CAPACITY
+
+
+def test_staged_e2e_path_matches_oracle():
+    """Copy-engine mode: host ring -> crk_ring_copy -> serve from HBM -> crk_ring_copy replies -> host."""
+    cfg = ocfg(F=8192)
+    ctx = ctx_for(cfg)
+    region = torch.zeros(1 << 22, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    host_region = np.zeros(1 << 22, np.uint8)
+    host_region[1 << 21:(1 << 21) + 300000] = gen.random_bytes(8, 300000)
+    region.copy_(torch.from_numpy(host_region))
+    hring, dring = crk.Ring.host(1 << 20), crk.Ring.device(1 << 20)
+    head = (1 << 20) - 5000
+    cur = head
+    for i in range(12):
+        if i % 2:
+            c = d2h_call(i + 1, base + (1 << 21) + 1000 * i, 20000 + 977 * i)
+        else:
+            c = h2d_call(i + 1, gen.random_bytes(i, 30000 + 311 * i), base + 40000 * i)
+        cur = place(hring, O.encode_call(*c, cfg, F=8192), cur)
+    hsend, dsend = crk.Ring.host(1 << 20), crk.Ring.device(1 << 20)
+    crk.ring_copy(dring, hring, head, cur)
+    idx = ctx.index(1, 1024, 64)
+    idx.serve([(dring, head, cur)], [dsend], [77], base, region.numel())
+    res = crk.PinnedResults(1)
+    idx.ring_results_async(res)
+    torch.cuda.synchronize()
+    n = res.rows()[0]["reply_bytes"]
+    crk.ring_copy(hsend, dsend, 77, 77 + n)
+    torch.cuda.synchronize()
+    want = O.serve([(hring.host_view().copy(), head, cur)], cfg, host_region, base, [1 << 20], [77])
+    assert n == want["reply_bytes"][0]
+    assert hsend.read(77, n) == bytes(want["send"][0][77:77 + n])
+    assert np.array_equal(region.cpu().numpy(), host_region)
