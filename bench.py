@@ -42,7 +42,7 @@ def parse_args():
     p.add_argument("--impl", default="crk", choices=["crk", "reference"])
     p.add_argument("--streams", type=int, default=16)
     p.add_argument("--payload-mib", type=int, default=64, help="payload per stream")
-    p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--e2e-steps", type=int, default=30)
     p.add_argument("--pipeline", type=int, default=3, help="batches in flight (server loop slots)")
     p.add_argument("--e2e-pipeline", type=int, default=3, help="batches in flight for the host-memory runs")
     p.add_argument("--no-e2e", action="store_true")

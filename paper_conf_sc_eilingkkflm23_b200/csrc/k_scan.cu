@@ -31,9 +31,9 @@ struct ScanState {
   int32_t status;
   uint64_t consumed;
   uint32_t kept_frags;
-  uint32_t valid_star, h_star, wide;
-  uint32_t code_f;
-  uint32_t gmin[32];
+  uint32_t wide;
+  uint32_t gmin[32], gh[32], gv[32];  // per warp: first mismatch, its header, its validity
+  uint32_t fmin[32], fcode[32];       // per warp: first failing check and its code
 };
 
 __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
@@ -65,41 +65,50 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     // a round uses kJ candidates per thread only after a round that accepted every candidate (a long
     // regular run: big records); otherwise one, which keeps the round short
     const uint32_t jn = S.wide ? kJ : 1u, TT = T * jn;
-    uint32_t hv[kJ];
+    uint32_t hv[kJ], w0[kJ], w1[kJ];
     bool vv[kJ];
     uint32_t first_bad = TT;
+    // all candidate loads are issued before any is used: each header is read as the two aligned words
+    // that contain it (branch-free, any alignment, across the wrap) and joined by a funnel shift
+#pragma unroll
+    for (uint32_t j = 0; j < kJ; ++j) {
+      const uint64_t q = p + (uint64_t)(u + j * T) * stride;
+      vv[j] = j < jn && q + 4 <= R.tail;
+      const uint64_t a = q & ~3ull;
+      w0[j] = vv[j] ? __ldg(reinterpret_cast<const uint32_t*>(R.base + (a & R.mask))) : 0u;
+      w1[j] = vv[j] ? __ldg(reinterpret_cast<const uint32_t*>(R.base + ((a + 4) & R.mask))) : 0u;
+    }
+    uint32_t bh = 0, bv = 0;  // header and validity of this thread's first mismatching candidate
 #pragma unroll
     for (uint32_t j = 0; j < kJ; ++j) {
       const uint32_t t = u + j * T;
-      if (j >= jn) { vv[j] = false; hv[j] = 0; continue; }
       const uint64_t q = p + (uint64_t)t * stride;
-      vv[j] = q + 4 <= R.tail;
-      hv[j] = vv[j] ? ring_be32(R, q) : 0u;
-      if (!(vv[j] && hv[j] == hpred)) first_bad = min(first_bad, t);
+      hv[j] = bswap32(__funnelshift_r(w0[j], w1[j], 8 * (uint32_t)(q & 3)));
+      if (j < jn && first_bad == TT && !(vv[j] && hv[j] == hpred)) { first_bad = t; bh = hv[j]; bv = vv[j]; }
     }
-    // per-group first mismatch (groups are whole warps)
-    uint32_t wm = __reduce_min_sync(0xffffffffu, first_bad);
-    if (lane == 0) S.gmin[warp] = wm;
+    // per-group first mismatch (groups are whole warps); the warp publishes the mismatching header too
+    const uint32_t wm = __reduce_min_sync(0xffffffffu, first_bad);
+    const uint32_t own = __ffs(__ballot_sync(0xffffffffu, first_bad == wm)) - 1;
+    const uint32_t oh = __shfl_sync(0xffffffffu, bh, own), ov = __shfl_sync(0xffffffffu, bv, own);
+    if (lane == 0) { S.gmin[warp] = wm; S.gh[warp] = oh; S.gv[warp] = ov; }
     __syncthreads();
-    uint32_t ts0 = TT, ts1 = TT;
+    uint32_t ts0 = TT, ts1 = TT, ws0 = 0, ws1 = 0;
     for (uint32_t w = 0; w < nw; ++w) {
-      if (w < wpg) ts0 = min(ts0, S.gmin[w]);
-      else ts1 = min(ts1, S.gmin[w]);
+      const uint32_t g = S.gmin[w];
+      if (w < wpg) { if (g < ts0) { ts0 = g; ws0 = w; } }
+      else if (g < ts1) { ts1 = g; ws1 = w; }
     }
     // the group with the longer verified run wins (ties: group 0)
     const uint32_t win = ts1 > ts0;
     const uint32_t tstar = win ? ts1 : ts0;
+    const uint32_t wstar = win ? ws1 : ws0;
     const bool mine = grp == win;
-#pragma unroll
-    for (uint32_t j = 0; j < kJ; ++j)
-      if (mine && u + j * T == tstar) { S.valid_star = vv[j]; S.h_star = hv[j]; }
-    __syncthreads();
     hpred = S.hp[win];
     const uint64_t Lp = hpred & 0x7fffffffu;
     const uint32_t lastp = hpred >> 31;
-    const bool end_at_star = tstar < TT && !S.valid_star;
+    const bool end_at_star = tstar < TT && !S.gv[wstar];
     const uint32_t n_hdr = tstar == TT ? TT : (end_at_star ? tstar : tstar + 1);
-    const uint32_t hstar = S.h_star;
+    const uint32_t hstar = S.gh[wstar];
 
     // per-header closed forms (headers 0..tstar-1 equal hpred); checks in the oracle's order
     uint32_t codes[kJ];
@@ -121,17 +130,20 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
         else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
       }
       codes[j] = code;
-      if (code != STOP_NONE) first_fail = min(first_fail, t);
+      if (code != STOP_NONE && first_fail == 0xffffffffu) first_fail = t;
     }
-    wm = __reduce_min_sync(0xffffffffu, first_fail);
-    if (lane == 0) S.gmin[warp] = wm;
-    __syncthreads();
-    uint32_t tf = 0xffffffffu;
-    for (uint32_t w = 0; w < nw; ++w) tf = min(tf, S.gmin[w]);
+    uint32_t my_code = STOP_NONE;
 #pragma unroll
     for (uint32_t j = 0; j < kJ; ++j)
-      if (mine && u + j * T == tf) S.code_f = codes[j];
+      if (u + j * T == first_fail) my_code = codes[j];
+    const uint32_t fm = __reduce_min_sync(0xffffffffu, first_fail);
+    const uint32_t fown = __ffs(__ballot_sync(0xffffffffu, first_fail == fm)) - 1;
+    const uint32_t fc = __shfl_sync(0xffffffffu, my_code, fown);
+    if (lane == 0) { S.fmin[warp] = fm; S.fcode[warp] = fc; }
     __syncthreads();
+    uint32_t tf = 0xffffffffu, code_f = STOP_NONE;
+    for (uint32_t w = 0; w < nw; ++w)
+      if (S.fmin[w] < tf) { tf = S.fmin[w]; code_f = S.fcode[w]; }
     const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
 
 #pragma unroll
@@ -167,7 +179,7 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
         S.kept_frags = start ? nf + t : f0;
         S.nr = nrec;
         if (tf < n_hdr) {
-          const uint32_t c = S.code_f;
+          const uint32_t c = code_f;
           S.status = c == STOP_FRAG ? CRK_E_FRAG
                    : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
                    : (nrec > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
