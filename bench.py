@@ -215,10 +215,17 @@ def main():
     from paper_conf_sc_eilingkkflm23_b200 import build, crk, parallel, workload
 
     world, rank, local = parallel.rank_env()
+    ndev = torch.cuda.device_count()
+    shared_gpu = world > ndev  # more ranks than GPUs (plumbing tests): ranks share devices, gloo plumbing
+    local = local % ndev
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        if shared_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
+    red_dev = "cpu" if shared_gpu else dev
     build.build()
 
     ctx_kw = {k: int(v, 0) for k, v in (kv.split("=") for kv in args.ctx.split(",") if kv)}
@@ -227,10 +234,10 @@ def main():
         parallel.barrier(dev)
 
     def max_over_ranks(x: float) -> float:
-        return parallel.max_over_ranks(x, dev)
+        return parallel.max_over_ranks(x, red_dev)
 
     def sum_over_ranks(x: float) -> float:
-        return parallel.sum_over_ranks(x, dev)
+        return parallel.sum_over_ranks(x, red_dev)
 
     # A server loop keeps `pipeline` batches in flight: each slot is a (context, index, stream, batch
     # buffers) set, so the front end (scan / parse / plan) of batch k+1 runs while the mover of batch k
