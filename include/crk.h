@@ -285,6 +285,19 @@ int crk_serve(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* ri
               const uint64_t* tails, const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
               uint64_t region_bytes, crk_stream_t stream);
 
+/* A server step captured once as a CUDA graph and replayed as the rings advance (the server loop).
+ * The ring cursors are read by the kernels at execution time from `doorbell` (device or mapped pinned
+ * memory, uint64 [heads 0..n-1 | tails 0..n-1 | send_offs 0..n-1]), so a replay serves whatever
+ * windows the host has published there; a ring whose published window is invalid (tail < head or
+ * longer than its capacity) gets status CRK_E_ARG and no records.  Everything else (rings, send rings,
+ * region, index, context) is fixed at capture.  The graph owns no memory of its own. */
+typedef struct crk_graph crk_graph;
+int crk_serve_graph_create(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings,
+                           const crk_ring* send_rings, uint64_t region_base, uint64_t region_bytes,
+                           const uint64_t* doorbell, crk_graph** out);
+int crk_graph_launch(crk_graph* graph, crk_stream_t stream);
+void crk_graph_destroy(crk_graph* graph);
+
 /* ---------------------------------------------------------------- memory utilities
  * Pinned, mapped, portable host memory for rings (cudaHostAlloc; with UVA the returned pointer is
  * also the device address), and a synchronous device->host copy for inspecting index tables. */

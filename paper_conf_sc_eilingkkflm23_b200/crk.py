@@ -109,6 +109,10 @@ def lib():
             "crk_call_logical_size": (u64, [C.POINTER(ItemSrc), u32]),
             "crk_serve": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(u64), C.POINTER(u64), C.POINTER(CRing),
                                     C.POINTER(u64), u64, u64, vp]),
+            "crk_serve_graph_create": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(CRing), u64, u64, vp,
+                                                 C.POINTER(vp)]),
+            "crk_graph_launch": (C.c_int, [vp, vp]),
+            "crk_graph_destroy": (None, [vp]),
             "crk_host_alloc": (C.c_int, [u64, C.POINTER(vp)]),
             "crk_host_free": (None, [vp]),
             "crk_copy_to_host": (C.c_int, [vp, vp, u64]),
@@ -429,6 +433,11 @@ class Index:
                                _stream(stream)), "crk_serve")
         self.n_rings = n
 
+    def serve_graph(self, rings, send_rings, region_base: int, region_bytes: int, doorbell) -> "ServeGraph":
+        """Captures one server step reading its cursors from `doorbell` (a device uint64 tensor or a
+        HostBuffer of 3 * n_rings uint64: heads | tails | send offsets)."""
+        return ServeGraph(self, rings, send_rings, region_base, region_bytes, doorbell)
+
     def ring_results(self, n: int | None = None, stream=None) -> list[dict]:
         n = self.n_rings if n is None else n
         out = (RingResult * max(1, n))()
@@ -503,3 +512,34 @@ class Index:
         _check(lib().crk_xdr_decode_items_batch(self.ctx.h, self.h, n, dev.data_ptr(), _stream(stream)),
                "crk_xdr_decode_items_batch")
         return dev
+
+
+class ServeGraph:
+    """crk_serve_graph_create / crk_graph_launch: a captured server step driven by a cursor doorbell."""
+
+    def __init__(self, idx: Index, rings, send_rings, region_base: int, region_bytes: int, doorbell):
+        n = len(rings)
+        cr = (CRing * n)(*[r.c() for r in rings])
+        sr = (CRing * n)(*[r.c() for r in send_rings])
+        self.doorbell = doorbell
+        ptr = doorbell.ptr if isinstance(doorbell, HostBuffer) else doorbell.data_ptr()
+        h = vp()
+        _check(lib().crk_serve_graph_create(idx.ctx.h, idx.h, n, cr, sr, region_base, region_bytes, ptr, C.byref(h)),
+               "crk_serve_graph_create")
+        self.h = h.value
+        self.idx = idx
+        idx.n_rings = n
+
+    def launch(self, stream=None):
+        _check(lib().crk_graph_launch(self.h, _stream(stream)), "crk_graph_launch")
+
+    def close(self):
+        if self.h:
+            lib().crk_graph_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

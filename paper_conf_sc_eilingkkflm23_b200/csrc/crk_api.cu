@@ -112,14 +112,21 @@ void add_builtin(SchemaTable& t, uint32_t proc, std::initializer_list<uint32_t> 
 }
 
 int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
-             const uint64_t* tails, cudaStream_t s) {
-  if (!rings || !heads || !tails || n_rings == 0 || n_rings > (uint32_t)kMaxRings || n_rings > idx->ix.max_rings)
+             const uint64_t* tails, cudaStream_t s, const uint64_t* doorbell = nullptr) {
+  if (!rings || (!doorbell && (!heads || !tails)) || n_rings == 0 || n_rings > (uint32_t)kMaxRings ||
+      n_rings > idx->ix.max_rings)
     return CRK_E_ARG;
   ScanRingsParam P;
   memset(&P, 0, sizeof(P));
   P.n_rings = n_rings;
+  P.doorbell = doorbell;
   for (uint32_t r = 0; r < n_rings; ++r) {
-    if (!ring_ok(rings[r]) || tails[r] < heads[r] || tails[r] - heads[r] > rings[r].cap) return CRK_E_ARG;
+    if (!ring_ok(rings[r])) return CRK_E_ARG;
+    if (doorbell) {
+      P.r[r] = ring_desc(rings[r], 0, 0);  // cursors come from the doorbell at execution time
+      continue;
+    }
+    if (tails[r] < heads[r] || tails[r] - heads[r] > rings[r].cap) return CRK_E_ARG;
     P.r[r] = ring_desc(rings[r], heads[r], tails[r]);
   }
   CK(cudaMemsetAsync(idx->ix.xid_hash, 0xff, sizeof(unsigned long long) * ((uint64_t)idx->ix.hash_mask + 1), s));
@@ -655,19 +662,93 @@ int crk_rpc_encode_call(crk_ctx* c, uint32_t xid, uint32_t proc, const crk_item_
   return move(c, nullptr, 1, s, wire);
 }
 
-int crk_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
+}  // extern "C"
+
+namespace {
+int run_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
               const uint64_t* tails, const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
-              uint64_t region_bytes, crk_stream_t stream) {
-  if (!c || !x || x->ctx != c || !send_rings || !send_offs) return CRK_E_ARG;
+              uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s) {
+  if (!c || !x || x->ctx != c || !send_rings || (!send_offs && !doorbell)) return CRK_E_ARG;
   if (2ull * x->ix.max_records > c->sc.max_jobs) return CRK_E_CAPACITY;
   for (uint32_t r = 0; r < n_rings && r < (uint32_t)kMaxRings; ++r)
     if (!ring_ok(send_rings[r])) return CRK_E_ARG;
-  DeviceGuard g(c->device);
-  cudaStream_t s = (cudaStream_t)stream;
-  int st = run_scan(c, x, n_rings, rings, heads, tails, s);
+  int st = run_scan(c, x, n_rings, rings, heads, tails, s, doorbell);
   if (st != CRK_OK) return st;
-  CK(launch_serve_plan(x->ix, c->cd, c->sc, n_rings, send_rings, send_offs, region_base, region_bytes, s));
+  CK(launch_serve_plan(x->ix, c->cd, c->sc, n_rings, send_rings, send_offs, region_base, region_bytes, doorbell,
+                       s));
   return move(c, &x->ix, 2 * x->ix.max_records, s);
+}
+}  // namespace
+
+struct crk_graph {
+  crk_ctx* ctx;
+  cudaGraph_t graph;
+  cudaGraphExec_t exec;
+  int launches;  // kernels per replay
+};
+
+extern "C" {
+
+int crk_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
+              const uint64_t* tails, const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
+              uint64_t region_bytes, crk_stream_t stream) {
+  if (!c) return CRK_E_ARG;
+  DeviceGuard g(c->device);
+  return run_serve(c, x, n_rings, rings, heads, tails, send_rings, send_offs, region_base, region_bytes, nullptr,
+                   (cudaStream_t)stream);
+}
+
+int crk_serve_graph_create(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings,
+                           const crk_ring* send_rings, uint64_t region_base, uint64_t region_bytes,
+                           const uint64_t* doorbell, crk_graph** out) {
+  if (!c || !x || !doorbell || !out) return CRK_E_ARG;
+  *out = nullptr;
+  DeviceGuard g(c->device);
+  cudaStream_t s;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  const bool prof = g_prof.on;
+  g_prof.on = false;  // no event nodes inside the graph
+  const int l0 = crk::g_launches.load();
+  cudaError_t e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+  int st = CRK_OK;
+  if (e == cudaSuccess)
+    st = run_serve(c, x, n_rings, rings, nullptr, nullptr, send_rings, nullptr, region_base, region_bytes, doorbell, s);
+  cudaGraph_t graph = nullptr;
+  const cudaError_t e2 = cudaStreamEndCapture(s, &graph);
+  g_prof.on = prof;
+  const int nk = crk::g_launches.load() - l0;
+  crk::g_launches.fetch_sub(nk);  // launches are counted when the graph is replayed
+  cudaStreamDestroy(s);
+  if (e != cudaSuccess) return cuda_fail(e);
+  if (st != CRK_OK) { if (graph) cudaGraphDestroy(graph); return st; }
+  if (e2 != cudaSuccess) return cuda_fail(e2);
+  cudaGraphExec_t exec;
+  e = cudaGraphInstantiate(&exec, graph, 0);
+  if (e != cudaSuccess) { cudaGraphDestroy(graph); return cuda_fail(e); }
+  crk_graph* G = new (std::nothrow) crk_graph;
+  if (!G) { cudaGraphExecDestroy(exec); cudaGraphDestroy(graph); return CRK_E_CAPACITY; }
+  G->ctx = c;
+  G->graph = graph;
+  G->exec = exec;
+  G->launches = nk;
+  *out = G;
+  return CRK_OK;
+}
+
+int crk_graph_launch(crk_graph* G, crk_stream_t stream) {
+  if (!G) return CRK_E_ARG;
+  DeviceGuard g(G->ctx->device);
+  CK(cudaGraphLaunch(G->exec, (cudaStream_t)stream));
+  crk::count_launch(G->launches);
+  return CRK_OK;
+}
+
+void crk_graph_destroy(crk_graph* G) {
+  if (!G) return;
+  DeviceGuard g(G->ctx->device);
+  cudaGraphExecDestroy(G->exec);
+  cudaGraphDestroy(G->graph);
+  delete G;
 }
 
 int crk_host_alloc(uint64_t bytes, void** out) {

@@ -116,6 +116,9 @@ struct ConfigDev {
 struct ScanRingsParam {
   uint32_t n_rings;
   RingDesc r[kMaxRings];
+  // optional: cursors read at execution time (device or mapped memory, u64 [heads n | tails n | send offs n]);
+  // lets a captured serve graph be replayed as the rings advance
+  const uint64_t* doorbell;
 };
 
 cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s);
@@ -143,7 +146,7 @@ cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scrat
                                  const crk_item_req* reqs, const crk_item_req* single, cudaStream_t s);
 cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
                               const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
-                              uint64_t region_bytes, cudaStream_t s);
+                              uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s);
 // Encode jobs built on the host (<= a few per call) are copied in by value.
 struct EncJobParam {
   uint32_t n_jobs, n_pieces;

@@ -173,6 +173,7 @@ struct SendRingsParam {
   uint32_t n_rings;
   RingDesc r[kMaxRings];
   uint64_t off[kMaxRings];
+  const uint64_t* doorbell;  // if set, send offsets are doorbell[2 * n_rings + r]
 };
 
 // pass 2: reply cursors (prefix of wire sizes within each ring) and the encode jobs
@@ -185,7 +186,7 @@ __global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendR
     const uint32_t ring = ix.p_ring[d];
     const uint32_t first = ix.rec_prefix[ring], end = ix.rec_prefix[ring + 1];
     const uint64_t w = ix.s_reply_wire[d];
-    const uint64_t off = S.off[ring] + (pre[d] - pre[first]);
+    const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre[d] - pre[first]);
     ix.s_reply_off[d] = off;
     const int32_t err = ix.s_reply_err[d];
     Job job{};
@@ -318,7 +319,7 @@ cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scrat
 
 cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
                               const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
-                              uint64_t region_bytes, cudaStream_t s) {
+                              uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s) {
   const uint32_t bound = ix.max_records;
   prof_mark(PROF_PLAN, true, s);
   serve_plan1_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, region_base, region_bytes);
@@ -333,8 +334,9 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
     S.r[r].base = send_rings[r].base;
     S.r[r].mask = send_rings[r].cap - 1;
     S.r[r].head = S.r[r].tail = 0;
-    S.off[r] = send_offs[r];
+    S.off[r] = send_offs ? send_offs[r] : 0;
   }
+  S.doorbell = doorbell;
   serve_plan2_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, S);
   count_launch();
   prof_mark(PROF_PLAN, false, s);

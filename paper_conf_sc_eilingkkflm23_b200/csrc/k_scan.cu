@@ -38,7 +38,14 @@ struct ScanState {
 
 __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
   const uint32_t ring = blockIdx.x;
-  const RingDesc R = P.r[ring];
+  RingDesc R = P.r[ring];
+  bool bad_window = false;
+  if (P.doorbell) {  // cursors published by the host at execution time
+    R.head = P.doorbell[ring];
+    R.tail = P.doorbell[P.n_rings + ring];
+    bad_window = R.tail < R.head || R.tail - R.head > R.mask + 1;
+    if (bad_window) R.tail = R.head;
+  }
   const uint32_t T = blockDim.x >> 1;                  // threads per group
   const uint32_t grp = threadIdx.x >= T, u = threadIdx.x - grp * T;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5, wpg = nw >> 1;
@@ -52,8 +59,11 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     S.f0 = S.nf = S.nr = 0;
     S.hp[0] = cfg.guess & 0x7fffffffu;
     S.hp[1] = kNoPred;
-    S.done = 0;
+    S.done = bad_window;
     S.wide = 0;
+    S.status = CRK_E_ARG;
+    S.consumed = R.head;
+    S.kept_frags = 0;
   }
   __syncthreads();
   while (!S.done) {

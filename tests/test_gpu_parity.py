@@ -649,3 +649,49 @@ def test_staged_e2e_path_matches_oracle():
     assert n == want["reply_bytes"][0]
     assert hsend.read(77, n) == bytes(want["send"][0][77:77 + n])
     assert np.array_equal(region.cpu().numpy(), host_region)
+
+
+def test_serve_graph_replays_with_doorbell_cursors():
+    """A captured serve step replayed over successive windows of the same ring == the oracle per window."""
+    cfg = ocfg(F=4096)
+    ctx = ctx_for(cfg)
+    region = torch.zeros(1 << 20, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    host_region = np.zeros(1 << 20, np.uint8)
+    host_region[600000:700000] = gen.random_bytes(2, 100000)
+    region.copy_(torch.from_numpy(host_region))
+    ring = make_ring(1 << 16)
+    send = make_ring(1 << 17)
+    idx = ctx.index(1, 4096, 256)
+    bell = crk.HostBuffer(3 * 8)
+    cells = bell.np.view(np.uint64)
+    graph = idx.serve_graph([ring], [send], base, region.numel(), bell)
+    head, out = 60000, 5
+    for batch in range(4):
+        wires = []
+        for i in range(3):
+            xid = 1000 * batch + i
+            if i == 1:
+                wires.append(O.encode_call(*d2h_call(xid, base + 600000 + 999 * batch, 3000 + 1000 * batch), cfg,
+                                           F=4096))
+            else:
+                wires.append(O.encode_call(*h2d_call(xid, gen.random_bytes(xid, 2000 + 777 * i),
+                                                     base + 10000 * (batch * 3 + i)), cfg, F=4096))
+        w = b"".join(wires)
+        tail = place(ring, w, head)
+        cells[:] = [head, tail, out]
+        torch.cuda.synchronize()
+        graph.launch()
+        torch.cuda.synchronize()
+        res = idx.ring_results(1)[0]
+        want = O.serve([(ring_np(ring), head, tail)], cfg, host_region, base, [1 << 17], [out])
+        assert res["status"] == O.OK and res["consumed"] == tail and res["reply_bytes"] == want["reply_bytes"][0]
+        n = want["reply_bytes"][0]
+        assert send.read(out, n) == bytes(want["send"][0][out:out + n])
+        assert np.array_equal(region.cpu().numpy(), host_region)
+        head, out = tail, out + n
+    cells[:] = [10, 5, 0]  # invalid window: E_ARG, nothing served
+    graph.launch()
+    torch.cuda.synchronize()
+    assert idx.ring_results(1)[0]["status"] == O.E_ARG
+    graph.close()
