@@ -440,3 +440,59 @@ def test_d2h_reply_round_trip(data, F, err):
         up.done()
     fl = [f["len"] for f in s.frags]
     assert all(x == F for x in fl[:-1]) and 0 < fl[-1] <= F or (len(L) == 0)
+
+
+def test_array_reply_vs_xdrlib():
+    """or_encode_array_reply (used as the expected value of the GPU typed-array encoder) decoded by xdrlib."""
+    for dt, unpack in ((np.int32, "unpack_int"), (np.uint32, "unpack_uint"), (np.int64, "unpack_hyper"),
+                       (np.uint64, "unpack_uhyper")):
+        a = gen.random_elems(gen.rng(7), dt, 3001)
+        for F in (97, 4096, 65536):
+            w = O.encode_array_reply(0xABCD, a, 0, F)
+            ring = ring_of(w, 1 << 16)
+            s = O.frame_scan(ring, 0, len(w))
+            assert s.status == O.OK and all(f["len"] == F for f in s.frags[:-1])
+            L = O.record_logical(ring, s, 0)
+            up = xdrlib.Unpacker(L)
+            assert [up.unpack_uint() for _ in range(6)] == [0xABCD, 1, 0, 0, 0, 0]
+            assert up.unpack_int() == 0
+            assert up.unpack_array(getattr(up, unpack)) == [int(x) for x in a]
+            up.done()
+    w = O.encode_array_reply(5, np.zeros(3, np.float64), 1, 4096)
+    assert w == struct.pack(">I", 0x80000000 | 28) + O.reply_header(5) + struct.pack(">i", 1)
+
+
+@given(st.binary(min_size=0, max_size=300), st.lists(st.integers(0, 40), min_size=0, max_size=12))
+def test_frame_lens_vs_hand_framing(L, cuts):
+    """or_frame_record_lens against record marks written with struct (RFC 5531 §11)."""
+    lens, left = [], len(L)
+    for c in cuts:
+        c = min(c, left)
+        lens.append(c)
+        left -= c
+    lens.append(left)
+    want, o = b"", 0
+    for i, n in enumerate(lens):
+        want += struct.pack(">I", n | (0x80000000 if i == len(lens) - 1 else 0)) + L[o:o + n]
+        o += n
+    assert O.frame_lens(L, lens) == want
+
+
+def test_serve_lenient_mode():
+    """Lenient serve (readings R5, R9): nonzero pads and trailing bytes pass, HtoD copies min(n, size)."""
+    lenient = O.Config(prog=CFG.prog, vers=CFG.vers, strict=False, proc_h2d=CFG.proc_h2d, proc_d2h=CFG.proc_d2h)
+    region = np.zeros(4096, np.uint8)
+    base = 0x10000
+    L1 = bytearray(call_logical(xid=1, data=b"abcde", size=3))       # n=5, size=3 -> copies 3
+    L1[20:24] = struct.pack(">I", CFG.proc_h2d)
+    L1[36:40] = struct.pack(">I", 0)
+    L1[40:48] = struct.pack(">Q", base + 100)
+    L2 = bytearray(call_logical(xid=2, data=b"xyz", extra=b"\0\0\0\0"))  # trailing bytes ignored
+    L2[40:48] = struct.pack(">Q", base + 200)
+    L2[52 + 3] = 9                                                       # nonzero pad ignored
+    wire = O.frame(bytes(L1), 64) + O.frame(bytes(L2), 64)
+    out = O.serve([(ring_of(wire, 4096), 0, len(wire))], lenient, region, base, [1 << 12], [0])
+    assert [r["status"] for r in out["records"]] == [O.OK, O.OK]
+    assert bytes(region[100:106]) == b"abc\0\0\0" and bytes(region[200:203]) == b"xyz"
+    strict = O.serve([(ring_of(wire, 4096), 0, len(wire))], CFG, np.zeros(4096, np.uint8), base, [1 << 12], [0])
+    assert [r["status"] for r in strict["records"]] == [O.E_SIZE, O.E_PAD]

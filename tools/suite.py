@@ -102,6 +102,26 @@ def c1(ctx):
             "batch_payload_gbs": round(n * 8192 / bms / 1e6, 1), "batch_ok": ok2}
 
 
+def serve_latency(ctx):
+    """One 4 KiB HtoD CALL served per step (scan, parse, plan, mover, reply): crk_serve launches versus the
+    same step replayed from a CUDA graph whose cursors come from a doorbell."""
+    region = torch.zeros(1 << 20, dtype=torch.uint8, device=dev)
+    base = region.data_ptr()
+    data = torch.from_numpy(gen.random_bytes(0xC1, 4096)).to(dev)
+    ring = crk.Ring.device(1 << 14)
+    w = ctx.encode_call(7, gen.PROC_H2D, [(crk.K_U64, base + 4096), (crk.K_OPAQUE_VAR, data), (crk.K_U64, 4096)],
+                        ring, 0)
+    send = crk.Ring.device(1 << 12)
+    idx = ctx.index(1, 64, 16)
+    us_launch = timed(lambda _: idx.serve([(ring, 0, w)], [send], [0], base, region.numel()), 500) * 1e3
+    bell = torch.tensor([0, w, 0], dtype=torch.int64, device=dev)
+    g = idx.serve_graph([ring], [send], base, region.numel(), bell)
+    us_graph = timed(lambda _: g.launch(), 500) * 1e3
+    ok = bool(torch.equal(region[4096:8192], data)) and idx.ring_results(1)[0]["reply_bytes"] == 32
+    g.close()
+    return {"serve_launches_us": round(us_launch, 2), "serve_graph_us": round(us_graph, 2), "ok": ok}
+
+
 def c2(ctx):
     A, B, C = gen.c2_matrices()
     region = torch.zeros(4 * MiB, dtype=torch.uint8, device=dev)
@@ -260,6 +280,7 @@ def main():
     ctx = crk.Context(0)
     t0 = time.time()
     out["C1"] = c1(ctx)
+    out["C1_serve_one_record"] = serve_latency(crk.Context(0))
     out["C2_matrixMul"] = c2(crk.Context(0))
     out["C3_sweep"] = c3(crk.Context(0))
     out["C4_typed_regular"] = c4(crk.Context(0), False)
