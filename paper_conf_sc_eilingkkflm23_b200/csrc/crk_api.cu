@@ -674,6 +674,12 @@ int run_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings,
     if (!ring_ok(send_rings[r])) return CRK_E_ARG;
   int st = run_scan(c, x, n_rings, rings, heads, tails, s, doorbell);
   if (st != CRK_OK) return st;
+  if (x->ix.max_records <= kSmallServe) {  // small batch: one planning launch, then the mover
+    CK(launch_serve_plan_small(x->ix, c->cd, c->sc, n_rings, send_rings, send_offs, region_base, region_bytes,
+                               doorbell, s));
+    CK(launch_mover(&x->ix, c->cd, c->sc, c->cd.run, c->move_ctas, s));
+    return CRK_OK;
+  }
   CK(launch_serve_plan(x->ix, c->cd, c->sc, n_rings, send_rings, send_offs, region_base, region_bytes, doorbell,
                        s));
   return move(c, &x->ix, 2 * x->ix.max_records, s);

@@ -164,6 +164,14 @@ cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n,
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
                                  uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s);
 int mover_occupancy(uint32_t tile_bytes, uint32_t stages);
+cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
+                         cudaStream_t s);
+// Serve planning for small batches (index max_records <= kSmallServe): statuses, reply offsets, decode
+// and encode jobs, their tile prefix and the mover cursors in one single-block kernel.
+constexpr uint32_t kSmallServe = 1024;
+cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
+                                    const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
+                                    uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s);
 
 // host-visible counter of our kernel launches
 void count_launch(int n = 1);

@@ -824,14 +824,22 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
       if (tiles_max < (uint64_t)move_ctas) move_ctas = (int)tiles_max;
     }
   }
+  return launch_mover(ix, cfg, sc, run, move_ctas, s);
+}
+
+// The mover over already-planned jobs: tile prefix in scan_tmp[0..n_jobs), total tiles at
+// scan_tmp[max_jobs + 1], job count in counters[1], queue split in counters[4], cursors reset.
+cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
+                         cudaStream_t s) {
+  cudaError_t e;
   MoveParams M;
   if (ix) M.ix = *ix; else memset(&M.ix, 0, sizeof(M.ix));
   M.sc = sc;
   M.cfg = cfg;
   M.cfg.run = run;
-  M.prefix = tiles;
-  M.n_jobs_dev = n_jobs_dev;
-  M.total_tiles = total;
+  M.prefix = sc.scan_tmp;
+  M.n_jobs_dev = sc.counters + 1;
+  M.total_tiles = sc.scan_tmp + sc.max_jobs + 1;
   M.stage_bytes = (1u << cfg.tile_shift) + 32 * kMaxSeg + 32;
   const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
   static uint32_t smem_set = 0;  // dynamic shared memory opt-in (per process, grows monotonically)

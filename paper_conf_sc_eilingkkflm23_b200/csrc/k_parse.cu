@@ -182,7 +182,11 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
 cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const ConfigDev& cfg, uint32_t n_rings,
                          int sms, cudaStream_t s) {
   prof_mark(PROF_PARSE, true, s);
-  parse_kernel<<<sms * 8, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
+  // no more CTAs than the index's record slots of these rings can occupy
+  const uint64_t bound = (uint64_t)ix.recs_per_ring * n_rings;
+  const uint64_t want = (bound + kParseWarps - 1) / kParseWarps, most = (uint64_t)sms * 8;
+  const uint32_t grid = (uint32_t)(want < most ? want : most);
+  parse_kernel<<<grid ? grid : 1, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
   count_launch();
   prof_mark(PROF_PARSE, false, s);
   return cudaGetLastError();

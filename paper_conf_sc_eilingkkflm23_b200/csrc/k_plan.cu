@@ -132,33 +132,78 @@ __device__ __forceinline__ void reply_words(Piece& p, uint32_t xid, int32_t err,
   p.nbytes = with_len ? 32 : 28;
 }
 
+// Serve decisions for dense record d (oracle or_serve): final status, reply discriminant (-1: no reply),
+// reply logical length, and the HtoD decode job.
+__device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev& cfg, uint32_t d, uint64_t region_base,
+                                             uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job) {
+  st = ix.p_status[d];
+  const uint32_t proc = ix.p_proc[d];
+  err = -1;
+  Ll = 0;
+  job = Job{};
+  if (st == CRK_OK && xid_lookup(ix, ix.p_xid[d]) != d) st = CRK_E_XID;
+  const uint64_t b = (uint64_t)d * kMaxItems;
+  if (st == CRK_OK && proc == cfg.proc_h2d) {
+    const uint64_t ptr = ix.p_value[b], nb = ix.p_count[b + 1], size = ix.p_value[b + 2];
+    const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
+    if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
+    else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
+    else { err = 0; job = dec_job(ptr, m, ix.p_off[b + 1], d, 1); }
+    Ll = 28;
+  } else if (st == CRK_OK && proc == cfg.proc_d2h) {
+    const uint64_t ptr = ix.p_value[b], size = ix.p_value[b + 1];
+    if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
+      st = CRK_E_PTR; err = 1; Ll = 28;
+    } else {
+      err = 0; Ll = 32 + size + pad4(size);
+    }
+  }
+}
+
+// The reply of record d as an encode job (pieces at 2d, 2d+1) written at send-ring cursor `off`.
+__device__ __forceinline__ Job serve_reply_job(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t d,
+                                               uint32_t ring, int32_t err, uint64_t off, uint64_t w) {
+  Job job{};
+  if (err < 0) return job;
+  const uint64_t b = (uint64_t)d * kMaxItems;
+  const bool d2h = ix.p_proc[d] == cfg.proc_d2h && err == 0;
+  const uint64_t n = d2h ? ix.p_value[b + 1] : 0;
+  Piece* P = sc.pieces + 2ull * d;
+  reply_words(P[0], ix.p_xid[d], err, d2h, n);
+  uint32_t np = 1;
+  uint64_t Ll = P[0].nbytes;
+  if (d2h) {
+    Piece q{};
+    q.type = PIECE_DATA;
+    q.loff = 32;
+    q.nbytes = n;
+    q.src = ix.p_value[b];
+    q.esize = 1;
+    P[1] = q;
+    np = 2;
+    Ll = 32 + n + pad4(n);
+  }
+  job.type = JOB_ENC;
+  job.out_start = off;
+  job.out_end = off + w;
+  job.loff = Ll;
+  job.piece0 = 2 * d;
+  job.n_pieces = np;
+  job.F = cfg.F;
+  job.out_ring = ring;
+  return job;
+}
+
 __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint64_t region_base,
                                    uint64_t region_bytes) {
   const uint32_t total = *ix.total;
   uint64_t* wire = sc.scan_tmp;  // reply wire sizes -> prefix
   for (uint32_t d = blockIdx.x * blockDim.x + threadIdx.x; d < total; d += gridDim.x * blockDim.x) {
-    int st = ix.p_status[d];
-    const uint32_t proc = ix.p_proc[d];
-    int32_t err = -1;
-    uint64_t Ll = 0;
-    Job job{};
-    if (st == CRK_OK && xid_lookup(ix, ix.p_xid[d]) != d) st = CRK_E_XID;
-    const uint64_t b = (uint64_t)d * kMaxItems;
-    if (st == CRK_OK && proc == cfg.proc_h2d) {
-      const uint64_t ptr = ix.p_value[b], nb = ix.p_count[b + 1], size = ix.p_value[b + 2];
-      const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
-      if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
-      else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
-      else { err = 0; job = dec_job(ptr, m, ix.p_off[b + 1], d, 1); }
-      Ll = 28;
-    } else if (st == CRK_OK && proc == cfg.proc_d2h) {
-      const uint64_t ptr = ix.p_value[b], size = ix.p_value[b + 1];
-      if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
-        st = CRK_E_PTR; err = 1; Ll = 28;
-      } else {
-        err = 0; Ll = 32 + size + pad4(size);
-      }
-    }
+    int st;
+    int32_t err;
+    uint64_t Ll;
+    Job job;
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, job);
     ix.s_status[d] = st;
     ix.s_reply_err[d] = err;
     const uint64_t w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
@@ -188,38 +233,88 @@ __global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendR
     const uint64_t w = ix.s_reply_wire[d];
     const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre[d] - pre[first]);
     ix.s_reply_off[d] = off;
-    const int32_t err = ix.s_reply_err[d];
-    Job job{};
-    if (err >= 0) {
-      const uint64_t b = (uint64_t)d * kMaxItems;
-      const bool d2h = ix.p_proc[d] == cfg.proc_d2h && err == 0;
-      const uint64_t n = d2h ? ix.p_value[b + 1] : 0;
-      Piece* P = sc.pieces + 2ull * d;
-      reply_words(P[0], ix.p_xid[d], err, d2h, n);
-      uint32_t np = 1;
-      uint64_t Ll = P[0].nbytes;
-      if (d2h) {
-        Piece q{};
-        q.type = PIECE_DATA;
-        q.loff = 32;
-        q.nbytes = n;
-        q.src = ix.p_value[b];
-        q.esize = 1;
-        P[1] = q;
-        np = 2;
-        Ll = 32 + n + pad4(n);
-      }
-      job.type = JOB_ENC;
-      job.out_start = off;
-      job.out_end = off + w;
-      job.loff = Ll;
-      job.piece0 = 2 * d;
-      job.n_pieces = np;
-      job.F = cfg.F;
-      job.out_ring = ring;
-    }
-    sc.jobs[total + d] = job;
+    sc.jobs[total + d] = serve_reply_job(ix, cfg, sc, d, ring, ix.s_reply_err[d], off, w);
     if (d + 1 == end) ix.res[ring].reply_bytes = pre[d] + w - pre[first];
+  }
+}
+
+// Block-wide exclusive sum (blockDim.x threads, <= 1024); returns the block total through *tot.
+__device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_sums, uint64_t* tot) {
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  uint64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  __syncthreads();
+  if (lane == 31) warp_sums[w] = x;
+  __syncthreads();
+  uint64_t base = 0, all = 0;
+  for (uint32_t i = 0; i < nw; ++i) {
+    if (i < w) base += warp_sums[i];
+    all += warp_sums[i];
+  }
+  *tot = all;
+  return base + x - v;
+}
+
+// Small batches: one block of kSmallServe threads, thread d owns record d.
+__global__ void __launch_bounds__(kSmallServe) serve_plan_small_kernel(IndexDev ix, ConfigDev cfg, Scratch sc,
+                                                                       SendRingsParam S, uint64_t region_base,
+                                                                       uint64_t region_bytes) {
+  __shared__ uint64_t warp_sums[32];
+  __shared__ uint64_t ring_first_pre[kMaxRings];
+  const uint32_t total = *ix.total;
+  const uint32_t d = threadIdx.x;
+  for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
+  int st = CRK_OK;
+  int32_t err = -1;
+  uint64_t Ll = 0, w = 0;
+  Job dec{};
+  uint32_t ring = 0, first = 0, end = 0;
+  if (d < total) {
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
+    w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
+    ring = ix.p_ring[d];
+    first = ix.rec_prefix[ring];
+    end = ix.rec_prefix[ring + 1];
+  }
+  uint64_t tot;
+  const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets
+  if (d < total && d == first) ring_first_pre[ring] = pre;
+  __syncthreads();
+  Job enc{};
+  if (d < total) {
+    const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre - ring_first_pre[ring]);
+    ix.s_status[d] = st;
+    ix.s_reply_err[d] = err;
+    ix.s_reply_wire[d] = w;
+    ix.s_reply_off[d] = off;
+    enc = serve_reply_job(ix, cfg, sc, d, ring, err, off, w);
+    sc.jobs[d] = dec;
+    sc.jobs[total + d] = enc;
+    if (d + 1 == end) ix.res[ring].reply_bytes = pre + w - ring_first_pre[ring];
+  }
+  // mover plan: tiles per job (decode jobs [0, total), encode jobs [total, 2 total)) and their prefix
+  auto tiles_of = [&](const Job& j) -> uint64_t {
+    if (j.type == JOB_NONE || j.out_end <= j.out_start) return 0;
+    return ((j.out_end - 1) >> cfg.tile_shift) - (j.out_start >> cfg.tile_shift) + 1;
+  };
+  const uint64_t td = d < total ? tiles_of(dec) : 0, te = d < total ? tiles_of(enc) : 0;
+  uint64_t tot_d, tot_e;
+  const uint64_t pd = block_excl_sum(td, warp_sums, &tot_d);
+  const uint64_t pe = block_excl_sum(te, warp_sums, &tot_e);
+  if (d < total) {
+    sc.scan_tmp[d] = pd;
+    sc.scan_tmp[total + d] = tot_d + pe;
+  }
+  if (d == 0) {
+    sc.scan_tmp[sc.max_jobs + 1] = tot_d + tot_e;
+    sc.counters[0] = 0;
+    sc.counters[2] = 0;
+    sc.counters[1] = 2 * total;
+    sc.counters[4] = total;
   }
 }
 
@@ -338,6 +433,24 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
   }
   S.doorbell = doorbell;
   serve_plan2_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, S);
+  count_launch();
+  prof_mark(PROF_PLAN, false, s);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
+                                    const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
+                                    uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s) {
+  SendRingsParam S{};
+  S.n_rings = n_rings;
+  for (uint32_t r = 0; r < n_rings; ++r) {
+    S.r[r].base = send_rings[r].base;
+    S.r[r].mask = send_rings[r].cap - 1;
+    S.off[r] = send_offs ? send_offs[r] : 0;
+  }
+  S.doorbell = doorbell;
+  prof_mark(PROF_PLAN, true, s);
+  serve_plan_small_kernel<<<1, kSmallServe, 0, s>>>(ix, cfg, sc, S, region_base, region_bytes);
   count_launch();
   prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();

@@ -20,11 +20,12 @@ __device__ __forceinline__ void st_volatile(unsigned long long* p, unsigned long
 
 template <typename T>
 __global__ void __launch_bounds__(kScanBlock) scan_kernel(T* data, uint32_t n_static, const uint32_t* n_dev, T* total,
-                                                          unsigned long long* state, uint32_t* block_counter) {
+                                                          unsigned long long* state, uint32_t* block_counter,
+                                                          uint32_t single) {
   __shared__ uint32_t s_bid;
   __shared__ uint64_t s_warp[kScanBlock / 32];
   __shared__ uint64_t s_excl;
-  if (threadIdx.x == 0) s_bid = atomicAdd(block_counter, 1u);  // launch-order ids: forward progress
+  if (threadIdx.x == 0) s_bid = single ? 0u : atomicAdd(block_counter, 1u);  // launch-order ids: forward progress
   __syncthreads();
   const uint32_t bid = s_bid;
   const uint32_t n = n_dev ? *n_dev : n_static;
@@ -63,7 +64,7 @@ __global__ void __launch_bounds__(kScanBlock) scan_kernel(T* data, uint32_t n_st
   if (threadIdx.x == 0) {
     uint64_t excl = 0;
     if (bid == 0) {
-      st_volatile(state, kFlagInc | (block_total & kValMask));
+      if (!single) st_volatile(state, kFlagInc | (block_total & kValMask));
     } else {
       st_volatile(state + bid, kFlagAgg | (block_total & kValMask));
       int64_t j = (int64_t)bid - 1;
@@ -93,11 +94,16 @@ cudaError_t launch_scan(T* data, uint32_t n, const uint32_t* n_dev, T* total, Sc
   // n is the (host-known) upper bound when n_dev is given
   const uint32_t per = kScanBlock * kScanIPT;
   const uint32_t blocks = n == 0 ? 1 : (n + per - 1) / per;
+  if (blocks == 1) {  // one block: no look-back, no state to reset
+    scan_kernel<T><<<1, kScanBlock, 0, s>>>(data, n, n_dev, total, sc.scan_state, sc.counters + 5, 1u);
+    count_launch();
+    return cudaGetLastError();
+  }
   cudaError_t e = cudaMemsetAsync(sc.scan_state, 0, sizeof(unsigned long long) * (blocks + 1), s);
   if (e != cudaSuccess) return e;
   e = cudaMemsetAsync(sc.counters + 5, 0, sizeof(uint32_t), s);
   if (e != cudaSuccess) return e;
-  scan_kernel<T><<<blocks, kScanBlock, 0, s>>>(data, n, n_dev, total, sc.scan_state, sc.counters + 5);
+  scan_kernel<T><<<blocks, kScanBlock, 0, s>>>(data, n, n_dev, total, sc.scan_state, sc.counters + 5, 0u);
   count_launch();
   return cudaGetLastError();
 }
