@@ -25,6 +25,7 @@ struct crk_ctx {
 
 struct crk_index {
   crk_ctx* ctx;
+  int device;  // kept here so destroy does not depend on the context outliving the index
   IndexDev ix;
   void* block;
   crk_ring_result* host_res;  // pinned
@@ -55,11 +56,14 @@ static thread_local int g_last_cuda = 0;
 
 namespace {
 
+// Makes `dev` current for the call and discards stale non-sticky errors left in the runtime's
+// last-error slot by unrelated calls, so CK(cudaGetLastError()) after a launch reports our launch only.
 struct DeviceGuard {
   int prev = -1;
   explicit DeviceGuard(int dev) {
     if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
     else prev = -1;
+    (void)cudaGetLastError();
   }
   ~DeviceGuard() {
     if (prev >= 0) cudaSetDevice(prev);
@@ -344,6 +348,7 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
   if (!x) return CRK_E_CAPACITY;
   memset(x, 0, sizeof(*x));
   x->ctx = c;
+  x->device = c->device;
   IndexDev& ix = x->ix;
   ix.max_rings = max_rings;
   ix.frags_per_ring = max_frags / max_rings;
@@ -406,7 +411,7 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
 
 void crk_index_destroy(crk_index* x) {
   if (!x) return;
-  DeviceGuard g(x->ctx->device);
+  DeviceGuard g(x->device);
   cudaFree(x->block);
   cudaFreeHost(x->host_res);
   delete x;
@@ -688,6 +693,7 @@ int run_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings,
 
 struct crk_graph {
   crk_ctx* ctx;
+  int device;
   cudaGraph_t graph;
   cudaGraphExec_t exec;
   int launches;  // kernels per replay
@@ -734,6 +740,7 @@ int crk_serve_graph_create(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk
   crk_graph* G = new (std::nothrow) crk_graph;
   if (!G) { cudaGraphExecDestroy(exec); cudaGraphDestroy(graph); return CRK_E_CAPACITY; }
   G->ctx = c;
+  G->device = c->device;
   G->graph = graph;
   G->exec = exec;
   G->launches = nk;
@@ -743,7 +750,7 @@ int crk_serve_graph_create(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk
 
 int crk_graph_launch(crk_graph* G, crk_stream_t stream) {
   if (!G) return CRK_E_ARG;
-  DeviceGuard g(G->ctx->device);
+  DeviceGuard g(G->device);
   CK(cudaGraphLaunch(G->exec, (cudaStream_t)stream));
   crk::count_launch(G->launches);
   return CRK_OK;
@@ -751,7 +758,7 @@ int crk_graph_launch(crk_graph* G, crk_stream_t stream) {
 
 void crk_graph_destroy(crk_graph* G) {
   if (!G) return;
-  DeviceGuard g(G->ctx->device);
+  DeviceGuard g(G->device);
   cudaGraphExecDestroy(G->exec);
   cudaGraphDestroy(G->graph);
   delete G;
