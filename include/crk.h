@@ -237,6 +237,27 @@ int crk_xdr_encode_memcpy_d2h(crk_ctx* ctx, uint32_t xid, const void* src, uint6
 int crk_xdr_encode_memcpy_d2h_batch(crk_ctx* ctx, uint32_t n, const uint32_t* xids, const void* const* srcs,
                                     const uint64_t* bytes, const int32_t* cuda_errs, crk_ring out, uint64_t out_off,
                                     uint64_t* wire_offs, uint64_t* total_dev, crk_stream_t stream);
+/* Generic batched REPLY encoder (control-path results): request i becomes
+ *   REPLY(xid, MSG_ACCEPTED, AUTH_NONE, SUCCESS) | int err | [err == 0 && kind != 0: one XDR item]
+ * where the item is `value` for CRK_K_U32 / CRK_K_U64, or `count` elements (bytes for opaque kinds)
+ * read from device memory at `src` for the opaque / array kinds (VAR kinds carry their count word,
+ * FIX kinds do not).  Replies are framed with cfg.frag_payload and written back to back from out_off
+ * in request order; wire_offs (dev, n) receives each reply's cursor, total_dev the sum.  reqs_dev is a
+ * device array owned by the caller; a kind outside 1..16 encodes no item (as kind 0); a request
+ * with err == 0 whose item cannot be encoded (count >= 2^32, count > 0 with src NULL, src not
+ * aligned to the element size) is encoded with err = CRK_E_ARG and no item.  Returns
+ * CRK_E_ARG for n > cfg.max_jobs or a bad ring, CRK_E_CUDA on launch failure. */
+typedef struct {
+  uint32_t xid;
+  int32_t err;
+  uint32_t kind;
+  uint32_t pad_;
+  uint64_t value;
+  const void* src;
+  uint64_t count;
+} crk_reply_req;
+int crk_rpc_encode_replies_batch(crk_ctx* ctx, uint32_t n, const crk_reply_req* reqs_dev, crk_ring out,
+                                 uint64_t out_off, uint64_t* wire_offs, uint64_t* total_dev, crk_stream_t stream);
 /* REPLY | int err | [err == 0: T data<> big-endian] (typed analogue of the memcpy reply). */
 int crk_xdr_encode_array_i32(crk_ctx*, uint32_t xid, const int32_t* src, uint64_t count, int32_t err, crk_ring out,
                              uint64_t out_off, uint64_t* wire_bytes, crk_stream_t);

@@ -484,6 +484,28 @@ uint64_t or_encode_array_reply(uint32_t xid, const uint8_t* elems, uint32_t coun
   return w;
 }
 
+/* Generic REPLY (control-path results): REPLY header | int err | [err == 0 && kind != 0: one item]:
+ * U32 / U64 -> value; opaque kinds -> count bytes of elems (VAR with its length word); array kinds ->
+ * count elements of elems in host order written big-endian (VAR with its count word). */
+uint64_t or_encode_reply_item(uint32_t xid, int32_t err, uint32_t kind, uint64_t value, const uint8_t* elems,
+                              uint32_t count, uint32_t F, uint8_t* out) {
+  uint64_t cap = 28 + 8 + (uint64_t)count * 8 + 8, pos = 0, w;
+  uint8_t* L = (uint8_t*)malloc(cap);
+  pos = or_rpc_put_reply_header(L, pos, xid);
+  pos = or_xdr_put_u32(L, pos, (uint32_t)err);
+  if (err == 0 && kind != 0) {
+    if (kind == OR_K_U32) pos = or_xdr_put_u32(L, pos, (uint32_t)value);
+    else if (kind == OR_K_U64) pos = or_xdr_put_u64(L, pos, value);
+    else if (kind == OR_K_OPAQUE_VAR) pos = or_xdr_put_opaque_var(L, pos, elems, count);
+    else if (kind == OR_K_OPAQUE_FIX) pos = or_xdr_put_opaque_fix(L, pos, elems, count);
+    else pos = or_xdr_put_array(L, pos, elems, count, or_elem_size(kind), or_kind_is_var(kind));
+  }
+  if (!out) { free(L); return or_frame_wire_size(pos, F); }
+  w = or_frame_record(L, pos, F, out);
+  free(L);
+  return w;
+}
+
 /* =====================================================================================
  * Server step over several rings (the north-star loop): frame-scan each ring, parse
  * every CALL, then in index order (ring 0's records first):

@@ -130,6 +130,8 @@ def lib():
         L.or_encode_memcpy_d2h.argtypes = [C.c_uint32, u8p, C.c_uint32, C.c_int32, C.c_uint32, u8p]
         L.or_encode_array_reply.restype = u64
         L.or_encode_array_reply.argtypes = [C.c_uint32, u8p, C.c_uint32, C.c_uint32, C.c_int32, C.c_uint32, u8p]
+        L.or_encode_reply_item.restype = u64
+        L.or_encode_reply_item.argtypes = [C.c_uint32, C.c_int32, C.c_uint32, u64, u8p, C.c_uint32, C.c_uint32, u8p]
         L.or_serve.restype = C.c_int
         L.or_serve.argtypes = [C.c_uint32, C.POINTER(u8p), C.POINTER(C.c_uint64), C.POINTER(C.c_uint64),
                                C.POINTER(C.c_uint64), u64, C.c_uint32, C.c_uint32, C.POINTER(Cfg),
@@ -360,6 +362,20 @@ def encode_array_reply(xid: int, elems: np.ndarray, err: int, F: int) -> bytes:
     w = lib().or_encode_array_reply(xid, ep, len(e), es, err, F, None)
     out = np.zeros(w, np.uint8)
     lib().or_encode_array_reply(xid, ep, len(e), es, err, F, _p(out))
+    return out.tobytes()
+
+
+def encode_reply_item(xid: int, err: int, kind: int, value=0, elems=None, F: int = 65536) -> bytes:
+    """Generic REPLY with one result item (see or_encode_reply_item)."""
+    if elems is None:
+        e, count = np.zeros(8, np.uint8), 0
+    else:
+        e = np.ascontiguousarray(elems)
+        count = len(e)
+        e = e.view(np.uint8) if e.size else np.zeros(8, np.uint8)
+    w = lib().or_encode_reply_item(xid, err, kind, value & 0xFFFFFFFFFFFFFFFF, _p(e), count, F, None)
+    out = np.zeros(w, np.uint8)
+    lib().or_encode_reply_item(xid, err, kind, value & 0xFFFFFFFFFFFFFFFF, _p(e), count, F, _p(out))
     return out.tobytes()
 
 

@@ -75,6 +75,11 @@ class ItemSrc(C.Structure):
                 ("count", C.c_uint64)]
 
 
+class ReplyReq(C.Structure):
+    _fields_ = [("xid", C.c_uint32), ("err", C.c_int32), ("kind", C.c_uint32), ("pad_", C.c_uint32),
+                ("value", C.c_uint64), ("src", C.c_void_p), ("count", C.c_uint64)]
+
+
 _lib = None
 vp, u32, u64, i32 = C.c_void_p, C.c_uint32, C.c_uint64, C.c_int32
 
@@ -104,6 +109,7 @@ def lib():
             "crk_wire_size_d2h": (u64, [u64, i32, u32]),
             "crk_xdr_encode_memcpy_d2h": (C.c_int, [vp, u32, vp, u64, i32, CRing, u64, C.POINTER(u64), vp]),
             "crk_xdr_encode_memcpy_d2h_batch": (C.c_int, [vp, u32, vp, vp, vp, vp, CRing, u64, vp, vp, vp]),
+            "crk_rpc_encode_replies_batch": (C.c_int, [vp, u32, vp, CRing, u64, vp, vp, vp]),
             "crk_rpc_encode_call": (C.c_int, [vp, u32, u32, C.POINTER(ItemSrc), u32, C.POINTER(u32), u32, CRing, u64,
                                               C.POINTER(u64), vp]),
             "crk_call_logical_size": (u64, [C.POINTER(ItemSrc), u32]),
@@ -383,6 +389,20 @@ class Context:
         _check(lib().crk_xdr_encode_memcpy_d2h_batch(self.h, xids.numel(), _ptr(xids), _ptr(srcs), _ptr(nbytes),
                                                      _ptr(errs), out.c(), out_off, _ptr(wire_offs), _ptr(total),
                                                      _stream(stream)), "crk_xdr_encode_memcpy_d2h_batch")
+
+    def encode_replies_batch(self, reqs, out: Ring, out_off: int, wire_offs: torch.Tensor | None = None,
+                             total: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+        """reqs: list of (xid, err, kind, value, src tensor | None, count).  Marshals them into a device
+        crk_reply_req array (kept alive until the stream is synchronised by the caller) and encodes."""
+        n = len(reqs)
+        arr = (ReplyReq * max(1, n))()
+        for i, (xid, err, kind, value, src, count) in enumerate(reqs):
+            arr[i] = ReplyReq(xid, err, kind, 0, value & 0xFFFFFFFFFFFFFFFF, _ptr(src), count)
+        host = torch.frombuffer(bytearray(arr), dtype=torch.uint8)
+        dev = host.to(f"cuda:{self.device}")
+        _check(lib().crk_rpc_encode_replies_batch(self.h, n, _ptr(dev), out.c(), out_off, _ptr(wire_offs),
+                                                  _ptr(total), _stream(stream)), "crk_rpc_encode_replies_batch")
+        return dev
 
 
 # ------------------------------------------------------------------ index

@@ -569,6 +569,16 @@ int crk_xdr_encode_memcpy_d2h_batch(crk_ctx* c, uint32_t n, const uint32_t* xids
   return move(c, nullptr, n, s);
 }
 
+int crk_rpc_encode_replies_batch(crk_ctx* c, uint32_t n, const crk_reply_req* reqs, crk_ring out, uint64_t out_off,
+                                 uint64_t* wire_offs, uint64_t* total_dev, crk_stream_t stream) {
+  if (!c || n > c->sc.max_jobs || !ring_ok(out) || (n && !reqs)) return CRK_E_ARG;
+  if (n == 0) return CRK_OK;
+  DeviceGuard g(c->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(launch_replies_jobs(c->sc, c->cd, n, reqs, ring_desc(out, 0, 0), out_off, wire_offs, total_dev, s));
+  return move(c, nullptr, n, s);
+}
+
 #define CRK_ENC_ARRAY(name, T)                                                                                   \
   int crk_xdr_encode_array_##name(crk_ctx* c, uint32_t xid, const T* src, uint64_t count, int32_t err,          \
                                   crk_ring out, uint64_t out_off, uint64_t* wire_bytes, crk_stream_t stream) {  \

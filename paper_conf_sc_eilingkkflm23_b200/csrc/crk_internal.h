@@ -159,6 +159,9 @@ cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n,
                                   const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
                                   cudaStream_t s);
 cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n, cudaStream_t s);
+cudaError_t launch_replies_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const crk_reply_req* reqs,
+                                const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
+                                cudaStream_t s);
 // Plans tiles for jobs [0, n_jobs) (n_jobs from counters[1] <= max_jobs_bound) and runs the mover.
 // out_bytes_bound (0 = unknown) caps the mover grid for small requests.
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,

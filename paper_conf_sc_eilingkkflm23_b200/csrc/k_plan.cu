@@ -378,6 +378,90 @@ __global__ void d2h_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uin
   }
 }
 
+// ---- generic replies: REPLY header | int err | [one item]
+__device__ __forceinline__ uint32_t esize_of(uint32_t kind) { return elem_size_k(kind); }
+__device__ __forceinline__ bool kind_var_k(uint32_t k) {
+  return k == CRK_K_OPAQUE_VAR || (k >= CRK_K_I32_VAR && k <= CRK_K_F64_VAR);
+}
+// A request whose item cannot be encoded (count >= 2^32, null or misaligned src) becomes err = CRK_E_ARG.
+__device__ __forceinline__ int32_t reply_err_eff(const crk_reply_req& r) {
+  if (r.err != 0 || r.kind < CRK_K_OPAQUE_VAR || r.kind > CRK_K_F64_FIX) return r.err;
+  const uint32_t es = esize_of(r.kind);
+  if (r.count > 0xffffffffull || (r.count && !r.src) || ((uintptr_t)r.src % es) != 0) return CRK_E_ARG;
+  return 0;
+}
+__device__ __forceinline__ uint64_t reply_item_logical(crk_reply_req r) {
+  uint64_t L = 28;  // header (24) + err (4)
+  r.err = reply_err_eff(r);
+  if (r.err != 0 || r.kind == 0 || r.kind > CRK_K_F64_FIX) return L;  // no item (unknown kinds: none)
+  if (r.kind == CRK_K_U32) return L + 4;
+  if (r.kind == CRK_K_U64) return L + 8;
+  const uint64_t nb = r.count * esize_of(r.kind);
+  return L + (kind_var_k(r.kind) ? 4 : 0) + nb + pad4(nb);
+}
+
+__global__ void replies_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const crk_reply_req* reqs) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    sc.scan_tmp[i] = wire_of(reply_item_logical(reqs[i]), cfg.F);
+  if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
+}
+
+__global__ void replies_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const crk_reply_req* reqs, RingDesc out,
+                                    uint64_t out_off, uint64_t* wire_offs, uint64_t* total_dev,
+                                    const uint64_t* total_scan) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    sc.out_rings[0] = out;
+    if (total_dev) *total_dev = *total_scan;
+  }
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    crk_reply_req r = reqs[i];
+    r.err = reply_err_eff(r);
+    const uint64_t off = out_off + sc.scan_tmp[i];
+    const uint64_t Ll = reply_item_logical(r);
+    Piece* P = sc.pieces + 2ull * i;
+    Piece w{};
+    w.type = PIECE_WORDS;
+    w.words[0] = r.xid;  // RFC 5531 §9 REPLY, MSG_ACCEPTED, verf AUTH_NONE, SUCCESS
+    w.words[1] = 1;
+    w.words[6] = (uint32_t)r.err;
+    uint32_t nw = 7, np = 1;
+    Piece q{};
+    const bool item = r.err == 0 && r.kind != 0 && r.kind <= CRK_K_F64_FIX;
+    if (item && r.kind == CRK_K_U32) {
+      w.words[nw++] = (uint32_t)r.value;
+    } else if (item && r.kind == CRK_K_U64) {  // RFC 4506 §4.5: most significant word first
+      w.words[nw++] = (uint32_t)(r.value >> 32);
+      q.type = PIECE_WORDS;
+      q.loff = 32;
+      q.nbytes = 4;
+      q.words[0] = (uint32_t)r.value;
+      np = 2;
+    } else if (item) {
+      if (kind_var_k(r.kind)) w.words[nw++] = (uint32_t)r.count;
+      q.type = PIECE_DATA;
+      q.loff = 4ull * nw;
+      q.nbytes = r.count * esize_of(r.kind);
+      q.src = (uint64_t)r.src;
+      q.esize = esize_of(r.kind);
+      np = 2;
+    }
+    w.nbytes = 4ull * nw;
+    P[0] = w;
+    if (np == 2) P[1] = q;
+    Job job{};
+    job.type = JOB_ENC;
+    job.out_start = off;
+    job.out_end = off + wire_of(Ll, cfg.F);
+    job.loff = Ll;
+    job.piece0 = 2 * i;
+    job.n_pieces = np;
+    job.F = cfg.F;
+    job.out_ring = 0;
+    sc.jobs[i] = job;
+    if (wire_offs) wire_offs[i] = off;
+  }
+}
+
 __global__ void lens_prep_kernel(Scratch sc, const uint32_t* lens32, uint32_t n) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     sc.lens_pool[i] = lens32[i];
@@ -475,6 +559,21 @@ cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n,
   if (e != cudaSuccess) return e;
   d2h_jobs_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
                                                  tot);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_replies_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const crk_reply_req* reqs,
+                                const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
+                                cudaStream_t s) {
+  replies_sizes_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, reqs);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
+  e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
+  if (e != cudaSuccess) return e;
+  replies_jobs_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, reqs, out, out_off, wire_offs, total, tot);
   count_launch();
   return cudaGetLastError();
 }

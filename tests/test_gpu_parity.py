@@ -473,6 +473,55 @@ def test_encode_memcpy_d2h_batch_matches_oracle():
     assert np.array_equal(offs.cpu().numpy(), ow + start)
 
 
+_NP = {O.K_OPAQUE_VAR: np.uint8, O.K_OPAQUE_FIX: np.uint8, O.K_I32_VAR: np.int32, O.K_U32_VAR: np.uint32,
+       O.K_F32_VAR: np.float32, O.K_I64_VAR: np.int64, O.K_U64_VAR: np.uint64, O.K_F64_VAR: np.float64,
+       O.K_I32_FIX: np.int32, O.K_U32_FIX: np.uint32, O.K_F32_FIX: np.float32, O.K_I64_FIX: np.int64,
+       O.K_U64_FIX: np.uint64, O.K_F64_FIX: np.float64}
+
+
+@pytest.mark.parametrize("host,F", [(False, 4096), (True, 65536), (False, 1 << 20)])
+def test_encode_replies_batch_matches_oracle(host, F):
+    """Generic batched REPLY encoder (NEXT-3) vs or_encode_reply_item, every kind, err != 0, unknown kind,
+    misaligned sources, multi-fragment records and ring wrap."""
+    ctx = ctx_for(ocfg(F=F))
+    out = crk.Ring.host(1 << 21) if host else make_ring(1 << 21)
+    g = gen.rng(31)
+    reqs, want, keep = [], [], []
+    for i in range(90):
+        kind = [0, O.K_U32, O.K_U64, 99, *range(3, 17)][i % 18]
+        err = 3 if i % 13 == 5 else 0
+        xid = 9000 + i
+        value = int(g.integers(0, 1 << 63)) * 2 + (i & 1)
+        src, count, elems = None, 0, None
+        if kind in _NP:
+            count = int(g.integers(0, [1, 7, 300, 20000][i % 4]))
+            elems = gen.random_elems(g, _NP[kind], count)
+            es = np.dtype(_NP[kind]).itemsize
+            mis = (i * 4) % 16 if es > 1 else i % 16  # misaligned 8-byte sources -> err = E_ARG
+            raw = np.concatenate([np.zeros(mis, np.uint8), elems.view(np.uint8)])
+            t = torch.from_numpy(raw).cuda()
+            keep.append(t)
+            src = t.data_ptr() + mis
+        reqs.append((xid, err, kind, value, src, count))
+        eff = O.E_ARG if err == 0 and elems is not None and mis % es else err
+        want.append(O.encode_reply_item(xid, eff, kind if kind != 99 else 0, value, elems, F))
+    reqs.append((9999, 0, O.K_U32_VAR, 0, None, 5))  # count > 0 with no source -> err = E_ARG
+    want.append(O.encode_reply_item(9999, O.E_ARG, O.K_U32_VAR, 0, None, F))
+    offs = torch.zeros(len(reqs), dtype=torch.int64, device="cuda")
+    tot = torch.zeros(1, dtype=torch.int64, device="cuda")
+    start = (1 << 21) - 70000
+    ctx.encode_replies_batch(reqs, out, start, offs, tot)
+    torch.cuda.synchronize()
+    allw = b"".join(want)
+    assert tot.item() == len(allw)
+    got = out.read(start, len(allw))
+    pos = 0
+    for i, w in enumerate(want):
+        assert got[pos:pos + len(w)] == w, f"reply {i} kind {reqs[i][2]} err {reqs[i][1]} count {reqs[i][5]}"
+        pos += len(w)
+    assert np.array_equal(offs.cpu().numpy(), np.cumsum([0] + [len(w) for w in want])[:-1] + start)
+
+
 @pytest.mark.parametrize("host", [False, True])
 def test_serve_matches_oracle(host):
     cfg = ocfg(F=16384)

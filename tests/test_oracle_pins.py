@@ -496,3 +496,30 @@ def test_serve_lenient_mode():
     assert bytes(region[100:106]) == b"abc\0\0\0" and bytes(region[200:203]) == b"xyz"
     strict = O.serve([(ring_of(wire, 4096), 0, len(wire))], CFG, np.zeros(4096, np.uint8), base, [1 << 12], [0])
     assert [r["status"] for r in strict["records"]] == [O.E_SIZE, O.E_PAD]
+
+
+def test_reply_item_vs_xdrlib():
+    """or_encode_reply_item (expected value of the GPU batched reply encoder) decoded by xdrlib."""
+    cases = [(O.K_U32, 0xDEADBEEF, None, "unpack_uint"), (O.K_U64, 0x0123456789ABCDEF, None, "unpack_uhyper"),
+             (O.K_OPAQUE_VAR, 0, gen.random_bytes(1, 13), "unpack_opaque"),
+             (O.K_I64_VAR, 0, gen.random_elems(gen.rng(2), np.int64, 9), "hyper_array"),
+             (O.K_F32_FIX, 0, np.arange(5, dtype=np.float32), "float_farray")]
+    for kind, value, elems, how in cases:
+        w = O.encode_reply_item(7, 0, kind, value, elems, 4096)
+        L = w[4:]
+        assert struct.unpack(">I", w[:4])[0] == 0x80000000 | len(L)
+        up = xdrlib.Unpacker(L)
+        assert [up.unpack_uint() for _ in range(6)] == [7, 1, 0, 0, 0, 0] and up.unpack_int() == 0
+        if how == "unpack_uint":
+            assert up.unpack_uint() == value
+        elif how == "unpack_uhyper":
+            assert up.unpack_uhyper() == value
+        elif how == "unpack_opaque":
+            assert up.unpack_opaque() == elems.tobytes()
+        elif how == "hyper_array":
+            assert up.unpack_array(up.unpack_hyper) == [int(x) for x in elems]
+        else:
+            assert up.unpack_farray(5, up.unpack_float) == [float(x) for x in elems]
+        up.done()
+    assert O.encode_reply_item(9, 35, O.K_U64, 5) == struct.pack(">I", 0x80000000 | 28) + O.reply_header(9) + \
+        struct.pack(">i", 35)
