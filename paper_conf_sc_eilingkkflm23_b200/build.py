@@ -48,5 +48,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_trace() -> str:
+    """Diagnostic variant with the scan's per-round clock trace (-DCRK_SCAN_TRACE); tools/scan_trace.py."""
+    out = os.path.join(PKG, "lib", "libcrk_trace.so")
+    if os.path.exists(out) and all(os.path.getmtime(d) <= os.path.getmtime(out) for d in deps()):
+        return out
+    r = subprocess.run([NVCC, *FLAGS, "-DCRK_SCAN_TRACE", "-o", out, *sources()], capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("nvcc failed building libcrk_trace.so")
+    return out
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

@@ -21,7 +21,37 @@ namespace {
 
 enum : uint32_t { STOP_NONE = 0, STOP_FRAG = 1, STOP_INCOMPLETE = 2, STOP_CAP = 3 };
 constexpr uint32_t kNoPred = 0xffffffffu;  // a predictor value no header is expected to match
-constexpr uint32_t kJ = 4;                 // candidate headers per thread and round (independent loads)
+constexpr uint32_t kJ = 4;                 // candidate headers per thread and CTA round (independent loads)
+constexpr uint32_t kWJ = 2;                // candidate headers per lane and warp round
+constexpr uint32_t kWTT = 16 * kWJ;        // candidates per group and warp round (16 lanes per group)
+constexpr uint32_t kChase = 512;           // max headers per chase pass (irregular framing)
+constexpr uint32_t kFull = 0xffffffffu;
+
+#ifdef CRK_SCAN_TRACE
+// Diagnostic build only (build.py build_trace -> lib/libcrk_trace.so): per ring, one entry per round /
+// chase hop = clock64 at its end (low 40 bits) | mode (3 bits) << 40 | headers accepted << 43.
+constexpr uint32_t kTraceRings = 64, kTraceLen = 4096;
+__device__ unsigned long long g_scan_trace[kTraceRings][kTraceLen];
+__device__ uint32_t g_scan_trace_n[kTraceRings];
+__device__ __forceinline__ void trace(uint32_t mode, uint32_t n) {
+  const uint32_t r = blockIdx.x;
+  if (r >= kTraceRings) return;
+  const uint32_t i = g_scan_trace_n[r];
+  if (i < kTraceLen) {
+    g_scan_trace[r][i] = (clock64() & ((1ull << 40) - 1)) | ((unsigned long long)mode << 40) |
+                         ((unsigned long long)n << 43);
+    g_scan_trace_n[r] = i + 1;
+  }
+}
+#define SCAN_TRACE(writer, mode, n) \
+  do {                              \
+    if (writer) trace(mode, n);     \
+  } while (0)
+#else
+#define SCAN_TRACE(writer, mode, n) \
+  do {                              \
+  } while (0)
+#endif
 
 struct ScanState {
   uint64_t p, r0, sum;
@@ -31,10 +61,238 @@ struct ScanState {
   int32_t status;
   uint64_t consumed;
   uint32_t kept_frags;
-  uint32_t wide;
+  uint32_t wide;                      // CTA rounds (a long regular run) instead of warp rounds
   uint32_t gmin[32], gh[32], gv[32];  // per warp: first mismatch, its header, its validity
   uint32_t fmin[32], fcode[32];       // per warp: first failing check and its code
 };
+
+// The walk state between rounds (uniform across the lanes of warp 0 in the warp modes).
+struct Walk {
+  uint64_t p, r0, sum;
+  uint32_t nf, nr, f0, hp0, hp1;
+  bool stop;
+  int32_t status;
+  uint64_t consumed;
+  uint32_t kept;
+};
+
+struct Env {
+  IndexDev ix;
+  RingDesc R;
+  uint64_t max_record_bytes, fbase, rbase;
+  uint32_t FC, RC;
+};
+
+// Header at cursor q, read as the aligned word(s) that contain it (any alignment, across the wrap); the
+// second word only when q is not 4-aligned (framing with lengths that are multiples of 4 never needs it).
+__device__ __forceinline__ void load_hdr(const RingDesc& R, uint64_t q, bool ok, uint32_t& w0, uint32_t& w1) {
+  const uint64_t a = q & ~3ull;
+  w0 = ok ? __ldg(reinterpret_cast<const uint32_t*>(R.base + (a & R.mask))) : 0u;
+  w1 = (ok && (q & 3)) ? __ldg(reinterpret_cast<const uint32_t*>(R.base + ((a + 4) & R.mask))) : 0u;
+}
+__device__ __forceinline__ uint32_t join_hdr(uint64_t q, uint32_t w0, uint32_t w1) {
+  return bswap32(__funnelshift_r(w0, w1, 8 * (uint32_t)(q & 3)));
+}
+
+// Index entries of fragment number nf (and of the record it completes).
+__device__ __forceinline__ void emit_frag(const Env& E, uint32_t nf, uint64_t q, uint64_t len, uint32_t last,
+                                          uint64_t send, bool start, uint64_t r0, uint32_t f0, uint32_t nrec) {
+  const uint64_t fs = E.fbase + nf;
+  E.ix.frag_phys[fs] = q + 4;
+  E.ix.frag_lstart[fs] = send - len;
+  E.ix.frag_hdr[fs] = (uint32_t)len | (last << 31);
+  if (last) {
+    const uint64_t rs = E.rbase + nrec;
+    E.ix.rec_begin[rs] = start ? q : r0;
+    E.ix.rec_len[rs] = send;
+    E.ix.rec_frag0[rs] = (uint32_t)(E.fbase + (start ? nf : f0));
+    E.ix.rec_nfrags[rs] = start ? 1u : nf - f0 + 1;
+  }
+}
+
+// Chase pass: the serial walk of the chain, one dependent header load per fragment, for framing no
+// predictor follows.  The per-header logic is the rounds' with u* = 0, in or_frame_scan's order
+// E_FRAG -> INCOMPLETE -> capacity.  Stops after kChase headers, at a stop, or at two equal consecutive
+// headers (a regular run the predictors can take over again).  Lanes walk the same chain (broadcast loads).
+__device__ void chase(const Env& E, Walk& W, bool writer) {
+  uint32_t prev = kNoPred;
+  for (uint32_t k = 0; k < kChase; ++k) {
+    const bool start = W.p == W.r0;
+    if (W.p + 4 > E.R.tail) {  // no readable header: the window ends here
+      W.stop = true;
+      W.status = (start && W.p == E.R.tail) ? CRK_OK : CRK_INCOMPLETE;
+      break;
+    }
+    uint32_t w0, w1;
+    load_hdr(E.R, W.p, true, w0, w1);
+    const uint32_t h = join_hdr(W.p, w0, w1);
+    const uint64_t len = h & 0x7fffffffu;
+    const uint32_t last = h >> 31;
+    const uint64_t send = start ? len : W.sum + len;
+    bool fail = true;
+    if (send > E.max_record_bytes) W.status = CRK_E_FRAG;
+    else if (W.p + 4 + len > E.R.tail) W.status = CRK_INCOMPLETE;
+    else if (W.nf >= E.FC || (start && W.nr >= E.RC)) W.status = W.nr > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY;
+    else fail = false;
+    if (fail) { W.stop = true; break; }
+    if (writer) emit_frag(E, W.nf, W.p, len, last, send, start, W.r0, W.f0, W.nr);
+    SCAN_TRACE(writer, 2, 1);
+    W.p += 4 + len;
+    W.nf++;
+    if (last) {
+      if (start) W.hp1 = h;
+      W.nr++;
+      W.r0 = W.p;
+      W.sum = 0;
+      W.f0 = W.nf;
+    } else {
+      W.hp0 = h;
+      W.sum = send;
+    }
+    if (h == prev) break;
+    prev = h;
+  }
+  if (W.stop) {
+    const bool start = W.p == W.r0;
+    W.consumed = W.r0;
+    W.kept = start ? W.nf : W.f0;
+  }
+}
+
+// Warp rounds: the CTA round's speculation (two predictor groups, first mismatch still a true header,
+// closed forms in u) on the 32 lanes of one warp -- 16 lanes x kWJ candidates per group -- with warp
+// reductions instead of block barriers, so a round costs one memory latency.  Records that are not
+// long regular runs (mixed HtoD / DtoH calls, small calls) are scanned here.  Returns true when a round
+// matched every candidate (a long regular run: hand over to the CTA rounds); false on a stop.  After
+// two rounds that accepted at most 2 headers each, a chase pass takes over.
+__device__ bool warp_rounds(const Env& E, Walk& W, uint32_t lane) {
+  const uint32_t grp = lane >> 4, u = lane & 15;
+  uint32_t miss = 0;
+  for (;;) {
+    if (miss >= 2) {
+      chase(E, W, lane == 0);
+      if (W.stop) return false;
+      miss = 0;
+      continue;
+    }
+    const uint64_t p = W.p, r0 = W.r0, sum = W.sum;
+    const uint32_t nf = W.nf, nr = W.nr, f0 = W.f0;
+    const uint32_t hmine = grp ? W.hp1 : W.hp0;
+    const uint64_t smine = 4 + (uint64_t)(hmine & 0x7fffffffu);
+    uint32_t w0[kWJ], w1[kWJ];
+    bool vv[kWJ];
+#pragma unroll
+    for (uint32_t j = 0; j < kWJ; ++j) {
+      const uint64_t q = p + (uint64_t)(u + 16 * j) * smine;
+      vv[j] = q + 4 <= E.R.tail;
+      load_hdr(E.R, q, vv[j], w0[j], w1[j]);
+    }
+    uint32_t first_bad = kWTT, bh = 0, bv = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < kWJ; ++j) {
+      const uint32_t t = u + 16 * j;
+      const uint32_t h = join_hdr(p + (uint64_t)t * smine, w0[j], w1[j]);
+      if (first_bad == kWTT && !(vv[j] && h == hmine)) { first_bad = t; bh = h; bv = vv[j]; }
+    }
+    const uint32_t ts0 = __reduce_min_sync(kFull, grp == 0 ? first_bad : kWTT);
+    const uint32_t ts1 = __reduce_min_sync(kFull, grp == 1 ? first_bad : kWTT);
+    const uint32_t win = ts1 > ts0, tstar = win ? ts1 : ts0;
+    SCAN_TRACE(lane == 0, 4, 0);  // candidate loads consumed
+    uint32_t hstar = 0, vstar = 1;
+    if (tstar < kWTT) {
+      const uint32_t own = __ffs(__ballot_sync(kFull, grp == win && first_bad == tstar)) - 1;
+      hstar = __shfl_sync(kFull, bh, own);
+      vstar = __shfl_sync(kFull, bv, own);
+    }
+    const uint32_t hp = win ? W.hp1 : W.hp0;
+    const uint64_t Lp = hp & 0x7fffffffu, stride = 4 + Lp;
+    const uint32_t lastp = hp >> 31;
+    const bool end_at_star = tstar < kWTT && !vstar;
+    const uint32_t n_hdr = tstar == kWTT ? kWTT : (end_at_star ? tstar : tstar + 1);
+    // closed forms of header t (headers 0..tstar-1 equal hp)
+    auto at = [&](uint32_t t, uint64_t& q, uint64_t& len, uint32_t& last, bool& start, uint64_t& send,
+                  uint32_t& nrec) {
+      q = p + (uint64_t)t * stride;
+      len = t < tstar ? Lp : (uint64_t)(hstar & 0x7fffffffu);
+      last = t < tstar ? lastp : (hstar >> 31);
+      start = t == 0 ? (p == r0) : (lastp != 0);
+      if (!lastp) send = sum + (uint64_t)t * Lp + len;
+      else send = t == 0 ? (start ? len : sum + len) : len;
+      nrec = lastp ? nr + t : nr;
+    };
+    uint32_t first_fail = kFull, my_code = STOP_NONE;
+#pragma unroll
+    for (uint32_t j = 0; j < kWJ; ++j) {
+      const uint32_t t = u + 16 * j;
+      if (grp != win || t >= n_hdr || first_fail != kFull) continue;
+      uint64_t q, len, send;
+      uint32_t last, nrec;
+      bool start;
+      at(t, q, len, last, start, send, nrec);
+      uint32_t code = STOP_NONE;
+      if (send > E.max_record_bytes) code = STOP_FRAG;
+      else if (q + 4 + len > E.R.tail) code = STOP_INCOMPLETE;
+      else if (nf + t >= E.FC || (start && nrec >= E.RC)) code = STOP_CAP;
+      if (code != STOP_NONE) { first_fail = t; my_code = code; }
+    }
+    const uint32_t tf = __reduce_min_sync(kFull, first_fail);
+    uint32_t code_f = STOP_NONE;
+    if (tf != kFull) code_f = __shfl_sync(kFull, my_code, __ffs(__ballot_sync(kFull, first_fail == tf)) - 1);
+    const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
+#pragma unroll
+    for (uint32_t j = 0; j < kWJ; ++j) {
+      const uint32_t t = u + 16 * j;
+      if (grp != win || t >= n_emit) continue;
+      uint64_t q, len, send;
+      uint32_t last, nrec;
+      bool start;
+      at(t, q, len, last, start, send, nrec);
+      emit_frag(E, nf + t, q, len, last, send, start, r0, f0, nrec);
+    }
+    uint64_t q, len, send;
+    uint32_t last, nrec;
+    bool start;
+    if (tf < n_hdr || end_at_star) {  // the stopping header records the outcome
+      const uint32_t t = tf < n_hdr ? tf : tstar;
+      at(t, q, len, last, start, send, nrec);
+      W.consumed = start ? q : r0;
+      W.kept = start ? nf + t : f0;
+      W.nr = nrec;
+      if (tf < n_hdr) {
+        W.status = code_f == STOP_FRAG ? CRK_E_FRAG
+                 : code_f == STOP_INCOMPLETE ? CRK_INCOMPLETE
+                 : (nrec > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
+      } else {
+        W.status = (start && q == E.R.tail) ? CRK_OK : CRK_INCOMPLETE;
+      }
+      W.stop = true;
+      return false;
+    }
+    // the last accepted header advances the state and the predictors
+    SCAN_TRACE(lane == 0, 1, n_hdr);
+    const uint32_t t = n_hdr - 1;
+    at(t, q, len, last, start, send, nrec);
+    W.p = q + 4 + len;
+    W.nf = nf + n_hdr;
+    if (last) {
+      W.nr = nrec + 1;
+      W.r0 = W.p;
+      W.sum = 0;
+      W.f0 = nf + n_hdr;
+    } else {
+      W.nr = nrec;
+      W.sum = send;
+      W.r0 = start ? q : r0;
+      W.f0 = start ? nf + t : f0;
+    }
+    if (tstar < kWTT) {
+      if (start && last) W.hp1 = hstar;
+      else if (!last) W.hp0 = hstar;
+    }
+    if (tstar == kWTT) return true;
+    miss = n_hdr <= 2 ? miss + 1 : 0;
+  }
+}
 
 __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
   const uint32_t ring = blockIdx.x;
@@ -66,7 +324,40 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     S.kept_frags = 0;
   }
   __syncthreads();
-  while (!S.done) {
+  const Env E{ix, R, cfg.max_record_bytes, fbase, rbase, FC, RC};
+  for (;;) {
+    const bool done = S.done, wide_mode = S.wide;
+    __syncthreads();  // everyone has read the mode before warp 0 / the round changes S
+    if (done) break;
+    if (!wide_mode) {
+      // warp rounds / chase passes in warp 0 until a stop or a long regular run; the others wait
+      if (warp == 0) {
+        Walk W{S.p, S.r0, S.sum, S.nf, S.nr, S.f0, S.hp[0], S.hp[1], false, 0, 0, 0};
+        const bool wide = warp_rounds(E, W, lane);
+        __syncwarp();
+        if (lane == 0) {
+          if (W.stop) {
+            S.consumed = W.consumed;
+            S.kept_frags = W.kept;
+            S.nr = W.nr;
+            S.status = W.status;
+            S.done = 1;
+          } else {
+            S.p = W.p;
+            S.r0 = W.r0;
+            S.sum = W.sum;
+            S.nf = W.nf;
+            S.nr = W.nr;
+            S.f0 = W.f0;
+            S.hp[0] = W.hp0;
+            S.hp[1] = W.hp1;
+            S.wide = wide;
+          }
+        }
+      }
+      __syncthreads();
+      continue;
+    }
     const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
     const uint32_t nf = S.nf, nr = S.nr, f0 = S.f0;
     // ---- both groups speculate from the true header at p; thread u owns candidates u + j*T
@@ -86,7 +377,7 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
       vv[j] = j < jn && q + 4 <= R.tail;
       const uint64_t a = q & ~3ull;
       w0[j] = vv[j] ? __ldg(reinterpret_cast<const uint32_t*>(R.base + (a & R.mask))) : 0u;
-      w1[j] = vv[j] ? __ldg(reinterpret_cast<const uint32_t*>(R.base + ((a + 4) & R.mask))) : 0u;
+      w1[j] = (vv[j] && (q & 3)) ? __ldg(reinterpret_cast<const uint32_t*>(R.base + ((a + 4) & R.mask))) : 0u;
     }
     uint32_t bh = 0, bv = 0;  // header and validity of this thread's first mismatching candidate
 #pragma unroll
@@ -120,40 +411,59 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     const uint32_t n_hdr = tstar == TT ? TT : (end_at_star ? tstar : tstar + 1);
     const uint32_t hstar = S.gh[wstar];
 
-    // per-header closed forms (headers 0..tstar-1 equal hpred); checks in the oracle's order
-    uint32_t codes[kJ];
-    uint32_t first_fail = 0xffffffffu;
-#pragma unroll
-    for (uint32_t j = 0; j < kJ; ++j) {
-      const uint32_t t = u + j * T;
+    // per-header closed forms (headers 0..tstar-1 equal hpred); checks in the oracle's order.  The checks
+    // are monotone along the run (a record's running length, the end of header t's data and the fragment
+    // / record counts only grow; with lastp every header 1..u*-1 is a whole record of length Lp), so
+    // headers 0, 1 and n_hdr - 1 passing means all pass, and the per-candidate search for the first
+    // failure (one more barrier) is skipped.
+    bool any_fail = false;
+    for (uint32_t k = 0; k < 3; ++k) {
+      const uint32_t t = k == 0 ? 0u : (k == 1 ? (n_hdr > 1 ? 1u : 0u) : (n_hdr ? n_hdr - 1 : 0u));
+      if (t >= n_hdr) continue;
       const uint64_t q = p + (uint64_t)t * stride;
       const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
       const bool start = (t == 0) ? (p == r0) : (lastp != 0);
-      uint64_t send;  // logical end of header t within its record (segmented prefix sum of lengths)
+      uint64_t send;
       if (!lastp) send = sum + (uint64_t)t * Lp + len;
       else send = (t == 0) ? (start ? len : sum + len) : len;
-      const uint32_t nrec = lastp ? nr + t : nr;  // completed records before header t
-      uint32_t code = STOP_NONE;
-      if (mine && j < jn && t < n_hdr) {
-        if (send > cfg.max_record_bytes) code = STOP_FRAG;
-        else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
-        else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
-      }
-      codes[j] = code;
-      if (code != STOP_NONE && first_fail == 0xffffffffu) first_fail = t;
+      const uint32_t nrec = lastp ? nr + t : nr;
+      any_fail |= send > cfg.max_record_bytes || q + 4 + len > R.tail || nf + t >= FC || (start && nrec >= RC);
     }
-    uint32_t my_code = STOP_NONE;
-#pragma unroll
-    for (uint32_t j = 0; j < kJ; ++j)
-      if (u + j * T == first_fail) my_code = codes[j];
-    const uint32_t fm = __reduce_min_sync(0xffffffffu, first_fail);
-    const uint32_t fown = __ffs(__ballot_sync(0xffffffffu, first_fail == fm)) - 1;
-    const uint32_t fc = __shfl_sync(0xffffffffu, my_code, fown);
-    if (lane == 0) { S.fmin[warp] = fm; S.fcode[warp] = fc; }
-    __syncthreads();
     uint32_t tf = 0xffffffffu, code_f = STOP_NONE;
-    for (uint32_t w = 0; w < nw; ++w)
-      if (S.fmin[w] < tf) { tf = S.fmin[w]; code_f = S.fcode[w]; }
+    if (any_fail) {
+      uint32_t codes[kJ];
+      uint32_t first_fail = 0xffffffffu;
+#pragma unroll
+      for (uint32_t j = 0; j < kJ; ++j) {
+        const uint32_t t = u + j * T;
+        const uint64_t q = p + (uint64_t)t * stride;
+        const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
+        const bool start = (t == 0) ? (p == r0) : (lastp != 0);
+        uint64_t send;  // logical end of header t within its record (segmented prefix sum of lengths)
+        if (!lastp) send = sum + (uint64_t)t * Lp + len;
+        else send = (t == 0) ? (start ? len : sum + len) : len;
+        const uint32_t nrec = lastp ? nr + t : nr;  // completed records before header t
+        uint32_t code = STOP_NONE;
+        if (mine && j < jn && t < n_hdr) {
+          if (send > cfg.max_record_bytes) code = STOP_FRAG;
+          else if (q + 4 + len > R.tail) code = STOP_INCOMPLETE;
+          else if (nf + t >= FC || (start && nrec >= RC)) code = STOP_CAP;
+        }
+        codes[j] = code;
+        if (code != STOP_NONE && first_fail == 0xffffffffu) first_fail = t;
+      }
+      uint32_t my_code = STOP_NONE;
+#pragma unroll
+      for (uint32_t j = 0; j < kJ; ++j)
+        if (u + j * T == first_fail) my_code = codes[j];
+      const uint32_t fm = __reduce_min_sync(0xffffffffu, first_fail);
+      const uint32_t fown = __ffs(__ballot_sync(0xffffffffu, first_fail == fm)) - 1;
+      const uint32_t fc = __shfl_sync(0xffffffffu, my_code, fown);
+      if (lane == 0) { S.fmin[warp] = fm; S.fcode[warp] = fc; }
+      __syncthreads();
+      for (uint32_t w = 0; w < nw; ++w)
+        if (S.fmin[w] < tf) { tf = S.fmin[w]; code_f = S.fcode[w]; }
+    }
     const uint32_t n_emit = tf < n_hdr ? tf : n_hdr;
 
 #pragma unroll
@@ -201,6 +511,7 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
       // the last accepted header advances the state and the predictors
       if (!stops_here && tf >= n_hdr && !end_at_star && t == n_hdr - 1) {
         S.wide = tstar == TT;
+        SCAN_TRACE(true, 3, n_hdr);
         S.p = q + 4 + len;
         S.nf = nf + n_hdr;
         if (last) {
@@ -224,6 +535,7 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
     }
     __syncthreads();
   }
+  SCAN_TRACE(threadIdx.x == 0, 0, 0);  // end marker
   if (threadIdx.x == 0) {
     crk_ring_result& rr = ix.res[ring];
     rr.status = S.status;
@@ -251,6 +563,18 @@ __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRings
 }
 
 }  // namespace
+
+#ifdef CRK_SCAN_TRACE
+extern "C" int crk_debug_scan_trace(unsigned long long* out, uint32_t* counts, int reset) {
+  if (out && cudaMemcpyFromSymbol(out, g_scan_trace, sizeof(g_scan_trace)) != cudaSuccess) return -100;
+  if (counts && cudaMemcpyFromSymbol(counts, g_scan_trace_n, sizeof(g_scan_trace_n)) != cudaSuccess) return -100;
+  if (reset) {
+    static const uint32_t zero[kTraceRings] = {};
+    if (cudaMemcpyToSymbol(g_scan_trace_n, zero, sizeof(zero)) != cudaSuccess) return -100;
+  }
+  return 0;
+}
+#endif
 
 cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s) {
   prof_mark(PROF_SCAN, true, s);

@@ -111,6 +111,44 @@ def test_scan_irregular_zero_fragments_and_regular_runs():
     compare_parse(T, 0, rb, s, cfg)
 
 
+@pytest.mark.parametrize("host", [False, True])
+def test_scan_chase_irregular_long_chains(host):
+    """Long runs of irregular fragment lengths (the scan's serial chase pass), interleaved with regular
+    runs (hand-back to the speculative rounds), across the ring wrap; then every stop inside a chase:
+    truncated windows, E_FRAG, fragment and record capacity."""
+    cfg = ocfg()
+    ctx = ctx_for(cfg)
+    g = gen.rng(4242)
+    cap = 1 << 22
+    ring = make_ring(cap, host)
+    head = cap - 300000
+    tail = head
+    for i in range(60):
+        L = O.call_header(i, gen.PROG, gen.VERS, gen.PROC_H2D) + O.put_u64(0) + \
+            O.put_opaque_var(gen.random_bytes(i, int(g.integers(0, 30000))).tobytes())
+        L += O.put_u64(len(L) - 52)
+        if i % 10 == 9:  # regular run: the speculative rounds take over again
+            lens = [64] * (len(L) // 64) + [len(L) % 64]
+        else:  # irregular, zero-length fragments included
+            lens = gen.split_points(1000 + i, len(L), 0, int(g.choice([8, 300, 4000])))
+        tail = place(ring, O.frame_lens(L, lens), tail)
+    rb = ring_np(ring)
+    idx = ctx.index(1, 1 << 20, 1 << 10)
+    idx.frame_scan([(ring, head, tail)])
+    s = compare_scan(idx.tables(), 0, rb, head, tail, 1 << 20, 1 << 10)
+    assert len(s.recs) == 60 and len(s.frags) > 20000
+    compare_parse(idx.tables(), 0, rb, s, cfg)
+    frag_ends = [f["phys"] + f["len"] for f in s.frags]
+    for t in [head + 3, frag_ends[5000] - 1, frag_ends[5000] + 2, frag_ends[12345], tail - 1]:
+        idx.frame_scan([(ring, head, t)])
+        compare_scan(idx.tables(), 0, rb, head, t, 1 << 20, 1 << 10)
+    for fpr, rpr, mrb in [(7000, 1 << 10, 1 << 32), (1 << 20, 13, 1 << 32), (1 << 20, 1 << 10, 20000)]:
+        c3 = crk.Context(0, frag_payload=65536, strict=1, prog=cfg.prog, vers=cfg.vers, max_record_bytes=mrb)
+        i3 = c3.index(1, fpr, rpr)
+        i3.frame_scan([(ring, head, tail)])
+        compare_scan(i3.tables(), 0, rb, head, tail, fpr, rpr, mrb)
+
+
 def test_scan_limits_frag_capacity_records():
     cfg = ocfg()
     ctx = ctx_for(cfg)

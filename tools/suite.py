@@ -227,9 +227,11 @@ def c4(ctx, irregular):
                                                          torch.cuda.current_stream().cuda_stream), "batch")
 
     ms = timed(dec, 10)
+    ms_scan = timed(lambda _: idx.frame_scan([(ring, 0, cur)]), 10)
     ok = bool((st == 0).all()) and all(torch.equal(o[:s.numel() * s.element_size()], s.view(torch.uint8).reshape(-1))
                                        for o, s in zip(outs, srcs))
     return {"records": len(calls), "items": len(reqs), "payload_bytes": total, "wire": cur, "ms": round(ms, 3),
+            "scan_ms": round(ms_scan, 3), "frags": int(idx.ring_results(1)[0]["n_frags"]),
             "decode_gbs": round(total / ms / 1e6, 1), "ok": ok}
 
 
@@ -276,19 +278,25 @@ def served(ctx, sizes_h2d, sizes_d2h, streams=1, reps=20):
 
 def main():
     build.build()
+    only = [x for x in os.environ.get("SUITE_ONLY", "").split(",") if x]
+    runs = {
+        "C1": lambda: c1(crk.Context(0)),
+        "C1_serve_one_record": lambda: serve_latency(crk.Context(0)),
+        "C2_matrixMul": lambda: c2(crk.Context(0)),
+        "C3_sweep": lambda: c3(crk.Context(0)),
+        "C4_typed_regular": lambda: c4(crk.Context(0), False),
+        "C4_typed_irregular": lambda: c4(crk.Context(0), True),
+        "NEXT1_striped_1GiB_16_rings": lambda: served(crk.Context(0), [64 * MiB] * 16, [], streams=16),
+        "NEXT1_single_1GiB_1_ring": lambda: served(crk.Context(0), [GiB], [], streams=1),
+        "NEXT2_cusolver_100_iters": lambda: served(crk.Context(0), [900 * 900 * 8] * 100, [900 * 8] * 100,
+                                                   streams=1, reps=10),
+        "NEXT2_histogram": lambda: served(crk.Context(0), [64 * MiB], [256 * 4], streams=1),
+    }
     out = {}
-    ctx = crk.Context(0)
     t0 = time.time()
-    out["C1"] = c1(ctx)
-    out["C1_serve_one_record"] = serve_latency(crk.Context(0))
-    out["C2_matrixMul"] = c2(crk.Context(0))
-    out["C3_sweep"] = c3(crk.Context(0))
-    out["C4_typed_regular"] = c4(crk.Context(0), False)
-    out["C4_typed_irregular"] = c4(crk.Context(0), True)
-    out["NEXT1_striped_1GiB_16_rings"] = served(crk.Context(0), [64 * MiB] * 16, [], streams=16)
-    out["NEXT1_single_1GiB_1_ring"] = served(crk.Context(0), [GiB], [], streams=1)
-    out["NEXT2_cusolver_100_iters"] = served(crk.Context(0), [900 * 900 * 8] * 100, [900 * 8] * 100, streams=1, reps=10)
-    out["NEXT2_histogram"] = served(crk.Context(0), [64 * MiB], [256 * 4], streams=1)
+    for name, fn in runs.items():
+        if not only or any(name.startswith(o) for o in only):
+            out[name] = fn()
     out["wall_s"] = round(time.time() - t0, 1)
     print(json.dumps(out))
 
