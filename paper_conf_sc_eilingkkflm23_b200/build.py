@@ -60,5 +60,16 @@ def build_trace() -> str:
     return out
 
 
+def build_variant(name: str, defines: list[str]) -> str:
+    """Experiment build with extra -D defines (e.g. scan prefetch knobs) -> lib/libcrk_<name>.so."""
+    out = os.path.join(PKG, "lib", f"libcrk_{name}.so")
+    r = subprocess.run([NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-o", out, *sources()], capture_output=True,
+                       text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError(f"nvcc failed building {out}")
+    return out
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

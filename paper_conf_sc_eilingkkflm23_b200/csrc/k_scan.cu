@@ -24,7 +24,7 @@ constexpr uint32_t kNoPred = 0xffffffffu;  // a predictor value no header is exp
 constexpr uint32_t kJ = 4;                 // candidate headers per thread and CTA round (independent loads)
 constexpr uint32_t kWJ = 2;                // candidate headers per lane and warp round
 constexpr uint32_t kWTT = 16 * kWJ;        // candidates per group and warp round (16 lanes per group)
-constexpr uint32_t kChase = 512;           // max headers per chase pass (irregular framing)
+constexpr uint32_t kChase = 4096;          // max headers per chase pass (irregular framing)
 constexpr uint32_t kFull = 0xffffffffu;
 
 #ifdef CRK_SCAN_TRACE
@@ -110,52 +110,153 @@ __device__ __forceinline__ void emit_frag(const Env& E, uint32_t nf, uint64_t q,
   }
 }
 
-// Chase pass: the serial walk of the chain, one dependent header load per fragment, for framing no
-// predictor follows.  The per-header logic is the rounds' with u* = 0, in or_frame_scan's order
-// E_FRAG -> INCOMPLETE -> capacity.  Stops after kChase headers, at a stop, or at two equal consecutive
-// headers (a regular run the predictors can take over again).  Lanes walk the same chain (broadcast loads).
-__device__ void chase(const Env& E, Walk& W, bool writer) {
+// L2 prefetch of a ring span through the TMA unit (no registers, no completion to wait for).
+__device__ __forceinline__ void prefetch_l2(const RingDesc& R, uint64_t c, uint32_t bytes) {
+  const uint64_t o = c & R.mask, room = R.mask + 1 - o;
+  const uint32_t n = room < bytes ? (uint32_t)room : bytes;
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(R.base + o), "r"(n) : "memory");
+}
+
+// Chase pass: the serial walk of the chain, for framing no predictor follows.  It runs in batches of 32
+// hops.  The walk itself carries only the chain (p -> p + 4 + len(be32(p))): every lane follows it
+// (broadcast loads) and lane k keeps hop k's cursor and header.  All per-header work -- the checks in
+// or_frame_scan's order E_FRAG -> INCOMPLETE -> capacity, the segmented prefix sum of lengths (logical
+// starts), record boundaries, the index writes -- is then done for the 32 hops at once with warp scans,
+// so a hop costs one load latency.  Hops past a failing header are walked but discarded (reads stay
+// inside the ring).  Once a pass is long (an irregular stream), the TMA prefetches the ring ahead of
+// the walk into L2 (kPfLead bytes ahead), so header reads hit L2 instead of HBM / the host link.
+// Stops after kChase headers, at a stop, or at two equal consecutive headers (a regular run the
+// predictors can take over again).
+#ifndef CRK_PF_LEAD
+#define CRK_PF_LEAD (1ull << 20)  // prefetch frontier lead over the walk (bytes; 0 = no prefetch)
+#endif
+#ifndef CRK_PF_CHUNK
+#define CRK_PF_CHUNK 65536u       // bytes per prefetch instruction (power of 2)
+#endif
+constexpr uint64_t kPfLead = CRK_PF_LEAD;
+constexpr uint32_t kPfChunk = CRK_PF_CHUNK;
+__device__ void chase(const Env& E, Walk& W, uint32_t lane) {
+  const uint64_t tail = E.R.tail;
   uint32_t prev = kNoPred;
-  for (uint32_t k = 0; k < kChase; ++k) {
-    const bool start = W.p == W.r0;
-    if (W.p + 4 > E.R.tail) {  // no readable header: the window ends here
+  uint64_t pf = 0;  // prefetch frontier (cursor), from the second batch of a pass on
+  for (uint32_t b = 0; b < kChase / 32; ++b) {
+    if (b == 1) pf = W.p & ~15ull;  // a long pass: start prefetching
+    // ---- walk up to 32 hops
+    uint64_t q = W.p, myq = 0;
+    uint32_t myh = 0, n = 0, hw = prev;
+#pragma unroll 1
+    for (; n < 32; ++n) {
+      if (q + 4 > tail) break;
+      if (CRK_PF_LEAD && b && lane == 0) {
+        const uint64_t want = min(q + kPfLead, tail);
+        for (uint32_t i = 0; i < 4 && pf < want; ++i) {
+          prefetch_l2(E.R, pf, kPfChunk);
+          pf += kPfChunk - (pf & (kPfChunk - 1));  // chunks aligned to kPfChunk (never cross the wrap)
+        }
+      }
+      const uint64_t a = q & ~3ull;
+      const uint32_t w0 = __ldg(reinterpret_cast<const uint32_t*>(E.R.base + (a & E.R.mask)));
+      const uint32_t w1 = __ldg(reinterpret_cast<const uint32_t*>(E.R.base + ((a + 4) & E.R.mask)));
+      const uint32_t h = join_hdr(q, w0, w1);
+      if (lane == n) { myq = q; myh = h; }
+      q += 4 + (uint64_t)(h & 0x7fffffffu);
+      if (h == hw) { ++n; break; }  // two equal headers: the batch ends here (the rounds take over)
+      hw = h;
+    }
+    SCAN_TRACE(lane == 0, 2, n);
+    // ---- per-hop closed forms (lane k = hop k)
+    const uint32_t vmask = n == 32 ? kFull : (1u << n) - 1;
+    const bool v = lane < n;
+    const uint64_t len = v ? (uint64_t)(myh & 0x7fffffffu) : 0ull;
+    const uint32_t last = v ? myh >> 31 : 0u;
+    const uint32_t lastm = __ballot_sync(kFull, last);
+    const uint32_t startm = ((lastm << 1) | (W.p == W.r0 ? 1u : 0u)) & vmask;
+    const bool start = (startm >> lane) & 1;
+    uint64_t P = len;  // inclusive prefix of lengths over the batch
+#pragma unroll
+    for (uint32_t o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(kFull, P, o);
+      if (lane >= o) P += y;
+    }
+    const uint64_t Ex = P - len;
+    const uint32_t below = startm & (lane == 31 ? kFull : (2u << lane) - 1);
+    const int j = below ? 31 - __clz(below) : -1;  // this hop's record began at hop j of the batch
+    const uint64_t Ej = __shfl_sync(kFull, Ex, j < 0 ? 0 : j);
+    const uint64_t qj = __shfl_sync(kFull, myq, j < 0 ? 0 : j);
+    const uint64_t send = j >= 0 ? P - Ej : W.sum + P;  // logical end of this fragment in its record
+    const uint64_t rbeg = j >= 0 ? qj : W.r0;
+    const uint32_t f0 = j >= 0 ? W.nf + (uint32_t)j : W.f0;
+    const uint32_t nrec = W.nr + __popc(lastm & ((1u << lane) - 1));
+    uint32_t code = STOP_NONE;
+    if (v) {
+      if (send > E.max_record_bytes) code = STOP_FRAG;
+      else if (myq + 4 + len > tail) code = STOP_INCOMPLETE;
+      else if (W.nf + lane >= E.FC || (start && nrec >= E.RC)) code = STOP_CAP;
+    }
+    const uint32_t failm = __ballot_sync(kFull, code != STOP_NONE);
+    const uint32_t hprev = __shfl_up_sync(kFull, myh, 1);
+    const uint32_t eqm = __ballot_sync(kFull, v && myh == (lane ? hprev : prev));
+    const uint32_t tf = failm ? __ffs(failm) - 1 : 32u, te = eqm ? __ffs(eqm) - 1 : 32u;
+    const bool fail_stop = tf < n && tf <= te;
+    const uint32_t n_acc = fail_stop ? tf : (te < n ? te + 1 : n);
+    if (lane < n_acc) {
+      const uint64_t fs = E.fbase + W.nf + lane;
+      E.ix.frag_phys[fs] = myq + 4;
+      E.ix.frag_lstart[fs] = send - len;
+      E.ix.frag_hdr[fs] = myh;
+      if (last) {
+        const uint64_t rs = E.rbase + nrec;
+        E.ix.rec_begin[rs] = start ? myq : rbeg;
+        E.ix.rec_len[rs] = send;
+        E.ix.rec_frag0[rs] = (uint32_t)(E.fbase + f0);
+        E.ix.rec_nfrags[rs] = W.nf + lane - f0 + 1;
+      }
+    }
+    if (fail_stop) {  // hop tf's check failed: the outcome is recorded there
+      const uint32_t c = __shfl_sync(kFull, code, tf);
+      const uint32_t nr_t = __shfl_sync(kFull, nrec, tf);
+      const bool st_t = (startm >> tf) & 1;
+      W.consumed = st_t ? __shfl_sync(kFull, myq, tf) : __shfl_sync(kFull, rbeg, tf);
+      W.kept = st_t ? W.nf + tf : __shfl_sync(kFull, f0, tf);
+      W.nr = nr_t;
+      W.status = c == STOP_FRAG ? CRK_E_FRAG : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
+               : (nr_t > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
       W.stop = true;
-      W.status = (start && W.p == E.R.tail) ? CRK_OK : CRK_INCOMPLETE;
-      break;
+      return;
     }
-    uint32_t w0, w1;
-    load_hdr(E.R, W.p, true, w0, w1);
-    const uint32_t h = join_hdr(W.p, w0, w1);
-    const uint64_t len = h & 0x7fffffffu;
-    const uint32_t last = h >> 31;
-    const uint64_t send = start ? len : W.sum + len;
-    bool fail = true;
-    if (send > E.max_record_bytes) W.status = CRK_E_FRAG;
-    else if (W.p + 4 + len > E.R.tail) W.status = CRK_INCOMPLETE;
-    else if (W.nf >= E.FC || (start && W.nr >= E.RC)) W.status = W.nr > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY;
-    else fail = false;
-    if (fail) { W.stop = true; break; }
-    if (writer) emit_frag(E, W.nf, W.p, len, last, send, start, W.r0, W.f0, W.nr);
-    SCAN_TRACE(writer, 2, 1);
-    W.p += 4 + len;
-    W.nf++;
-    if (last) {
-      if (start) W.hp1 = h;
-      W.nr++;
-      W.r0 = W.p;
-      W.sum = 0;
-      W.f0 = W.nf;
-    } else {
-      W.hp0 = h;
-      W.sum = send;
+    if (n_acc) {  // advance the state to after hop n_acc - 1 and update the predictors
+      const uint32_t L = n_acc - 1, am = n_acc == 32 ? kFull : (1u << n_acc) - 1;
+      const uint64_t qL = __shfl_sync(kFull, myq, L), lenL = __shfl_sync(kFull, len, L);
+      const uint64_t sendL = __shfl_sync(kFull, send, L), rbegL = __shfl_sync(kFull, rbeg, L);
+      const uint32_t f0L = __shfl_sync(kFull, f0, L), nrecL = __shfl_sync(kFull, nrec, L);
+      const uint32_t hL = __shfl_sync(kFull, myh, L);
+      const uint32_t singlem = __ballot_sync(kFull, start && last) & am, nonlastm = ~lastm & am;
+      if (singlem) W.hp1 = __shfl_sync(kFull, myh, 31 - __clz(singlem));
+      if (nonlastm) W.hp0 = __shfl_sync(kFull, myh, 31 - __clz(nonlastm));
+      W.p = qL + 4 + lenL;
+      W.nf += n_acc;
+      if (hL >> 31) {
+        W.nr = nrecL + 1;
+        W.r0 = W.p;
+        W.sum = 0;
+        W.f0 = W.nf;
+      } else {
+        W.nr = nrecL;
+        W.sum = sendL;
+        W.r0 = rbegL;
+        W.f0 = f0L;
+      }
+      prev = hL;
     }
-    if (h == prev) break;
-    prev = h;
-  }
-  if (W.stop) {
-    const bool start = W.p == W.r0;
-    W.consumed = W.r0;
-    W.kept = start ? W.nf : W.f0;
+    if (te < n) return;  // two equal headers: back to the speculative rounds
+    if (n < 32) {        // no readable header at W.p: the window ends here
+      const bool st = W.p == W.r0;
+      W.status = (st && W.p == tail) ? CRK_OK : CRK_INCOMPLETE;
+      W.consumed = W.r0;
+      W.kept = st ? W.nf : W.f0;
+      W.stop = true;
+      return;
+    }
   }
 }
 
@@ -170,7 +271,7 @@ __device__ bool warp_rounds(const Env& E, Walk& W, uint32_t lane) {
   uint32_t miss = 0;
   for (;;) {
     if (miss >= 2) {
-      chase(E, W, lane == 0);
+      chase(E, W, lane);
       if (W.stop) return false;
       miss = 0;
       continue;
