@@ -319,6 +319,48 @@ int crk_serve_graph_create(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const
 int crk_graph_launch(crk_graph* graph, crk_stream_t stream);
 void crk_graph_destroy(crk_graph* graph);
 
+/* ---------------------------------------------------------------- persistent server
+ * The API-latency side of the paper: Cricket's overhead tracks the number of forwarded calls, most of them
+ * small (Fig. 6 at P:228-234).  crk_server_start launches ONE resident CTA on `stream` that
+ * polls a doorbell and runs every published step in place -- the crk_serve semantics above (scan, parse,
+ * per-record decisions, HtoD copies, framed replies), with the same index tables and per-ring results --
+ * with no kernel launch per step.  It is meant for streams of small calls (control RPCs, small memcpys):
+ * one CTA moves the payloads, so bulk batches belong to crk_serve.
+ *
+ * Protocol.  The bell is caller-owned memory the device can read and write (mapped pinned host memory from
+ * crk_host_alloc, or device memory).  To run a step the host writes head/tail/send_off for every ring,
+ * then increments `seq` (a plain store after the others; x86 stores are ordered).  The kernel sees the new
+ * seq (system-scope acquire), serves the windows, copies the per-ring results into `res`, sets `status`
+ * and the device-timer stamps, and publishes done_seq = seq (system-scope release).  A window with
+ * tail < head or longer than its ring is served as an empty ring with status CRK_E_ARG.  Setting `stop`
+ * (then bumping seq) ends the kernel.  One step at a time: the host waits for done_seq == seq before
+ * writing the next.
+ *
+ * Ownership.  While the server runs, it owns `ctx`'s scratch and `idx`: issue no other crk call on them
+ * (other contexts are unaffected).  The kernel runs until stopped, so any host call that waits for the
+ * whole device (cudaDeviceSynchronize, and allocator calls that synchronise implicitly) blocks until
+ * crk_server_stop; use stream-ordered work on other non-blocking streams meanwhile.
+ * The index must have max_records <= 1024 and 2 * max_records <=
+ * the context's max_jobs.  crk_server_stop sets stop, waits for the kernel to exit and frees the handle
+ * (not the bell). */
+typedef struct {
+  volatile uint64_t seq;       /* host -> device: step number (increment to run a step) */
+  volatile uint64_t stop;      /* host -> device: nonzero ends the kernel at the next seq change */
+  uint64_t head[CRK_MAX_RINGS];
+  uint64_t tail[CRK_MAX_RINGS];
+  uint64_t send_off[CRK_MAX_RINGS];
+  volatile uint64_t done_seq;  /* device -> host: last completed step */
+  volatile int32_t status;     /* device -> host: CRK_OK, or CRK_E_ARG when the step had an invalid window */
+  uint32_t pad_;
+  volatile uint64_t t_begin_ns, t_end_ns; /* device %globaltimer at the step's start (seq seen) and end */
+  crk_ring_result res[CRK_MAX_RINGS];     /* device -> host: per-ring results of the last step */
+} crk_server_bell;
+typedef struct crk_server crk_server;
+int crk_server_start(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings,
+                     const crk_ring* send_rings, uint64_t region_base, uint64_t region_bytes, crk_server_bell* bell,
+                     crk_stream_t stream, crk_server** out);
+int crk_server_stop(crk_server* server);
+
 /* ---------------------------------------------------------------- memory utilities
  * Pinned, mapped, portable host memory for rings (cudaHostAlloc; with UVA the returned pointer is
  * also the device address), and a synchronous device->host copy for inspecting index tables. */

@@ -80,6 +80,14 @@ class ReplyReq(C.Structure):
                 ("value", C.c_uint64), ("src", C.c_void_p), ("count", C.c_uint64)]
 
 
+class ServerBell(C.Structure):
+    """crk_server_bell (include/crk.h): the persistent server's doorbell and result block."""
+    _fields_ = [("seq", C.c_uint64), ("stop", C.c_uint64), ("head", C.c_uint64 * MAX_RINGS),
+                ("tail", C.c_uint64 * MAX_RINGS), ("send_off", C.c_uint64 * MAX_RINGS), ("done_seq", C.c_uint64),
+                ("status", C.c_int32), ("pad_", C.c_uint32), ("t_begin_ns", C.c_uint64), ("t_end_ns", C.c_uint64),
+                ("res", RingResult * MAX_RINGS)]
+
+
 _lib = None
 vp, u32, u64, i32 = C.c_void_p, C.c_uint32, C.c_uint64, C.c_int32
 
@@ -118,6 +126,9 @@ def lib():
             "crk_serve_graph_create": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(CRing), u64, u64, vp,
                                                  C.POINTER(vp)]),
             "crk_graph_launch": (C.c_int, [vp, vp]),
+            "crk_server_start": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(CRing), u64, u64, vp, vp,
+                                           C.POINTER(vp)]),
+            "crk_server_stop": (C.c_int, [vp]),
             "crk_graph_destroy": (None, [vp]),
             "crk_host_alloc": (C.c_int, [u64, C.POINTER(vp)]),
             "crk_host_free": (None, [vp]),
@@ -561,5 +572,55 @@ class ServeGraph:
     def __del__(self):
         try:
             self.close()
+        except Exception:
+            pass
+
+
+class Server:
+    """Persistent server (crk_server_start): one resident CTA serving each step the host publishes in a
+    mapped pinned doorbell (ServerBell).  step() writes the windows, bumps seq and spins until the device
+    publishes done_seq; it returns the per-ring results, the step status and the device service time."""
+
+    def __init__(self, index: "Index", rings, send_rings, region_base: int, region_bytes: int, stream=None):
+        self.index = index
+        self.n = len(rings)
+        self.buf = HostBuffer(C.sizeof(ServerBell))
+        self.buf.np[:] = 0
+        self.bell = ServerBell.from_address(self.buf.ptr)
+        self.rings, self.send_rings = list(rings), list(send_rings)
+        self.stream = stream if stream is not None else torch.cuda.Stream()
+        cr = (CRing * self.n)(*[r.c() for r in self.rings])
+        sr = (CRing * self.n)(*[r.c() for r in self.send_rings])
+        h = vp()
+        _check(lib().crk_server_start(index.ctx.h, index.h, self.n, cr, sr, region_base, region_bytes, self.buf.ptr,
+                                      _stream(self.stream), C.byref(h)), "crk_server_start")
+        self.h = h.value
+        index.n_rings = self.n
+
+    def step(self, windows, send_offs, timeout_s: float = 30.0) -> dict:
+        import time
+        b = self.bell
+        for r, (head, tail) in enumerate(windows):
+            b.head[r] = head
+            b.tail[r] = tail
+            b.send_off[r] = send_offs[r]
+        seq = b.seq + 1
+        b.seq = seq
+        t0 = time.perf_counter()
+        while b.done_seq != seq:
+            if time.perf_counter() - t0 > timeout_s:
+                raise CrkError(E_CUDA, "crk_server step timed out")
+        res = [dict(status=x.status, n_records=x.n_records, n_frags=x.n_frags, rec_base=x.rec_base,
+                    consumed=x.consumed, reply_bytes=x.reply_bytes) for x in b.res[:self.n]]
+        return {"status": b.status, "results": res, "device_ns": b.t_end_ns - b.t_begin_ns}
+
+    def stop(self):
+        if self.h:
+            h, self.h = self.h, None
+            _check(lib().crk_server_stop(h), "crk_server_stop")
+
+    def __del__(self):
+        try:
+            self.stop()
         except Exception:
             pass

@@ -272,6 +272,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.tile_shift = (uint32_t)__builtin_ctz(cfg.tile_bytes);
   d.max_record_bytes = cfg.max_record_bytes;
   d.scan_threads = cfg.scan_threads;
+  d.tl = nullptr;
   d.stages = cfg.mover_stages;
   d.run = cfg.mover_run;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
@@ -772,6 +773,84 @@ void crk_graph_destroy(crk_graph* G) {
   cudaGraphExecDestroy(G->exec);
   cudaGraphDestroy(G->graph);
   delete G;
+}
+
+#ifdef CRK_TIMELINE
+// Diagnostic build only: kernels of this context stamp [min start, max end] per stage into dev_buf
+// (TL_STAGES x 2 u64, device memory; nullptr turns it off).
+int crk_debug_timeline(crk_ctx* c, unsigned long long* dev_buf) {
+  if (!c) return CRK_E_ARG;
+  c->cd.tl = dev_buf;
+  return CRK_OK;
+}
+#endif
+
+struct crk_server {
+  crk_ctx* ctx;
+  int device;
+  cudaStream_t stream;
+  crk_server_bell* bell;
+  bool host_bell;  // mapped host memory: the CPU writes it directly
+};
+
+namespace {
+// Writes `stop` and bumps `seq` (CPU stores for a host bell, a copy on a private stream otherwise).
+int server_signal(crk_server* S, uint64_t stop) {
+  if (S->host_bell) {
+    S->bell->stop = stop;
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    S->bell->seq = S->bell->seq + 1;
+    return CRK_OK;
+  }
+  cudaStream_t s;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  uint64_t seq = 0;
+  cudaError_t e = cudaMemcpyAsync(&seq, (const void*)&S->bell->seq, 8, cudaMemcpyDefault, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  seq += 1;
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)&S->bell->stop, &stop, 8, cudaMemcpyDefault, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync((void*)&S->bell->seq, &seq, 8, cudaMemcpyDefault, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  return e == cudaSuccess ? CRK_OK : cuda_fail(e);
+}
+}  // namespace
+
+int crk_server_start(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings, const crk_ring* send_rings,
+                     uint64_t region_base, uint64_t region_bytes, crk_server_bell* bell, crk_stream_t stream,
+                     crk_server** out) {
+  if (!c || !x || x->ctx != c || !rings || !send_rings || !bell || !out) return CRK_E_ARG;
+  *out = nullptr;
+  if (n_rings == 0 || n_rings > x->ix.max_rings || n_rings > (uint32_t)CRK_MAX_RINGS) return CRK_E_ARG;
+  for (uint32_t r = 0; r < n_rings; ++r)
+    if (!ring_ok(rings[r]) || !ring_ok(send_rings[r])) return CRK_E_ARG;
+  if (x->ix.max_records > crk::server_threads() || 2ull * x->ix.max_records > c->sc.max_jobs) return CRK_E_CAPACITY;
+  DeviceGuard g(c->device);
+  cudaPointerAttributes a;
+  CK(cudaPointerGetAttributes(&a, bell));
+  crk_server* S = new (std::nothrow) crk_server;
+  if (!S) return CRK_E_CAPACITY;
+  S->ctx = c;
+  S->device = c->device;
+  S->stream = (cudaStream_t)stream;
+  S->bell = bell;
+  S->host_bell = a.type == cudaMemoryTypeHost;
+  const cudaError_t e = launch_server(x->ix, c->cd, c->sc, c->d_schemas, bell, n_rings, rings, send_rings,
+                                      region_base, region_bytes, S->stream);
+  if (e != cudaSuccess) { delete S; return cuda_fail(e); }
+  *out = S;
+  return CRK_OK;
+}
+
+int crk_server_stop(crk_server* S) {
+  if (!S) return CRK_E_ARG;
+  DeviceGuard g(S->device);
+  int st = server_signal(S, 1);
+  const cudaError_t e = cudaStreamSynchronize(S->stream);
+  delete S;
+  if (st != CRK_OK) return st;
+  return e == cudaSuccess ? CRK_OK : cuda_fail(e);
 }
 
 int crk_host_alloc(uint64_t bytes, void** out) {

@@ -10,6 +10,14 @@ namespace crk {
 
 __device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }
 
+// Loads of ring bytes that stay constant for a kernel's lifetime go through the read-only path.  The
+// persistent server (k_server.cu) sees rings change under it, so it defines these as coherent loads.
+#ifdef CRK_COHERENT_LOADS
+#define CRK_RO_LD(p) __ldcg(p)
+#else
+#define CRK_RO_LD(p) __ldg(p)
+#endif
+
 // Byte at ring cursor c (RFC 5531 §11 stream position), wrap at cap (reading R16).
 __device__ __forceinline__ uint8_t ring_byte(const RingDesc& R, uint64_t c) { return R.base[c & R.mask]; }
 
@@ -24,7 +32,11 @@ __device__ __forceinline__ uint32_t ring_be32(const RingDesc& R, uint64_t c) {
 // 16-byte streaming load of an aligned chunk (read-only for the kernel's lifetime).
 __device__ __forceinline__ uint4 ld16_stream(const void* p) {
   uint4 r;
+#ifdef CRK_COHERENT_LOADS
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+#else
   asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+#endif
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
                : "l"(p));
   return r;
@@ -69,6 +81,27 @@ __device__ __forceinline__ uint4 swap16(uint4 v, uint32_t esize) {
 }
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+
+// RFC 4506 §3: bytes of zero pad after n bytes of opaque / array data
+__device__ __forceinline__ uint64_t pad4(uint64_t n) { return (4 - (n & 3)) & 3; }
+
+// Diagnostic timeline (-DCRK_TIMELINE builds; tools/timeline.py): per stage, the earliest start and the
+// latest end over the CTAs of a launch, from %globaltimer (ns).
+enum : uint32_t { TL_SCAN = 0, TL_PARSE = 1, TL_PLAN = 2, TL_MOVE = 3, TL_FUSED = 4, TL_STAGES = 8 };
+#ifdef CRK_TIMELINE
+__device__ __forceinline__ unsigned long long tl_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TL_BEGIN(cfg, st) \
+  do { if ((cfg).tl && threadIdx.x == 0) atomicMin((cfg).tl + 2 * (st), tl_now()); } while (0)
+#define TL_END(cfg, st) \
+  do { if ((cfg).tl && threadIdx.x == 0) atomicMax((cfg).tl + 2 * (st) + 1, tl_now()); } while (0)
+#else
+#define TL_BEGIN(cfg, st) do { } while (0)
+#define TL_END(cfg, st) do { } while (0)
+#endif
 
 // Block-wide min of a u32 (all threads must call).  smem: >= 32 words.
 __device__ __forceinline__ uint32_t block_min_u32(uint32_t v, uint32_t* smem) {

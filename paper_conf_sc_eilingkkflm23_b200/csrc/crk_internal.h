@@ -110,6 +110,7 @@ struct ConfigDev {
   uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
   uint32_t scan_threads, stages, run, pad_;
   uint64_t max_record_bytes;
+  unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };
 
 // ---- launchers (defined in the k_*.cu files) ------------------------------------------------------
@@ -175,6 +176,12 @@ constexpr uint32_t kSmallServe = 1024;
 cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, uint32_t n_rings,
                                     const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
                                     uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s);
+
+// Persistent server (k_server.cu): one resident CTA of server_threads() threads.
+uint32_t server_threads();
+cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SchemaTable* schemas,
+                          crk_server_bell* bell, uint32_t n_rings, const crk_ring* rings, const crk_ring* send_rings,
+                          uint64_t region_base, uint64_t region_bytes, cudaStream_t s);
 
 // host-visible counter of our kernel launches
 void count_launch(int n = 1);

@@ -1,0 +1,217 @@
+// Serve planning helpers (oracle or_serve decisions, reply jobs, block sums) shared by the planning
+// kernels (k_plan.cu) and the persistent server (k_server.cu).
+#pragma once
+#include "crk_device.cuh"
+
+namespace crk {
+
+namespace {
+
+constexpr uint32_t kNotFound = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t elem_size_k(uint32_t kind) {
+  switch (kind) {
+    case CRK_K_OPAQUE_VAR: case CRK_K_OPAQUE_FIX: return 1;
+    case CRK_K_I32_VAR: case CRK_K_U32_VAR: case CRK_K_F32_VAR:
+    case CRK_K_I32_FIX: case CRK_K_U32_FIX: case CRK_K_F32_FIX: return 4;
+    case CRK_K_I64_VAR: case CRK_K_U64_VAR: case CRK_K_F64_VAR:
+    case CRK_K_I64_FIX: case CRK_K_U64_FIX: case CRK_K_F64_FIX: return 8;
+    default: return 0;
+  }
+}
+
+// xid -> dense id of the earliest record carrying it (reading R11)
+__device__ __forceinline__ uint32_t xid_lookup(const IndexDev& ix, uint32_t xid) {
+  uint32_t h = (xid * 0x9E3779B1u) & ix.hash_mask;
+  for (;;) {
+    const unsigned long long k = ix.xid_hash[h];
+    if (k == ~0ull) return kNotFound;
+    if ((uint32_t)(k >> 32) == xid) return (uint32_t)k;
+    h = (h + 1) & ix.hash_mask;
+  }
+}
+
+__device__ __forceinline__ uint64_t wire_of(uint64_t Ll, uint32_t F) {
+  const uint64_t nfr = Ll == 0 ? 1 : (Ll + F - 1) / F;  // reading R3: >= 1 fragment, no empty trailer
+  return Ll + 4 * nfr;
+}
+
+__device__ __forceinline__ Job dec_job(uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec, uint32_t es) {
+  Job j{};
+  j.type = nbytes ? JOB_DEC : JOB_NONE;
+  j.esize = es;
+  j.rec = rec;
+  j.out_start = dst;
+  j.out_end = dst + nbytes;
+  j.loff = loff;
+  return j;
+}
+
+// ---- serve: statuses, HtoD decode jobs and reply sizes (pass 1) --------------------------------
+__device__ __forceinline__ void reply_words(Piece& p, uint32_t xid, int32_t err, bool with_len, uint64_t n) {
+  p = Piece{};
+  p.type = PIECE_WORDS;
+  p.loff = 0;
+  p.words[0] = xid;  // RFC 5531 §9: xid, REPLY, MSG_ACCEPTED, verf AUTH_NONE (0, len 0), SUCCESS
+  p.words[1] = 1;
+  p.words[2] = 0;
+  p.words[3] = 0;
+  p.words[4] = 0;
+  p.words[5] = 0;
+  p.words[6] = (uint32_t)err;  // mem_result discriminant (reading R10)
+  if (with_len) p.words[7] = (uint32_t)n;
+  p.nbytes = with_len ? 32 : 28;
+}
+
+// Serve decisions for dense record d (oracle or_serve): final status, reply discriminant (-1: no reply),
+// reply logical length, and the HtoD decode job.
+__device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev& cfg, uint32_t d, uint64_t region_base,
+                                             uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job) {
+  st = ix.p_status[d];
+  const uint32_t proc = ix.p_proc[d];
+  err = -1;
+  Ll = 0;
+  job = Job{};
+  if (st == CRK_OK && xid_lookup(ix, ix.p_xid[d]) != d) st = CRK_E_XID;
+  const uint64_t b = (uint64_t)d * kMaxItems;
+  if (st == CRK_OK && proc == cfg.proc_h2d) {
+    const uint64_t ptr = ix.p_value[b], nb = ix.p_count[b + 1], size = ix.p_value[b + 2];
+    const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
+    if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
+    else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
+    else { err = 0; job = dec_job(ptr, m, ix.p_off[b + 1], d, 1); }
+    Ll = 28;
+  } else if (st == CRK_OK && proc == cfg.proc_d2h) {
+    const uint64_t ptr = ix.p_value[b], size = ix.p_value[b + 1];
+    if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
+      st = CRK_E_PTR; err = 1; Ll = 28;
+    } else {
+      err = 0; Ll = 32 + size + pad4(size);
+    }
+  }
+}
+
+// The reply of record d as an encode job (pieces at 2d, 2d+1) written at send-ring cursor `off`.
+__device__ __forceinline__ Job serve_reply_job(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, uint32_t d,
+                                               uint32_t ring, int32_t err, uint64_t off, uint64_t w) {
+  Job job{};
+  if (err < 0) return job;
+  const uint64_t b = (uint64_t)d * kMaxItems;
+  const bool d2h = ix.p_proc[d] == cfg.proc_d2h && err == 0;
+  const uint64_t n = d2h ? ix.p_value[b + 1] : 0;
+  Piece* P = sc.pieces + 2ull * d;
+  reply_words(P[0], ix.p_xid[d], err, d2h, n);
+  uint32_t np = 1;
+  uint64_t Ll = P[0].nbytes;
+  if (d2h) {
+    Piece q{};
+    q.type = PIECE_DATA;
+    q.loff = 32;
+    q.nbytes = n;
+    q.src = ix.p_value[b];
+    q.esize = 1;
+    P[1] = q;
+    np = 2;
+    Ll = 32 + n + pad4(n);
+  }
+  job.type = JOB_ENC;
+  job.out_start = off;
+  job.out_end = off + w;
+  job.loff = Ll;
+  job.piece0 = 2 * d;
+  job.n_pieces = np;
+  job.F = cfg.F;
+  job.out_ring = ring;
+  return job;
+}
+
+struct SendRingsParam {
+  uint32_t n_rings;
+  RingDesc r[kMaxRings];
+  uint64_t off[kMaxRings];
+  const uint64_t* doorbell;  // if set, send offsets are doorbell[2 * n_rings + r]
+};
+
+// Block-wide exclusive sum (blockDim.x threads, <= 1024); returns the block total through *tot.
+__device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_sums, uint64_t* tot) {
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  uint64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
+  }
+  __syncthreads();
+  if (lane == 31) warp_sums[w] = x;
+  __syncthreads();
+  uint64_t base = 0, all = 0;
+  for (uint32_t i = 0; i < nw; ++i) {
+    if (i < w) base += warp_sums[i];
+    all += warp_sums[i];
+  }
+  *tot = all;
+  return base + x - v;
+}
+
+// Small batches (<= kSmallServe records): statuses, reply offsets, decode and encode jobs, their tile
+// prefix and the mover cursors, by one block of kSmallServe threads (thread d owns record d).
+// warp_sums (32) and ring_first_pre (kMaxRings) are the block's shared scratch.  Used by the
+// single-block planning kernel and by the persistent server.
+__device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
+                                 uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
+                                 uint64_t* ring_first_pre) {
+  const uint32_t total = *ix.total;
+  const uint32_t d = threadIdx.x;
+  for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
+  int st = CRK_OK;
+  int32_t err = -1;
+  uint64_t Ll = 0, w = 0;
+  Job dec{};
+  uint32_t ring = 0, first = 0, end = 0;
+  if (d < total) {
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
+    w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
+    ring = ix.p_ring[d];
+    first = ix.rec_prefix[ring];
+    end = ix.rec_prefix[ring + 1];
+  }
+  uint64_t tot;
+  const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets
+  if (d < total && d == first) ring_first_pre[ring] = pre;
+  __syncthreads();
+  Job enc{};
+  if (d < total) {
+    const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre - ring_first_pre[ring]);
+    ix.s_status[d] = st;
+    ix.s_reply_err[d] = err;
+    ix.s_reply_wire[d] = w;
+    ix.s_reply_off[d] = off;
+    enc = serve_reply_job(ix, cfg, sc, d, ring, err, off, w);
+    sc.jobs[d] = dec;
+    sc.jobs[total + d] = enc;
+    if (d + 1 == end) ix.res[ring].reply_bytes = pre + w - ring_first_pre[ring];
+  }
+  // mover plan: tiles per job (decode jobs [0, total), encode jobs [total, 2 total)) and their prefix
+  auto tiles_of = [&](const Job& j) -> uint64_t {
+    if (j.type == JOB_NONE || j.out_end <= j.out_start) return 0;
+    return ((j.out_end - 1) >> cfg.tile_shift) - (j.out_start >> cfg.tile_shift) + 1;
+  };
+  const uint64_t td = d < total ? tiles_of(dec) : 0, te = d < total ? tiles_of(enc) : 0;
+  uint64_t tot_d, tot_e;
+  const uint64_t pd = block_excl_sum(td, warp_sums, &tot_d);
+  const uint64_t pe = block_excl_sum(te, warp_sums, &tot_e);
+  if (d < total) {
+    sc.scan_tmp[d] = pd;
+    sc.scan_tmp[total + d] = tot_d + pe;
+  }
+  if (d == 0) {
+    sc.scan_tmp[sc.max_jobs + 1] = tot_d + tot_e;
+    sc.counters[0] = 0;
+    sc.counters[2] = 0;
+    sc.counters[1] = 2 * total;
+    sc.counters[4] = total;
+  }
+}
+
+}  // namespace
+}  // namespace crk

@@ -1,0 +1,238 @@
+// Persistent server (include/crk.h crk_server_*): one resident CTA polls a
+// doorbell and runs each published step with the same device functions as the launched pipeline --
+// scan_ring_cta (K1), parse_record (K3), plan_small_block (serve planning), the generic movers (K4-K7) --
+// so a small call costs a few dependent memory round trips instead of five kernel launches.
+//
+// Rings change under a running kernel, so this translation unit reads them with coherent loads
+// (CRK_COHERENT_LOADS: ld.global.cg instead of the read-only path), and every phase boundary
+// invalidates the SM's L1 (__threadfence) so loads see the previous phase's L2 atomics and stores.
+#define CRK_COHERENT_LOADS 1
+#include "k_move.cuh"
+#include "k_parse.cuh"
+#include "k_plan.cuh"
+#include "k_scan.cuh"
+
+namespace crk {
+
+namespace {
+
+constexpr uint32_t kServerThreads = kSmallServe;  // plan_small_block: thread d owns record d
+constexpr uint32_t kServerWarps = kServerThreads / 32;
+
+struct ServerParams {
+  IndexDev ix;
+  ConfigDev cfg;
+  Scratch sc;
+  const SchemaTable* schemas;
+  crk_server_bell* bell;
+  uint32_t n_rings;
+  RingDesc rings[kMaxRings];   // base / mask; cursors come from the bell
+  RingDesc send[kMaxRings];
+  uint64_t region_base, region_bytes;
+};
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const volatile uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(volatile uint64_t* p, uint64_t v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Phase boundary: the block's writes are visible to the block and the SM's L1 holds nothing older
+// than L2 (atomics of the previous phase happened there).
+__device__ __forceinline__ void phase_sync() {
+  __syncthreads();
+  if (threadIdx.x == 0) __threadfence();
+  __syncthreads();
+}
+
+// Moves output tile t (kTileShift-aligned in output space, like the mover's tiles) of job J with team T
+// (generic paths of k_move.cuh).
+constexpr uint32_t kTileShift = 13;  // 8 KiB tiles, dealt to warps round-robin
+__device__ __forceinline__ uint64_t job_tiles(const Job& J) {
+  if (J.type == JOB_NONE || J.out_end <= J.out_start) return 0;
+  return ((J.out_end - 1) >> kTileShift) - (J.out_start >> kTileShift) + 1;
+}
+__device__ __forceinline__ void move_tile(const Team& T, const ServerParams& P, const Job& J, uint64_t t) {
+  const uint64_t A = J.out_start >> kTileShift;
+  const uint64_t a = max(J.out_start, (A + t) << kTileShift), b = min(J.out_end, (A + t + 1) << kTileShift);
+  if (J.type == JOB_DEC) {
+    DecCtx c;
+    dec_ctx_init(c, P.ix, J);
+    dec_tile_generic(T, c, a, b, 0);
+  } else if (J.type == JOB_ENC) {
+    EncCtx c;
+    enc_ctx_init(c, P.sc, J, P.sc.out_rings[J.out_ring], P.sc.pieces + J.piece0);
+    enc_tile_generic(T, c, a - J.out_start, b - J.out_start);
+  }
+}
+
+__global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams P) {
+  __shared__ ScanState S;
+  __shared__ SchemaTable sch;
+  __shared__ __align__(16) uint8_t heads[kServerWarps][kHead];
+  __shared__ SendRingsParam send;
+  __shared__ uint64_t warp_sums[32];
+  __shared__ uint64_t ring_first_pre[kMaxRings];
+  __shared__ uint32_t prefix[kMaxRings + 1];
+  __shared__ uint64_t win_head[kMaxRings], win_tail[kMaxRings];
+  __shared__ uint64_t seq_s;
+  __shared__ uint32_t stop_s, bad_s;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  crk_server_bell* B = P.bell;
+  const IndexDev& ix = P.ix;
+  uint64_t seen = B->done_seq;
+  for (;;) {
+    // ---- wait for a new step
+    if (threadIdx.x == 0) {
+      uint64_t s;
+      while ((s = ld_acquire_sys(&B->seq)) == seen) __nanosleep(64);
+      seq_s = s;
+      stop_s = B->stop != 0;
+      bad_s = 0;
+      B->t_begin_ns = gtimer();
+    }
+    phase_sync();
+    if (stop_s) break;
+    TL_END(P.cfg, 6);
+    seen = seq_s;
+    // ---- step setup: schemas (re-read: registrations may follow the start), send cursors, xid table
+    for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
+      reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
+    // the step's cursors: one read of the bell per value, all in flight at once (a host bell is read
+    // over PCIe; every later use is from shared memory)
+    for (uint32_t r = threadIdx.x; r < P.n_rings; r += blockDim.x) {
+      send.r[r] = P.send[r];
+      send.off[r] = *(volatile uint64_t*)&B->send_off[r];
+      win_head[r] = *(volatile uint64_t*)&B->head[r];
+      win_tail[r] = *(volatile uint64_t*)&B->tail[r];
+    }
+    if (threadIdx.x == 0) {
+      send.n_rings = P.n_rings;
+      send.doorbell = nullptr;
+    }
+    for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
+    phase_sync();
+    TL_END(P.cfg, 0);
+    // ---- K1: each ring in turn by the whole CTA
+    SCAN_TRACE(threadIdx.x == 0, 5, 0);
+    for (uint32_t r = 0; r < P.n_rings; ++r) {
+      RingDesc R = P.rings[r];
+      R.head = win_head[r];
+      R.tail = win_tail[r];
+      const bool bad = R.tail < R.head || R.tail - R.head > R.mask + 1;
+      if (bad) {
+        R.tail = R.head;
+        if (threadIdx.x == 0) bad_s = 1;
+      }
+      scan_ring_cta(ix, R, bad, r, P.cfg, S);
+    }
+    if (threadIdx.x == 0) dense_numbering(ix, P.n_rings);
+    phase_sync();
+    TL_END(P.cfg, 1);
+#ifdef CRK_TIMELINE_SCAN2  // diagnostic: the scan again, with its code and data now cached
+    for (uint32_t r = 0; r < P.n_rings; ++r) {
+      RingDesc R = P.rings[r];
+      R.head = win_head[r];
+      R.tail = win_tail[r];
+      const bool bad = R.tail < R.head || R.tail - R.head > R.mask + 1;
+      if (bad) R.tail = R.head;
+      scan_ring_cta(ix, R, bad, r, P.cfg, S);
+    }
+    if (threadIdx.x == 0) dense_numbering(ix, P.n_rings);
+    phase_sync();
+    TL_END(P.cfg, 7);
+#endif
+    // ---- K3: one warp per record
+    for (uint32_t i = threadIdx.x; i <= P.n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
+    __syncthreads();
+    const uint32_t total = prefix[P.n_rings];
+    for (uint32_t d = warp; d < total; d += kServerWarps) {
+      uint32_t lo = 0, hi = P.n_rings;  // ring of dense record d
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (prefix[mid] <= d) lo = mid; else hi = mid;
+      }
+      parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane);
+      __syncwarp();
+    }
+    phase_sync();
+    TL_END(P.cfg, 2);
+    // ---- serve planning (statuses, reply offsets, jobs)
+    plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre);
+    phase_sync();
+    TL_END(P.cfg, 3);
+    // ---- movers: every job cut into 8 KiB output tiles, tiles dealt to the warps round-robin
+    const uint32_t n_jobs = 2 * total;
+    const Team TW{lane, 32, 0, 1};
+    uint64_t first = 0;  // global number of the job's first tile
+    for (uint32_t j = 0; j < n_jobs; ++j) {
+      const Job J = P.sc.jobs[j];
+      const uint64_t nt = job_tiles(J);
+      for (uint64_t t = (warp + kServerWarps - first % kServerWarps) % kServerWarps; t < nt; t += kServerWarps)
+        move_tile(TW, P, J, t);
+      first += nt;
+    }
+    phase_sync();
+    TL_END(P.cfg, 4);
+    // ---- publish: results into the bell, then done_seq
+    for (uint32_t r = threadIdx.x; r < P.n_rings; r += blockDim.x) B->res[r] = ix.res[r];
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      B->status = bad_s ? CRK_E_ARG : CRK_OK;
+      B->t_end_ns = gtimer();
+      __threadfence_system();
+      st_release_sys(&B->done_seq, seen);
+    }
+    TL_END(P.cfg, 5);
+  }
+}
+
+}  // namespace
+
+uint32_t server_threads() { return kServerThreads; }
+
+#ifdef CRK_SCAN_TRACE
+// Diagnostic build only: the server translation unit's copy of the scan clock trace (k_scan.cuh).
+extern "C" int crk_debug_server_scan_trace(unsigned long long* out, uint32_t* counts, int reset) {
+  if (out && cudaMemcpyFromSymbol(out, g_scan_trace, sizeof(g_scan_trace)) != cudaSuccess) return -100;
+  if (counts && cudaMemcpyFromSymbol(counts, g_scan_trace_n, sizeof(g_scan_trace_n)) != cudaSuccess) return -100;
+  if (reset) {
+    static const uint32_t zero[kTraceRings] = {};
+    if (cudaMemcpyToSymbol(g_scan_trace_n, zero, sizeof(zero)) != cudaSuccess) return -100;
+  }
+  return 0;
+}
+#endif
+
+cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SchemaTable* schemas,
+                          crk_server_bell* bell, uint32_t n_rings, const crk_ring* rings, const crk_ring* send_rings,
+                          uint64_t region_base, uint64_t region_bytes, cudaStream_t s) {
+  ServerParams P;
+  memset(&P, 0, sizeof(P));
+  P.ix = ix;
+  P.cfg = cfg;
+  P.sc = sc;
+  P.schemas = schemas;
+  P.bell = bell;
+  P.n_rings = n_rings;
+  for (uint32_t r = 0; r < n_rings; ++r) {
+    P.rings[r].base = rings[r].base;
+    P.rings[r].mask = rings[r].cap - 1;
+    P.send[r].base = send_rings[r].base;
+    P.send[r].mask = send_rings[r].cap - 1;
+  }
+  P.region_base = region_base;
+  P.region_bytes = region_bytes;
+  server_kernel<<<1, kServerThreads, 0, s>>>(P);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace crk

@@ -1,0 +1,131 @@
+"""GPU parity of the persistent server (crk_server_*) against the oracle's serve
+step (oracle/oracle.c or_serve), bit-exact: several steps through one resident kernel, each appending a
+batch of calls (HtoD / DtoH memcpys, control calls, every error kind serve reports) to every ring.
+
+While a server runs, nothing here may synchronise the whole device (its kernel never ends until stop):
+results come from the doorbell block, memory is read with stream-ordered copies."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_sc_eilingkkflm23_b200 import crk, gen
+from tests.gpu_util import ctx_for, d2h_call, h2d_call, ocfg
+
+pytestmark = [pytest.mark.gpu, pytest.mark.timeout(300)]
+
+if not torch.cuda.is_available():
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+
+def ring_bytes(ring: crk.Ring) -> np.ndarray:
+    hv = ring.host_view()
+    if hv is not None:
+        return hv.copy()
+    return ring.tensor().cpu().numpy()  # stream-ordered copy, no device-wide synchronisation
+
+
+def batch(g, step: int, ring: int, base: int, region_bytes: int, host_region: np.ndarray, cfg, F: int):
+    """Wire bytes of one step's calls on one ring: small HtoD / DtoH memcpys, a control call of a
+    registered proc, and (some steps) error records."""
+    wire = b""
+    for i in range(int(g.integers(1, 6))):
+        xid = (step << 20) | (ring << 12) | i
+        kind = int(g.integers(0, 3))
+        if kind == 0:  # destinations: a private slot of the region's lower half (reading R18: disjoint)
+            size = int(g.integers(0, 20000))
+            off = (ring * 6 + i) * 20480 + int(g.integers(0, 16))
+            data = gen.random_bytes((step * 131 + ring * 17 + i) & 0xFFFFFFFF, size)
+            c = h2d_call(xid, data, base + off)
+        elif kind == 1:  # sources: the upper half, never written
+            size = int(g.integers(0, 40000))
+            off = region_bytes // 2 + int(g.integers(0, region_bytes // 2 - size))
+            c = d2h_call(xid, base + off, size)
+        else:
+            c = (xid, 33, [(O.K_U32, int(g.integers(0, 1 << 32))), (O.K_I32_VAR, gen.random_elems(g, np.int32, 17))])
+        wire += O.encode_call(*c, cfg, F=F)
+    if step % 3 == 2:  # a duplicate xid, a pointer outside the region, a wrong program version
+        wire += O.encode_call(*h2d_call((step << 20) | (ring << 12), np.zeros(8, np.uint8), base), cfg, F=F)
+        wire += O.encode_call(*d2h_call(0xE0000000 + step, base + region_bytes, 16), cfg, F=F)
+        wire += O.frame(O.call_header(0xE2000000 + step, gen.PROG, 3, 1), 100)
+    return wire
+
+
+@pytest.mark.parametrize("host", [False, True])
+def test_server_steps_match_oracle(host):
+    F = 4096
+    cfg = ocfg(F=F, user={33: [O.K_U32, O.K_I32_VAR]})
+    ctx = ctx_for(cfg)
+    n_rings, cap, scap = 3, 1 << 18, 1 << 18
+    region_bytes = 1 << 20
+    region = torch.zeros(region_bytes, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    g = gen.rng(0x5E)
+    host_region = gen.random_bytes(0x5E5E, region_bytes).copy()
+    region.copy_(torch.from_numpy(host_region))
+    rings = [crk.Ring.host(cap) if host else crk.Ring.device(cap) for _ in range(n_rings)]
+    sends = [crk.Ring.host(scap) if host else crk.Ring.device(scap) for _ in range(n_rings)]
+    idx = ctx.index(n_rings, 1 << 12, 3 * 64)
+    torch.cuda.synchronize()
+    srv = crk.Server(idx, rings, sends, base, region_bytes)
+    try:
+        tails = [cap - 5000 + 97 * r for r in range(n_rings)]  # windows cross the wrap on later steps
+        send_offs = [scap - 3000 + 11 * r for r in range(n_rings)]
+        for step in range(8):
+            heads = list(tails)
+            for r in range(n_rings):
+                w = batch(g, step, r, base, region_bytes, host_region, cfg, F)
+                rings[r].write(tails[r], w)
+                tails[r] += len(w)
+            if step == 5:  # a truncated window: the last record is incomplete
+                tails[1] -= 3
+            before = [ring_bytes(r) for r in rings]
+            out = srv.step(list(zip(heads, tails)), send_offs)
+            want = O.serve([(b, h, t) for b, h, t in zip(before, heads, tails)], cfg, host_region, base,
+                           [scap] * n_rings, send_offs, max_frags_per_ring=(1 << 12) // n_rings,
+                           max_records_per_ring=64)
+            assert out["status"] == O.OK
+            for r in range(n_rings):
+                res = out["results"][r]
+                assert res["status"] == want["scan_status"][r], (step, r, res)
+                assert res["consumed"] == want["consumed"][r], (step, r)
+                assert res["reply_bytes"] == want["reply_bytes"][r], (step, r)
+                n = want["reply_bytes"][r]
+                got = sends[r].read(send_offs[r], n)
+                exp = bytes(np.roll(want["send"][r], -(send_offs[r] % scap))[:n])
+                assert got == exp, (step, r)
+            assert np.array_equal(region.cpu().numpy(), host_region), step
+            for r in range(n_rings):
+                tails[r] = want["consumed"][r] if step == 5 and r == 1 else tails[r]
+                send_offs[r] += want["reply_bytes"][r]
+    finally:
+        srv.stop()
+
+
+def test_server_rejects_bad_window_and_stops():
+    cfg = ocfg()
+    ctx = ctx_for(cfg)
+    region = torch.zeros(1 << 16, dtype=torch.uint8, device="cuda")
+    ring, send = crk.Ring.device(1 << 12), crk.Ring.device(1 << 12)
+    idx = ctx.index(1, 64, 16)
+    torch.cuda.synchronize()
+    srv = crk.Server(idx, [ring], [send], region.data_ptr(), region.numel())
+    try:
+        out = srv.step([(100, 50)], [0])  # tail < head
+        assert out["status"] == crk.E_ARG and out["results"][0]["n_records"] == 0
+        w = O.encode_call(*h2d_call(9, np.arange(100, dtype=np.uint8), region.data_ptr() + 8), cfg)
+        ring.write(0, w)
+        out = srv.step([(0, len(w))], [0])
+        assert out["status"] == crk.OK and out["results"][0]["status"] == crk.OK
+        assert out["results"][0]["consumed"] == len(w) and out["device_ns"] > 0
+        assert np.array_equal(region[8:108].cpu().numpy(), np.arange(100, dtype=np.uint8))
+    finally:
+        srv.stop()
+    torch.cuda.synchronize()  # the kernel has exited
+
+
+def test_server_capacity_limits():
+    ctx = ctx_for(ocfg())
+    ring, send = crk.Ring.device(1 << 12), crk.Ring.device(1 << 12)
+    with pytest.raises(crk.CrkError):
+        crk.Server(ctx.index(1, 1 << 12, 2048), [ring], [send], 0, 0)  # > 1024 records

@@ -144,6 +144,58 @@ def serve_latency(ctx):
     return {"serve_launches_us": round(us_launch, 2), "serve_graph_us": round(us_graph, 2), "ok": ok}
 
 
+def server_latency(ctx, reps=2000):
+    """Persistent server (crk_server): one 4 KiB HtoD CALL per step, published through a mapped doorbell;
+    host round trip (write cursors, bump seq, spin on done_seq) and the device's service time per step.
+    Then the C2 matrixMul batch (A, B HtoD; C DtoH) as one step."""
+    import time
+    region = torch.zeros(4 * MiB, dtype=torch.uint8, device=dev)
+    base = region.data_ptr()
+    data = torch.from_numpy(gen.random_bytes(0xC1, 4096)).to(dev)
+    ring = crk.Ring.device(1 << 14)
+    w = ctx.encode_call(7, gen.PROC_H2D, [(crk.K_U64, base + 4096), (crk.K_OPAQUE_VAR, data), (crk.K_U64, 4096)],
+                        ring, 0)
+    send = crk.Ring.device(1 << 21)
+    idx = ctx.index(1, 64, 16)
+    # the C2 matrixMul batch, encoded before any server owns the context
+    A, B, Cm = gen.c2_matrices()
+    a, b = torch.from_numpy(A.view(np.uint8)).to(dev), torch.from_numpy(B.view(np.uint8)).to(dev)
+    ring2 = crk.Ring.device(1 << 21)
+    cur = ctx.encode_call(1, gen.PROC_H2D, [(crk.K_U64, base), (crk.K_OPAQUE_VAR, a), (crk.K_U64, a.numel())],
+                          ring2, 0)
+    cur += ctx.encode_call(2, gen.PROC_H2D, [(crk.K_U64, base + MiB), (crk.K_OPAQUE_VAR, b), (crk.K_U64, b.numel())],
+                           ring2, cur)
+    cur += ctx.encode_call(3, gen.PROC_D2H, [(crk.K_U64, base + 3 * MiB), (crk.K_U64, Cm.nbytes)], ring2, cur)
+    torch.cuda.synchronize()
+    srv = crk.Server(idx, [ring], [send], base, region.numel())
+    try:
+        rt, dv = [], []
+        for i in range(reps):
+            t0 = time.perf_counter_ns()
+            out = srv.step([(0, w)], [0])
+            rt.append(time.perf_counter_ns() - t0)
+            dv.append(out["device_ns"])
+        ok = out["results"][0]["status"] == 0 and out["results"][0]["reply_bytes"] == 32
+    finally:
+        srv.stop()
+    ok &= bool(torch.equal(region[4096:8192], data))  # device allocations wait for a running server
+    idx2 = ctx.index(1, 1024, 16)
+    srv2 = crk.Server(idx2, [ring2], [send], base, region.numel())
+    try:
+        c2dv = []
+        for i in range(50):
+            out2 = srv2.step([(0, cur)], [0])
+            c2dv.append(out2["device_ns"])
+        ok2 = out2["results"][0]["status"] == 0
+    finally:
+        srv2.stop()
+    ok2 &= bool(torch.equal(region[:a.numel()], a))
+    return {"one_record_roundtrip_us_median": round(float(np.median(rt)) / 1e3, 2),
+            "one_record_device_us_median": round(float(np.median(dv)) / 1e3, 2),
+            "one_record_roundtrip_us_p99": round(float(np.percentile(rt, 99)) / 1e3, 2), "ok": bool(ok),
+            "c2_batch_device_us_median": round(float(np.median(c2dv)) / 1e3, 2), "c2_ok": bool(ok2)}
+
+
 def c2(ctx):
     A, B, C = gen.c2_matrices()
     region = torch.zeros(4 * MiB, dtype=torch.uint8, device=dev)
@@ -305,6 +357,7 @@ def main():
         "C1": lambda: c1(crk.Context(0)),
         "C1_serve_one_record": lambda: serve_latency(crk.Context(0)),
         "C2_matrixMul": lambda: c2(crk.Context(0)),
+        "NEXT3_server": lambda: server_latency(crk.Context(0)),
         "C3_sweep": lambda: c3(crk.Context(0)),
         "C4_typed_regular": lambda: c4(crk.Context(0), False),
         "C4_typed_irregular": lambda: c4(crk.Context(0), True),
