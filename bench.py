@@ -113,8 +113,9 @@ class ClockSampler:
 
 # ------------------------------------------------------------------ CPU baseline (oracle)
 
-def oracle_sample(n_streams: int, payload_mib: int, rank: int = 0):
-    """Oracle-encoded rings for the first streams of endpoint `rank` (a bounded sample of the workload)."""
+def oracle_sample(stream_ids, payload_mib: int, rank: int = 0):
+    """Oracle-encoded rings for streams `stream_ids` of endpoint `rank` (a bounded sample of the workload),
+    with a host region of their own (their destinations / sources rebased to its start)."""
     import numpy as np
     import oracle as O
     from paper_conf_sc_eilingkkflm23_b200 import gen
@@ -122,27 +123,31 @@ def oracle_sample(n_streams: int, payload_mib: int, rank: int = 0):
                                  h2d_budget=payload_mib * MiB - payload_mib * MiB // 16)
     cfg = O.Config(prog=gen.PROG, vers=gen.VERS, proc_h2d=gen.PROC_H2D, proc_d2h=gen.PROC_D2H, frag_payload=65536)
     base = 0x7F0000000000
-    sample = streams[:n_streams]
-    top = max(r.region_off + r.size for s in sample for r in s.records)
+    sample = [streams[i] for i in stream_ids]
+    lo = min(r.region_off for s in sample for r in s.records) & ~255
+    top = max(r.region_off + r.size for s in sample for r in s.records) - lo
     region = np.zeros(top + 256, np.uint8)
-    rings, payload = [], 0
+    rings, send_caps, payload = [], [], 0
     for s in sample:
-        wires = []
+        wires, reply = [], 0
         for r in s.records:
             d = gen.random_bytes(r.seed & 0xFFFFFFFF, r.size)
             payload += r.size
+            off = r.region_off - lo
             if r.kind == gen.PROC_H2D:
-                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + r.region_off), (O.K_OPAQUE_VAR, d),
+                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + off), (O.K_OPAQUE_VAR, d),
                                                            (O.K_U64, r.size)], cfg))
+                reply += 64
             else:
-                region[r.region_off:r.region_off + r.size] = d
-                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + r.region_off), (O.K_U64, r.size)], cfg))
+                region[off:off + r.size] = d
+                wires.append(O.encode_call(r.xid, r.kind, [(O.K_U64, base + off), (O.K_U64, r.size)], cfg))
+                reply += r.size + 64 + 4 * (r.size // 65536 + 1)
         w = b"".join(wires)
         cap = 1 << max(8, len(w).bit_length())
         ring = np.zeros(cap, np.uint8)
         ring[:len(w)] = np.frombuffer(w, np.uint8)
         rings.append((ring, 0, len(w)))
-    send_caps = [1 << 28] * len(rings)
+        send_caps.append(1 << max(8, reply.bit_length()))
 
     def step():
         out = O.serve(rings, cfg, region, base, send_caps, [0] * len(rings), max_frags_per_ring=1 << 16,
@@ -150,12 +155,10 @@ def oracle_sample(n_streams: int, payload_mib: int, rank: int = 0):
         assert all(s == O.OK for s in out["scan_status"])
         return out
 
-    return step, payload
+    return step, payload, region
 
 
-def cpu_baseline(args, seconds: float):
-    n_streams = 2
-    step, payload = oracle_sample(n_streams, args.payload_mib)
+def _timed_loop(step, seconds: float):
     step()  # warm (page-in)
     t0 = time.perf_counter()
     reps = 0
@@ -164,10 +167,73 @@ def cpu_baseline(args, seconds: float):
         reps += 1
         el = time.perf_counter() - t0
         if el >= seconds:
-            break
-    return {"value": round(payload * reps / el / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"oracle or_serve (plain C, 1 thread) over streams 0-{n_streams - 1} of endpoint 0 "
-                      f"({payload / MiB:.0f} MiB payload) x{reps} reps, {el:.1f} s"}
+            return reps, el
+
+
+def cpu_baseline(args, seconds: float):
+    """The oracle as it stands, on this box's host cores (SURVEY.md §8(d) "Oracle (CPU baseline)"):
+    (i) one thread -- the analogue of Cricket's single-core RPC path (P:238) -- is `value`;
+    (ii) one thread per core over independent client streams (ctypes releases the GIL in or_serve);
+    (iii) Cricket-style: decode into a pageable host buffer, then cudaMemcpy it to the device."""
+    import torch
+    n_streams = 2
+    step, payload, _ = oracle_sample(list(range(n_streams)), args.payload_mib)
+    reps, el = _timed_loop(step, seconds)
+    out = {"value": round(payload * reps / el / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+           "sample": f"oracle or_serve (plain C, 1 thread) over streams 0-{n_streams - 1} of endpoint 0 "
+                     f"({payload / MiB:.0f} MiB payload) x{reps} reps, {el:.1f} s"}
+    try:
+        import platform
+        out["cpu_model"] = next((l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo")
+                                 if l.startswith("model name")), platform.processor())
+    except OSError:
+        pass
+    # (ii) one thread per core, each serving its own stream (own ring, region and send ring)
+    nthr = max(1, min(len(os.sched_getaffinity(0)), 16))  # the cores bench.py is bound to (GPU NUMA node)
+    samples = [oracle_sample([t], args.payload_mib) for t in range(nthr)]
+    for st, _, _ in samples:
+        st()
+    done = [0] * nthr
+    stop_at = time.perf_counter() + seconds / 2
+
+    def worker(i):
+        while time.perf_counter() < stop_at:
+            samples[i][0]()
+            done[i] += 1
+
+    t0 = time.perf_counter()
+    ths = [threading.Thread(target=worker, args=(i,)) for i in range(nthr)]
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join()
+    el = time.perf_counter() - t0
+    moved = sum(done[i] * samples[i][1] for i in range(nthr))
+    out["threads"] = {"value": round(moved / el / 1e9, 4), "unit": "GB/s", "cores": nthr,
+                      "sample": f"{nthr} threads, thread t serves stream t of endpoint 0 alone "
+                                f"({args.payload_mib} MiB payload each), {sum(done)} stream-steps in {el:.1f} s"}
+    del samples
+    # (iii) Cricket-style: DtoH sources cudaMemcpy'd into the pageable host region, the oracle decodes and
+    # encodes there, then the region (HtoD destinations) is cudaMemcpy'd back to the device
+    if torch.cuda.is_available():
+        dev = torch.device("cuda", torch.cuda.current_device())
+        step3, payload3, region = oracle_sample(list(range(n_streams)), args.payload_mib)
+        host = torch.from_numpy(region)
+        d_region = host.to(dev)
+
+        def cricket_step():
+            host.copy_(d_region)   # pageable D2H
+            step3()
+            d_region.copy_(host)   # pageable H2D
+            torch.cuda.synchronize(dev)
+
+        reps, el = _timed_loop(cricket_step, seconds / 2)
+        out["cricket_style"] = {"value": round(payload3 * reps / el / 1e9, 4), "unit": "GB/s", "cores": 1,
+                                "sample": f"oracle or_serve into a pageable host buffer + cudaMemcpy of the "
+                                          f"{region.size / MiB:.0f} MiB region each way, streams 0-{n_streams - 1}, "
+                                          f"x{reps} reps, {el:.1f} s"}
+        del d_region
+    return out
 
 
 def run_reference(args):
@@ -176,7 +242,7 @@ def run_reference(args):
     if rank != 0:
         return
     n_streams = 2
-    step, payload = oracle_sample(n_streams, args.payload_mib)
+    step, payload, _ = oracle_sample(list(range(n_streams)), args.payload_mib)
     for _ in range(args.warmup):
         step()
     t0 = time.perf_counter()
@@ -225,6 +291,7 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
+    numa = parallel.bind_numa(local)  # before any pinned host allocation
     red_dev = "cpu" if shared_gpu else dev
     build.build()
 
@@ -335,23 +402,39 @@ def main():
             hslots[-1].res = crk.PinnedResults(args.streams)
         ep_h = hslots[0].ep
 
+        for s in hslots:  # inbound and outbound DMA get their own streams so the two directions never
+            s.in_stream, s.out_stream = torch.cuda.Stream(dev), torch.cuda.Stream(dev)  # wait on each other
+            s.ev_in, s.ev_served, s.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
+            s.ev_out.record(s.out_stream)
+            s.ev_served.record(s.stream)
+
         def run_staged(n_steps):
-            # copy-engine mode: DMA in -> serve from HBM -> results; the host finishes step k-1 (reply
-            # bytes known) by queueing its reply DMA while step k's inbound DMA runs: both directions busy
+            # copy-engine mode, per slot: inbound DMA (in_stream, after the slot's previous serve has read
+            # its device rings) -> serve from HBM (stream, after the previous reply DMA has drained the
+            # device send rings) -> reply DMA (out_stream, queued by the host once the reply sizes are
+            # known).  Inbound DMA of later batches never waits behind a reply DMA.
             pend = []
             for k in range(n_steps):
                 s = hslots[k % P]
-                workload.staged_in_and_serve(s.idx, s.ep, s.res, s.stream)
-                ev = torch.cuda.Event()
-                ev.record(s.stream)
-                pend.append((s, ev))
+                s.in_stream.wait_event(s.ev_served)
+                workload.staged_in(s.ep, s.in_stream)
+                s.ev_in.record(s.in_stream)
+                s.stream.wait_event(s.ev_in)
+                s.stream.wait_event(s.ev_out)
+                workload.staged_serve(s.idx, s.ep, s.res, s.stream)
+                s.ev_served.record(s.stream)
+                pend.append(s)
                 if len(pend) >= P:
-                    ps, pev = pend.pop(0)
-                    pev.synchronize()
-                    workload.staged_out(ps.ep, ps.res.rows(), ps.stream)
-            for ps, pev in pend:
-                pev.synchronize()
-                workload.staged_out(ps.ep, ps.res.rows(), ps.stream)
+                    ps = pend.pop(0)
+                    ps.ev_served.synchronize()
+                    ps.out_stream.wait_event(ps.ev_served)
+                    workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream)
+                    ps.ev_out.record(ps.out_stream)
+            for ps in pend:
+                ps.ev_served.synchronize()
+                ps.out_stream.wait_event(ps.ev_served)
+                workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream)
+                ps.ev_out.record(ps.out_stream)
             torch.cuda.synchronize()
 
         run_staged(max(2, min(args.warmup, 4)))
@@ -429,7 +512,7 @@ def main():
         "stage_share": stage_share,
         "payload_bytes_per_gpu": ep.payload, "wire_in_bytes_per_gpu": ep.wire_in,
         "reply_bytes_per_gpu": ep.reply_wire, "records_per_gpu": ep.n_records,
-        "gpu_launches": launches, "check": check,
+        "gpu_launches": launches, "check": check, "host_numa": numa,
         "clocks": clk.summary(),
         "e2e": e2e,
     }

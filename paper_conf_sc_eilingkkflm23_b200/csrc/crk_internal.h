@@ -97,7 +97,7 @@ struct Job {              // 64 bytes
 struct Scratch {          // ctx-owned device scratch
   Job* jobs;              // [max_jobs]
   Piece* pieces;          // [2 * max_jobs]
-  uint32_t* counters;     // [8]: 0 mover tile cursor, 1 n_jobs, 5 K2 block counter
+  uint32_t* counters;     // [8]: 0/2 mover decode/encode run cursors, 3/6 their single-tile tail cursors, 1 n_jobs, 4 queue split, 5 K2 block counter
   uint64_t* lens_pool;    // explicit framing: [2 * max_lens] (lens, then wire starts)
   uint32_t* lens32;       // [max_lens] staging for host-given fragment lengths
   unsigned long long* scan_state;  // decoupled look-back state for K2

@@ -264,8 +264,22 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           const uint32_t q = pref ^ tries;
           const uint64_t lo = q ? split : 0, hi = q ? total : split;
           if (lo < hi) {
-            const uint64_t t = lo + (uint64_t)kRun * atomicAdd(M.sc.counters + (q ? 2 : 0), 1u);
-            if (t < hi) { t0 = t; t1 = min(hi, t + kRun); }
+            // the queue's last ~2 tiles per CTA are claimed one at a time (second cursor) so the
+            // kernel's tail is one tile, not one run
+#ifdef CRK_MOVER_NO_TAIL
+            const uint64_t tail = 0;
+#else
+            const uint64_t tail = 2ull * gridDim.x;
+#endif
+            const uint64_t cut = (kRun > 1 && hi - lo > tail) ? lo + (hi - lo - tail) / kRun * kRun : lo;
+            uint64_t t = ~0ull;
+            if (cut > lo) t = lo + (uint64_t)kRun * atomicAdd(M.sc.counters + (q ? 2 : 0), 1u);
+            if (t < cut) {
+              t0 = t; t1 = min(cut, t + kRun);
+            } else {
+              t = cut + atomicAdd(M.sc.counters + (q ? 6 : 3), 1u);
+              if (t < hi) { t0 = t; t1 = t + 1; }
+            }
           }
         }
       }
@@ -494,8 +508,10 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
 __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, const uint32_t* n_jobs_dev) {
   const uint32_t n = *n_jobs_dev;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
-    sc.counters[0] = 0;  // decode-queue tile cursor
-    sc.counters[2] = 0;  // encode-queue tile cursor
+    sc.counters[0] = 0;  // decode-queue run cursor
+    sc.counters[2] = 0;  // encode-queue run cursor
+    sc.counters[3] = 0;  // decode-queue tail (single-tile) cursor
+    sc.counters[6] = 0;  // encode-queue tail cursor
   }
   for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
     const Job jb = sc.jobs[j];
@@ -516,6 +532,8 @@ __global__ void __launch_bounds__(256) plan_small_kernel(Scratch sc, ConfigDev c
   if (threadIdx.x == 0) {
     sc.counters[0] = 0;
     sc.counters[2] = 0;
+    sc.counters[3] = 0;
+    sc.counters[6] = 0;
   }
   constexpr uint32_t IPT = kSmallJobs / 256;
   uint64_t v[IPT], acc = 0;

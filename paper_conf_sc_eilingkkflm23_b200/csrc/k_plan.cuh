@@ -208,6 +208,8 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     sc.scan_tmp[sc.max_jobs + 1] = tot_d + tot_e;
     sc.counters[0] = 0;
     sc.counters[2] = 0;
+    sc.counters[3] = 0;
+    sc.counters[6] = 0;
     sc.counters[1] = 2 * total;
     sc.counters[4] = total;
   }

@@ -44,3 +44,35 @@ def aggregate(units_local: float, seconds_local: float, device="cpu") -> dict:
     t = max_over_ranks(seconds_local, device)
     u = sum_over_ranks(units_local, device)
     return {"seconds": t, "units": u, "per_second": u / t if t > 0 else 0.0}
+
+
+def _cpulist(text: str) -> set[int]:
+    cpus: set[int] = set()
+    for part in text.strip().split(","):
+        if not part:
+            continue
+        a, _, b = part.partition("-")
+        cpus.update(range(int(a), int(b or a) + 1))
+    return cpus
+
+
+def bind_numa(device: int, sysfs: str = "/sys") -> dict:
+    """Pins this process to the host cores of the NUMA node that `device` hangs off (SURVEY.md §8(d):
+    rings sit on the GPU's NUMA node, so pinned buffers allocated afterwards are first-touched there and
+    host-link traffic does not cross the socket interconnect).  Returns what was done, for the bench line."""
+    p = torch.cuda.get_device_properties(device)
+    bdf = f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+    try:
+        node = int(open(f"{sysfs}/bus/pci/devices/{bdf}/numa_node").read().strip())
+    except (OSError, ValueError):
+        return {"pci": bdf, "numa_node": None}
+    if node < 0:
+        return {"pci": bdf, "numa_node": node}
+    try:
+        cpus = _cpulist(open(f"{sysfs}/devices/system/node/node{node}/cpulist").read())
+        cpus &= os.sched_getaffinity(0)
+        if cpus:
+            os.sched_setaffinity(0, cpus)
+    except OSError:
+        cpus = set()
+    return {"pci": bdf, "numa_node": node, "cores": len(cpus)}

@@ -127,8 +127,18 @@ def serve_step(idx: crk.Index, ep: Endpoint, stream=None):
 def staged_in_and_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResults", stream):
     """Copy-engine mode, first half of a step: DMA each host receive window into its device ring,
     serve from HBM into the device send rings, and queue the per-ring results to pinned memory."""
+    staged_in(ep, stream)
+    staged_serve(idx, ep, results, stream)
+
+
+def staged_in(ep: Endpoint, stream):
+    """DMA each host receive window into its device ring."""
     for (hr, h, t), dr in zip(ep.rings, ep.dev_rings):
         crk.ring_copy(dr, hr, h, t, stream=stream)
+
+
+def staged_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResults", stream):
+    """Serve the staged device rings into the device send rings; queue the per-ring results."""
     idx.serve([(dr, h, t) for dr, (_, h, t) in zip(ep.dev_rings, ep.rings)], ep.dev_sends, ep.offs, ep.base,
               ep.region.numel(), stream=stream)
     idx.ring_results_async(results, stream=stream)
