@@ -100,6 +100,11 @@ typedef struct {
   uint32_t scan_threads;     /* K1 threads per ring, two predictor groups, 64..1024, multiple of 64 (default 256) */
   uint32_t mover_stages;     /* mover pipeline stages, 2..8 (default 3) */
   uint32_t mover_run;        /* tiles per mover claim, 1..64 (default 8) */
+  uint32_t mover_tail_tiles; /* per mover CTA, the last tiles of each queue claimed one at a time, 0..64 (default 2;
+                                shortens the kernel's tail when it runs alone) */
+  uint32_t mover_reserve_ctas; /* mover CTA slots left free (default 0), < half the grid: with several batches in
+                                  flight on other streams, the next batch's scan / parse / plan kernels and the
+                                  start of its mover find room on the GPU while this mover streams */
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;

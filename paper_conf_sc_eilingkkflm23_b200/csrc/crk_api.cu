@@ -236,6 +236,8 @@ void crk_config_init(crk_config* c) {
   c->scan_threads = 256;
   c->mover_stages = 3;
   c->mover_run = 8;
+  c->mover_tail_tiles = 2;
+  c->mover_reserve_ctas = 0;
 }
 
 int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
@@ -246,7 +248,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   if (cfg.frag_payload == 0 || cfg.frag_payload > 0x7fffffffu || !pow2(cfg.tile_bytes) || cfg.tile_bytes < 1024 ||
       cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 64 ||
       cfg.scan_threads > 1024 || (cfg.scan_threads & 63) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
-      cfg.mover_run < 1 || cfg.mover_run > 64)
+      cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64)
     return CRK_E_ARG;
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -261,6 +263,8 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   CK(cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device));
   int occ = cfg.ctas_per_sm ? (int)cfg.ctas_per_sm : mover_occupancy(cfg.tile_bytes, cfg.mover_stages);
   c->move_ctas = c->sms * (occ > 0 ? occ : 1);
+  if (2ull * cfg.mover_reserve_ctas >= (uint64_t)c->move_ctas) { delete c; return CRK_E_ARG; }
+  c->move_ctas -= (int)cfg.mover_reserve_ctas;
   ConfigDev& d = c->cd;
   d.F = cfg.frag_payload;
   d.strict = cfg.strict ? 1 : 0;
@@ -275,6 +279,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.tl = nullptr;
   d.stages = cfg.mover_stages;
   d.run = cfg.mover_run;
+  d.tail = cfg.mover_tail_tiles;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
   // scratch: one block

@@ -108,7 +108,7 @@ struct Scratch {          // ctx-owned device scratch
 
 struct ConfigDev {
   uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
-  uint32_t scan_threads, stages, run, pad_;
+  uint32_t scan_threads, stages, run, tail;  // tail: per-CTA single-tile claims at the end of each queue
   uint64_t max_record_bytes;
   unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };

@@ -28,7 +28,10 @@ namespace {
 
 constexpr int kMaxSeg = 8;      // segments a stage can describe
 constexpr int kMaxStages = 8;   // pipeline depth limit (runtime: cfg.stages)
-constexpr int kConsumerWarps = 8;
+#ifndef CRK_MOVER_CONSUMERS
+#define CRK_MOVER_CONSUMERS 8
+#endif
+constexpr int kConsumerWarps = CRK_MOVER_CONSUMERS;
 constexpr int kMoverThreads = 32 * (1 + kConsumerWarps);
 
 struct Seg {               // 32 bytes
@@ -264,13 +267,9 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           const uint32_t q = pref ^ tries;
           const uint64_t lo = q ? split : 0, hi = q ? total : split;
           if (lo < hi) {
-            // the queue's last ~2 tiles per CTA are claimed one at a time (second cursor) so the
-            // kernel's tail is one tile, not one run
-#ifdef CRK_MOVER_NO_TAIL
-            const uint64_t tail = 0;
-#else
-            const uint64_t tail = 2ull * gridDim.x;
-#endif
+            // the queue's last cfg.tail tiles per CTA are claimed one at a time (second cursor) so
+            // the kernel's tail is one tile, not one run
+            const uint64_t tail = (uint64_t)M.cfg.tail * gridDim.x;
             const uint64_t cut = (kRun > 1 && hi - lo > tail) ? lo + (hi - lo - tail) / kRun * kRun : lo;
             uint64_t t = ~0ull;
             if (cut > lo) t = lo + (uint64_t)kRun * atomicAdd(M.sc.counters + (q ? 2 : 0), 1u);

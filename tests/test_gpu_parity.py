@@ -560,10 +560,14 @@ def test_encode_replies_batch_matches_oracle(host, F):
     assert np.array_equal(offs.cpu().numpy(), np.cumsum([0] + [len(w) for w in want])[:-1] + start)
 
 
-@pytest.mark.parametrize("host", [False, True])
-def test_serve_matches_oracle(host):
+MOVER_CONFIGS = [{}, {"mover_tail_tiles": 0, "mover_reserve_ctas": 16},
+                 {"mover_tail_tiles": 64, "mover_run": 1, "tile_bytes": 4096}, {"mover_tail_tiles": 1, "mover_run": 64}]
+
+
+@pytest.mark.parametrize("host,mover", [(False, m) for m in range(len(MOVER_CONFIGS))] + [(True, 0)])
+def test_serve_matches_oracle(host, mover):
     cfg = ocfg(F=16384)
-    ctx = ctx_for(cfg)
+    ctx = ctx_for(cfg, **MOVER_CONFIGS[mover])
     streams, region_bytes = gen.c5_endpoint(0, n_streams=4, payload_per_stream=3 << 20, h2d_budget=2 << 20,
                                             lo=1, hi=1 << 20, misalign=True)
     region = torch.zeros(region_bytes + 64, dtype=torch.uint8, device="cuda")
@@ -693,6 +697,13 @@ def test_serve_cred_bodies_lenient_and_duplicates_match_oracle(strict):
     n = want["reply_bytes"][0]
     assert T["rings"][0]["reply_bytes"] == n
     assert send.read(40, n) == bytes(want["send"][0][40:40 + n])
+
+
+def test_ctx_rejects_bad_mover_config():
+    for kw in ({"mover_tail_tiles": 65}, {"mover_reserve_ctas": 10 ** 6}, {"mover_run": 0}):
+        with pytest.raises(crk.CrkError) as e:
+            crk.Context(0, **kw)
+        assert e.value.status == crk.E_ARG
 
 
 def test_serve_rejects_index_larger_than_job_scratch():
