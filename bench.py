@@ -42,7 +42,7 @@ def parse_args():
     p.add_argument("--impl", default="crk", choices=["crk", "reference"])
     p.add_argument("--streams", type=int, default=16)
     p.add_argument("--payload-mib", type=int, default=64, help="payload per stream")
-    p.add_argument("--e2e-steps", type=int, default=30)
+    p.add_argument("--e2e-steps", type=int, default=100)
     p.add_argument("--pipeline", type=int, default=3, help="batches in flight (server loop slots)")
     p.add_argument("--e2e-pipeline", type=int, default=3, help="batches in flight for the host-memory runs")
     p.add_argument("--no-e2e", action="store_true")
@@ -493,7 +493,8 @@ def main():
                           "h2d_bytes_per_step": ep_h.wire_in, "d2h_bytes_per_step": ep_h.reply_wire + res_bytes,
                           "ms_per_step": round(step_s * 1e3, 3), "mode": name,
                           "wire_gbs": round((ep_h.wire_in + ep_h.reply_wire) / step_s / 1e9, 3),
-                          "host_link": {**link, "bound_ms": round(t_link * 1e3, 3),
+                          "host_link": {**link, "pcie_gen5_x16_theoretical_gbs": 63.0,
+                                        "bound_ms": round(t_link * 1e3, 3),
                                         "frac": round(t_link / step_s, 4)},
                           "check": chk})
         modes.sort(key=lambda m: -m["value"] if m["check"]["ok"] else 0)
@@ -518,6 +519,7 @@ def main():
                                          "how": "mover algorithmic bytes per step / ms_per_step of the pipelined "
                                                 "timed region (a lower bound: the step also holds scan/parse/plan)"},
                      "mover_config": {k: ctx_kw.get(k) for k in ("mover_reserve_ctas", "mover_tail_tiles")}},
+        "wire_gbs": round(sum_over_ranks(ep.wire_in + ep.reply_wire) / (ms_max / 1e3) / 1e9, 2),
         "pipeline": P, "serial_ms_per_step": round(serial_ms, 4),
         "serial_value": round(payload_all / (serial_ms / 1e3) / 1e9, 2),
         "stages_ms_per_step": {k: round(v[0] / max(1, v[1]), 4) for k, v in prof.items()},

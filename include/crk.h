@@ -358,6 +358,8 @@ typedef struct {
   volatile int32_t status;     /* device -> host: CRK_OK, or CRK_E_ARG when the step had an invalid window */
   uint32_t pad_;
   volatile uint64_t t_begin_ns, t_end_ns; /* device %globaltimer at the step's start (seq seen) and end */
+  volatile uint64_t t_phase_ns[5];        /* device %globaltimer at the end of the step's setup, scan, parse,
+                                             planning and mover phases */
   crk_ring_result res[CRK_MAX_RINGS];     /* device -> host: per-ring results of the last step */
 } crk_server_bell;
 typedef struct crk_server crk_server;

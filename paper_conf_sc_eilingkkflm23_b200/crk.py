@@ -85,7 +85,7 @@ class ServerBell(C.Structure):
     _fields_ = [("seq", C.c_uint64), ("stop", C.c_uint64), ("head", C.c_uint64 * MAX_RINGS),
                 ("tail", C.c_uint64 * MAX_RINGS), ("send_off", C.c_uint64 * MAX_RINGS), ("done_seq", C.c_uint64),
                 ("status", C.c_int32), ("pad_", C.c_uint32), ("t_begin_ns", C.c_uint64), ("t_end_ns", C.c_uint64),
-                ("res", RingResult * MAX_RINGS)]
+                ("t_phase_ns", C.c_uint64 * 5), ("res", RingResult * MAX_RINGS)]
 
 
 _lib = None
@@ -612,7 +612,9 @@ class Server:
                 raise CrkError(E_CUDA, "crk_server step timed out")
         res = [dict(status=x.status, n_records=x.n_records, n_frags=x.n_frags, rec_base=x.rec_base,
                     consumed=x.consumed, reply_bytes=x.reply_bytes) for x in b.res[:self.n]]
-        return {"status": b.status, "results": res, "device_ns": b.t_end_ns - b.t_begin_ns}
+        ph = [b.t_phase_ns[i] - b.t_begin_ns for i in range(5)]
+        return {"status": b.status, "results": res, "device_ns": b.t_end_ns - b.t_begin_ns,
+                "phase_end_ns": dict(zip(("setup", "scan", "parse", "plan", "move"), ph))}
 
     def stop(self):
         if self.h:

@@ -9,7 +9,7 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
                                                                   ConfigDev cfg, uint32_t n_rings) {
   __shared__ SchemaTable sch;
   __shared__ uint32_t prefix[kMaxRings + 1];
-  __shared__ __align__(16) uint8_t heads[kParseWarps][kHead];
+  __shared__ __align__(16) uint8_t heads[kParseWarps][kHeadBuf];
   TL_BEGIN(cfg, TL_PARSE);
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(tab)[i];

@@ -27,17 +27,24 @@ __device__ __forceinline__ bool kind_is_var(uint32_t k) {
 }
 
 constexpr uint32_t kHead = 64;  // record head prefetched by the warp (CALL header + memcpy args)
+constexpr uint32_t kTail = 64;  // record tail prefetched with it (the arguments after a bulk opaque<>)
+constexpr uint32_t kHeadBuf = kHead + kTail;  // per-warp shared buffer
 
 struct Parser {
   LogicalRecord L;
   uint64_t o;
   const uint8_t* head;  // first `nhead` logical bytes, already in shared memory
   uint32_t nhead;
-  __device__ __forceinline__ uint8_t byte(uint64_t at) { return at < nhead ? head[at] : L.byte(at); }
+  const uint8_t* tail;  // logical bytes [tail_lo, L.len), already in shared memory (tail_lo == L.len: none)
+  uint64_t tail_lo;
+  __device__ __forceinline__ uint8_t byte(uint64_t at) {
+    return at < nhead ? head[at] : (at >= tail_lo && at < L.len) ? tail[at - tail_lo] : L.byte(at);
+  }
   __device__ int get_u32(uint32_t& v) {
     if (o + 4 > L.len) return CRK_E_TRUNCATED;
-    if (o + 4 <= nhead)
-      v = ((uint32_t)head[o] << 24) | ((uint32_t)head[o + 1] << 16) | ((uint32_t)head[o + 2] << 8) | head[o + 3];
+    const uint8_t* b = o + 4 <= nhead ? head + o : o >= tail_lo ? tail + (o - tail_lo) : nullptr;
+    if (b)
+      v = ((uint32_t)b[0] << 24) | ((uint32_t)b[1] << 16) | ((uint32_t)b[2] << 8) | b[3];
     else
       v = L.be32(o);
     o += 4;
@@ -63,20 +70,36 @@ struct Parser {
 };
 
 // Parse of dense record d (ring `ring`, index slot `slot`) by one warp: lane 0 runs the checks in the
-// oracle's order and writes the parsed-call tables and the xid table; head_buf is the warp's kHead-byte
+// oracle's order and writes the parsed-call tables and the xid table; head_buf is the warp's kHeadBuf-byte
 // shared buffer for the record head.  Used by K3 (one warp per record) and by the persistent server.
 __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const ConfigDev& cfg, uint32_t d,
                              uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane) {
   Parser P;
   P.L.init(ix, ix.rings[ring], slot);
   P.o = 0;
-  // the warp prefetches the record head from its first fragment in one round trip
+  // the warp prefetches, in one round trip, the record head from its first fragment and the record tail
+  // from its last fragment (when the tail lies inside it): a memcpy CALL's header, pointer, opaque length
+  // and, after the bulk data, its pad and size argument
   const uint64_t n0 = P.L.flen(0);
   const uint64_t nh = n0 < P.L.len ? n0 : P.L.len;
   P.nhead = nh < kHead ? (uint32_t)nh : kHead;
-  if (lane < P.nhead) head_buf[lane] = ring_byte(P.L.R, P.L.phys[0] + lane);
-  if (lane + 32 < P.nhead) head_buf[lane + 32] = ring_byte(P.L.R, P.L.phys[0] + lane + 32);
+  const uint32_t kl = P.L.nfrags - 1;
+  const uint64_t ls_last = P.L.lstart[kl], ph_last = P.L.phys[kl];
+  const uint64_t want = P.L.len > kTail ? P.L.len - kTail : 0;
+  const uint64_t tlo = want > P.nhead ? want : P.nhead;
+  P.tail_lo = (P.L.len > P.nhead && ls_last <= tlo) ? tlo : P.L.len;
+  const uint32_t ntail = (uint32_t)(P.L.len - P.tail_lo);
   P.head = head_buf;
+  P.tail = head_buf + kHead;
+  uint8_t b[4];
+  b[0] = lane < P.nhead ? ring_byte(P.L.R, P.L.phys[0] + lane) : 0;
+  b[1] = lane + 32 < P.nhead ? ring_byte(P.L.R, P.L.phys[0] + lane + 32) : 0;
+  b[2] = lane < ntail ? ring_byte(P.L.R, ph_last + (P.tail_lo - ls_last) + lane) : 0;
+  b[3] = lane + 32 < ntail ? ring_byte(P.L.R, ph_last + (P.tail_lo - ls_last) + lane + 32) : 0;
+  head_buf[lane] = b[0];
+  head_buf[lane + 32] = b[1];
+  head_buf[kHead + lane] = b[2];
+  head_buf[kHead + lane + 32] = b[3];
   __syncwarp();
   if (lane != 0) return;
   const bool strict = cfg.strict != 0;

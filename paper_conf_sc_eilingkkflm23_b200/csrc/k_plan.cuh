@@ -67,22 +67,25 @@ __device__ __forceinline__ void reply_words(Piece& p, uint32_t xid, int32_t err,
 // reply logical length, and the HtoD decode job.
 __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev& cfg, uint32_t d, uint64_t region_base,
                                              uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job) {
+  // every field the decision can need is loaded at once (one memory round trip), then the xid lookup
+  const uint64_t b = (uint64_t)d * kMaxItems;
   st = ix.p_status[d];
-  const uint32_t proc = ix.p_proc[d];
+  const uint32_t proc = ix.p_proc[d], xid = ix.p_xid[d];
+  const uint64_t v0 = ix.p_value[b], v1 = ix.p_value[b + 1], v2 = ix.p_value[b + 2];
+  const uint64_t c1 = ix.p_count[b + 1], o1 = ix.p_off[b + 1];
   err = -1;
   Ll = 0;
   job = Job{};
-  if (st == CRK_OK && xid_lookup(ix, ix.p_xid[d]) != d) st = CRK_E_XID;
-  const uint64_t b = (uint64_t)d * kMaxItems;
+  if (st == CRK_OK && xid_lookup(ix, xid) != d) st = CRK_E_XID;
   if (st == CRK_OK && proc == cfg.proc_h2d) {
-    const uint64_t ptr = ix.p_value[b], nb = ix.p_count[b + 1], size = ix.p_value[b + 2];
+    const uint64_t ptr = v0, nb = c1, size = v2;
     const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
     if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
     else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
-    else { err = 0; job = dec_job(ptr, m, ix.p_off[b + 1], d, 1); }
+    else { err = 0; job = dec_job(ptr, m, o1, d, 1); }
     Ll = 28;
   } else if (st == CRK_OK && proc == cfg.proc_d2h) {
-    const uint64_t ptr = ix.p_value[b], size = ix.p_value[b + 1];
+    const uint64_t ptr = v0, size = v1;
     if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
       st = CRK_E_PTR; err = 1; Ll = 28;
     } else {
@@ -169,11 +172,11 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   Job dec{};
   uint32_t ring = 0, first = 0, end = 0;
   if (d < total) {
-    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
-    w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
     ring = ix.p_ring[d];
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
     first = ix.rec_prefix[ring];
     end = ix.rec_prefix[ring + 1];
+    w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   }
   uint64_t tot;
   const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets

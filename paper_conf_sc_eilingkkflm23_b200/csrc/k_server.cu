@@ -4,8 +4,11 @@
 // so a small call costs a few dependent memory round trips instead of five kernel launches.
 //
 // Rings change under a running kernel, so this translation unit reads them with coherent loads
-// (CRK_COHERENT_LOADS: ld.global.cg instead of the read-only path), and every phase boundary
-// invalidates the SM's L1 (__threadfence) so loads see the previous phase's L2 atomics and stores.
+// (CRK_COHERENT_LOADS: ld.global.cg instead of the read-only path).  Each step starts with a system-scope
+// acquire of the doorbell (the host's ring writes, and device writes of other streams released before it,
+// are visible to every thread after the following barrier).  Phases hand data to each other only inside
+// this one CTA, so a block barrier orders them (CUDA memory model: __syncthreads makes the block's prior
+// global writes and atomics visible to the block); no device-wide fence per phase (≈1 µs each).
 #define CRK_COHERENT_LOADS 1
 #include "k_move.cuh"
 #include "k_parse.cuh"
@@ -44,24 +47,27 @@ __device__ __forceinline__ uint64_t gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-// Phase boundary: the block's writes are visible to the block and the SM's L1 holds nothing older
-// than L2 (atomics of the previous phase happened there).
+// Phase boundary: the block's global writes and atomics of the previous phase are visible to the block.
 __device__ __forceinline__ void phase_sync() {
   __syncthreads();
+#ifdef CRK_SERVER_PHASE_FENCE  // diagnostic: a device-wide fence per phase as well
   if (threadIdx.x == 0) __threadfence();
   __syncthreads();
+#endif
 }
 
-// Moves output tile t (kTileShift-aligned in output space, like the mover's tiles) of job J with team T
+// Moves output tile t (2^sh-aligned in output space, like the mover's tiles) of job J with team T
 // (generic paths of k_move.cuh).
-constexpr uint32_t kTileShift = 13;  // 8 KiB tiles, dealt to warps round-robin
-__device__ __forceinline__ uint64_t job_tiles(const Job& J) {
+// tiles dealt to the warps round-robin: 2 KiB (one chunk-loop pass per warp) when the step moves at most
+// ~4 mover tiles' worth of bytes, else 8 KiB
+constexpr uint32_t kJobCache = 32;   // jobs staged in shared memory at the start of the move phase
+__device__ __forceinline__ uint64_t job_tiles(const Job& J, uint32_t sh) {
   if (J.type == JOB_NONE || J.out_end <= J.out_start) return 0;
-  return ((J.out_end - 1) >> kTileShift) - (J.out_start >> kTileShift) + 1;
+  return ((J.out_end - 1) >> sh) - (J.out_start >> sh) + 1;
 }
-__device__ __forceinline__ void move_tile(const Team& T, const ServerParams& P, const Job& J, uint64_t t) {
-  const uint64_t A = J.out_start >> kTileShift;
-  const uint64_t a = max(J.out_start, (A + t) << kTileShift), b = min(J.out_end, (A + t + 1) << kTileShift);
+__device__ __forceinline__ void move_tile(const Team& T, const ServerParams& P, const Job& J, uint64_t t, uint32_t sh) {
+  const uint64_t A = J.out_start >> sh;
+  const uint64_t a = max(J.out_start, (A + t) << sh), b = min(J.out_end, (A + t + 1) << sh);
   if (J.type == JOB_DEC) {
     DecCtx c;
     dec_ctx_init(c, P.ix, J);
@@ -76,13 +82,14 @@ __device__ __forceinline__ void move_tile(const Team& T, const ServerParams& P, 
 __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams P) {
   __shared__ ScanState S;
   __shared__ SchemaTable sch;
-  __shared__ __align__(16) uint8_t heads[kServerWarps][kHead];
+  __shared__ __align__(16) uint8_t heads[kServerWarps][kHeadBuf];
   __shared__ SendRingsParam send;
   __shared__ uint64_t warp_sums[32];
   __shared__ uint64_t ring_first_pre[kMaxRings];
   __shared__ uint32_t prefix[kMaxRings + 1];
   __shared__ uint64_t win_head[kMaxRings], win_tail[kMaxRings];
   __shared__ uint64_t seq_s;
+  __shared__ Job jobs_s[kJobCache];
   __shared__ uint32_t stop_s, bad_s;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   crk_server_bell* B = P.bell;
@@ -120,6 +127,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
     phase_sync();
     TL_END(P.cfg, 0);
+    if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     // ---- K1: each ring in turn by the whole CTA
     SCAN_TRACE(threadIdx.x == 0, 5, 0);
     for (uint32_t r = 0; r < P.n_rings; ++r) {
@@ -136,6 +144,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) dense_numbering(ix, P.n_rings);
     phase_sync();
     TL_END(P.cfg, 1);
+    if (threadIdx.x == 0) B->t_phase_ns[1] = gtimer();
 #ifdef CRK_TIMELINE_SCAN2  // diagnostic: the scan again, with its code and data now cached
     for (uint32_t r = 0; r < P.n_rings; ++r) {
       RingDesc R = P.rings[r];
@@ -164,23 +173,33 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     }
     phase_sync();
     TL_END(P.cfg, 2);
+    if (threadIdx.x == 0) B->t_phase_ns[2] = gtimer();
     // ---- serve planning (statuses, reply offsets, jobs)
     plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre);
     phase_sync();
     TL_END(P.cfg, 3);
+    if (threadIdx.x == 0) B->t_phase_ns[3] = gtimer();
     // ---- movers: every job cut into 8 KiB output tiles, tiles dealt to the warps round-robin
     const uint32_t n_jobs = 2 * total;
     const Team TW{lane, 32, 0, 1};
+    {  // the first kJobCache jobs in one round trip (every warp walks every job's descriptor)
+      const uint32_t nc = n_jobs < kJobCache ? n_jobs : kJobCache;
+      for (uint32_t i = threadIdx.x; i < nc * (uint32_t)(sizeof(Job) / 4); i += blockDim.x)
+        reinterpret_cast<uint32_t*>(jobs_s)[i] = reinterpret_cast<const uint32_t*>(P.sc.jobs)[i];
+      __syncthreads();
+    }
+    const uint32_t sh = P.sc.scan_tmp[P.sc.max_jobs + 1] <= 4 ? 11u : 13u;  // plan's tile total (cfg tiles)
     uint64_t first = 0;  // global number of the job's first tile
     for (uint32_t j = 0; j < n_jobs; ++j) {
-      const Job J = P.sc.jobs[j];
-      const uint64_t nt = job_tiles(J);
+      const Job J = j < kJobCache ? jobs_s[j] : P.sc.jobs[j];
+      const uint64_t nt = job_tiles(J, sh);
       for (uint64_t t = (warp + kServerWarps - first % kServerWarps) % kServerWarps; t < nt; t += kServerWarps)
-        move_tile(TW, P, J, t);
+        move_tile(TW, P, J, t, sh);
       first += nt;
     }
     phase_sync();
     TL_END(P.cfg, 4);
+    if (threadIdx.x == 0) B->t_phase_ns[4] = gtimer();
     // ---- publish: results into the bell, then done_seq
     for (uint32_t r = threadIdx.x; r < P.n_rings; r += blockDim.x) B->res[r] = ix.res[r];
     __syncthreads();

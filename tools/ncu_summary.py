@@ -95,6 +95,30 @@ def main():
                       open(os.path.join(PROF, "mover_ncu.json"), "w"), indent=1)
         json.dump(d, open(os.path.join(PROF, f"{tag}_{name}_ncu.json"), "w"), indent=1)
         print(name, json.dumps(d)[:600])
+    host = os.path.join(OUT, "host_step_metrics.csv")
+    if os.path.exists(host):
+        d = host_step(host)
+        json.dump(d, open(os.path.join(PROF, f"{tag}_host_step_ncu.json"), "w"), indent=1)
+        print("host step", json.dumps(d)[:600])
+
+
+def host_step(path):
+    """tools/gpu_ncu_host.sh: per kernel of one zero-copy server step (rings in pinned host memory), the
+    PCIe bytes against the wire bytes the step must move (profile_step.py --host prints them)."""
+    out = {}
+    for r in csv.reader(open(path)):
+        if len(r) < 15 or r[0] == "ID":
+            continue
+        k = r[4].split("(")[0].replace("unnamed>::", "")
+        out.setdefault(k, {})[r[12]] = r[14]
+    log = os.path.join(OUT, "ncu_host.log")
+    if os.path.exists(log):
+        for line in open(log):
+            if line.startswith("{") and "wire_in" in line:
+                out["step"] = json.loads(line)
+    out["note"] = ("pcie__read_bytes / pcie__write_bytes are link-level counts (they include TLP protocol "
+                   "overhead); compare them with the step's wire_in / reply_wire")
+    return out
 
 
 if __name__ == "__main__":

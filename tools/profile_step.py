@@ -7,6 +7,7 @@
       -c 1 -o gpurun_out/mover python tools/profile_step.py --steps 1
 """
 import argparse
+import json
 import os
 import sys
 
@@ -39,6 +40,8 @@ def main():
     torch.cuda.synchronize()
     torch.cuda.profiler.stop()
     print(workload.check_results(idx, ep))
+    print(json.dumps({"wire_in": ep.wire_in, "reply_wire": ep.reply_wire, "h2d_payload": ep.h2d_payload,
+                      "d2h_payload": ep.d2h_payload, "host_rings": a.host, "steps_profiled": a.steps}))
 
 
 if __name__ == "__main__":

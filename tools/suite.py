@@ -169,12 +169,13 @@ def server_latency(ctx, reps=2000):
     torch.cuda.synchronize()
     srv = crk.Server(idx, [ring], [send], base, region.numel())
     try:
-        rt, dv = [], []
+        rt, dv, ph = [], [], []
         for i in range(reps):
             t0 = time.perf_counter_ns()
             out = srv.step([(0, w)], [0])
             rt.append(time.perf_counter_ns() - t0)
             dv.append(out["device_ns"])
+            ph.append(list(out["phase_end_ns"].values()))
         ok = out["results"][0]["status"] == 0 and out["results"][0]["reply_bytes"] == 32
     finally:
         srv.stop()
@@ -193,6 +194,8 @@ def server_latency(ctx, reps=2000):
     return {"one_record_roundtrip_us_median": round(float(np.median(rt)) / 1e3, 2),
             "one_record_device_us_median": round(float(np.median(dv)) / 1e3, 2),
             "one_record_roundtrip_us_p99": round(float(np.percentile(rt, 99)) / 1e3, 2), "ok": bool(ok),
+            "one_record_phase_end_us_median": dict(zip(("setup", "scan", "parse", "plan", "move"),
+                                                      [round(float(x) / 1e3, 2) for x in np.median(ph, axis=0)])),
             "c2_batch_device_us_median": round(float(np.median(c2dv)) / 1e3, 2), "c2_ok": bool(ok2)}
 
 
