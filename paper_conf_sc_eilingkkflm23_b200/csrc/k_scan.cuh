@@ -458,7 +458,10 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
     const uint32_t nf = S.nf, nr = S.nr, f0 = S.f0;
     // ---- both groups speculate from the true header at p; thread u owns candidates u + j*T
-    uint32_t hpred = S.hp[grp];
+    // both predictors are read here, before the round's first barrier: the thread that advances the
+    // walk rewrites S.hp at the end of this round, possibly while others are still past that barrier
+    const uint32_t hp0 = S.hp[0], hp1 = S.hp[1];
+    uint32_t hpred = grp ? hp1 : hp0;
     const uint64_t stride = 4 + (uint64_t)(hpred & 0x7fffffffu);
     // a round uses kJ candidates per thread only after a round that accepted every candidate (a long
     // regular run: big records); otherwise one, which keeps the round short
@@ -501,8 +504,9 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     const uint32_t tstar = win ? ts1 : ts0;
     const uint32_t wstar = win ? ws1 : ws0;
     const bool mine = grp == win;
-    hpred = S.hp[win];
+    hpred = win ? hp1 : hp0;
     const uint64_t Lp = hpred & 0x7fffffffu;
+    const uint64_t wstride = 4 + Lp;  // the winning predictor's stride (stride is this group's own)
     const uint32_t lastp = hpred >> 31;
     const bool end_at_star = tstar < TT && !S.gv[wstar];
     const uint32_t n_hdr = tstar == TT ? TT : (end_at_star ? tstar : tstar + 1);
@@ -517,7 +521,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     for (uint32_t k = 0; k < 3; ++k) {
       const uint32_t t = k == 0 ? 0u : (k == 1 ? (n_hdr > 1 ? 1u : 0u) : (n_hdr ? n_hdr - 1 : 0u));
       if (t >= n_hdr) continue;
-      const uint64_t q = p + (uint64_t)t * stride;
+      const uint64_t q = p + (uint64_t)t * wstride;
       const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
       const bool start = (t == 0) ? (p == r0) : (lastp != 0);
       uint64_t send;
@@ -533,7 +537,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
 #pragma unroll
       for (uint32_t j = 0; j < kJ; ++j) {
         const uint32_t t = u + j * T;
-        const uint64_t q = p + (uint64_t)t * stride;
+        const uint64_t q = p + (uint64_t)t * wstride;
         const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
         const bool start = (t == 0) ? (p == r0) : (lastp != 0);
         uint64_t send;  // logical end of header t within its record (segmented prefix sum of lengths)
@@ -567,7 +571,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     for (uint32_t j = 0; j < kJ; ++j) {
       const uint32_t t = u + j * T;
       if (!mine || j >= jn) break;
-      const uint64_t q = p + (uint64_t)t * stride;
+      const uint64_t q = p + (uint64_t)t * wstride;
       const uint64_t len = (t < tstar) ? Lp : (uint64_t)(hstar & 0x7fffffffu);
       const uint32_t last = (t < tstar) ? lastp : (hstar >> 31);
       const bool start = (t == 0) ? (p == r0) : (lastp != 0);
