@@ -27,6 +27,12 @@ from paper_conf_sc_eilingkkflm23_b200 import build, crk, gen  # noqa: E402
 
 MiB, GiB = 1 << 20, 1 << 30
 dev = torch.device("cuda:0")
+# crk_config overrides for every context of the suite, e.g. SUITE_CTX=scan_threads=512
+CTX_KW = {k: int(v, 0) for k, v in (kv.split("=") for kv in os.environ.get("SUITE_CTX", "").split(",") if kv)}
+
+
+def Ctx():
+    return crk.Context(0, **CTX_KW)
 
 
 def timed(fn, reps, warm=3):
@@ -357,18 +363,18 @@ def main():
     build.build()
     only = [x for x in os.environ.get("SUITE_ONLY", "").split(",") if x]
     runs = {
-        "C1": lambda: c1(crk.Context(0)),
-        "C1_serve_one_record": lambda: serve_latency(crk.Context(0)),
-        "C2_matrixMul": lambda: c2(crk.Context(0)),
-        "NEXT3_server": lambda: server_latency(crk.Context(0)),
-        "C3_sweep": lambda: c3(crk.Context(0)),
-        "C4_typed_regular": lambda: c4(crk.Context(0), False),
-        "C4_typed_irregular": lambda: c4(crk.Context(0), True),
-        "NEXT1_striped_1GiB_16_rings": lambda: served(crk.Context(0), [64 * MiB] * 16, [], streams=16),
-        "NEXT1_single_1GiB_1_ring": lambda: served(crk.Context(0), [GiB], [], streams=1),
-        "NEXT2_cusolver_100_iters": lambda: served(crk.Context(0), [900 * 900 * 8] * 100, [900 * 8] * 100,
+        "C1": lambda: c1(Ctx()),
+        "C1_serve_one_record": lambda: serve_latency(Ctx()),
+        "C2_matrixMul": lambda: c2(Ctx()),
+        "NEXT3_server": lambda: server_latency(Ctx()),
+        "C3_sweep": lambda: c3(Ctx()),
+        "C4_typed_regular": lambda: c4(Ctx(), False),
+        "C4_typed_irregular": lambda: c4(Ctx(), True),
+        "NEXT1_striped_1GiB_16_rings": lambda: served(Ctx(), [64 * MiB] * 16, [], streams=16),
+        "NEXT1_single_1GiB_1_ring": lambda: served(Ctx(), [GiB], [], streams=1),
+        "NEXT2_cusolver_100_iters": lambda: served(Ctx(), [900 * 900 * 8] * 100, [900 * 8] * 100,
                                                    streams=1, reps=10),
-        "NEXT2_histogram": lambda: served(crk.Context(0), [64 * MiB], [256 * 4], streams=1),
+        "NEXT2_histogram": lambda: served(Ctx(), [64 * MiB], [256 * 4], streams=1),
     }
     out = {}
     t0 = time.time()
