@@ -105,6 +105,12 @@ typedef struct {
   uint32_t mover_reserve_ctas; /* mover CTA slots left free (default 0), < half the grid: with several batches in
                                   flight on other streams, the next batch's scan / parse / plan kernels and the
                                   start of its mover find room on the GPU while this mover streams */
+  uint32_t fused_front_max_records; /* crk_serve with an index of at most this many records (and one ring, or
+                                       at most fused_front_max_window bytes of ring windows) runs scan + parse +
+                                       planning as ONE single-CTA launch before the mover (default 128, at most
+                                       1024 takes effect; 0 = always separate kernels) */
+  uint32_t pad0_;
+  uint64_t fused_front_max_window; /* default 1 MiB (one CTA scans the rings in turn) */
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;
@@ -377,7 +383,8 @@ int crk_copy_to_host(void* host_dst, const void* dev_src, uint64_t bytes);
 
 /* ---------------------------------------------------------------- profiling
  * When enabled, CUDA events are recorded on the launching stream around each pipeline stage:
- * 0 = frame scan (K1), 1 = CALL parse (K3), 2 = serve planning (statuses, K2 reply offsets, jobs),
+ * 0 = frame scan (K1; or the fused small-step front end, which also parses and plans), 1 = CALL parse (K3),
+ * 2 = serve planning (statuses, K2 reply offsets, jobs),
  * 3 = the bulk mover (K4-K7).  crk_profile_read waits for the events, returns the summed device time
  * (ms[4]) and the number of timed launches (launches[4]) since the last read, and resets them. */
 int crk_profile_enable(int on);

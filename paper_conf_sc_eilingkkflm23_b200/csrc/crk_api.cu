@@ -115,12 +115,12 @@ void add_builtin(SchemaTable& t, uint32_t proc, std::initializer_list<uint32_t> 
   for (uint32_t k : items) s.items[s.n_items++] = k;
 }
 
-int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
-             const uint64_t* tails, cudaStream_t s, const uint64_t* doorbell = nullptr) {
+// Validated scan parameters (host-argument checks of crk_rpc_frame_scan / crk_serve).
+int scan_param(crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
+               const uint64_t* tails, const uint64_t* doorbell, ScanRingsParam& P) {
   if (!rings || (!doorbell && (!heads || !tails)) || n_rings == 0 || n_rings > (uint32_t)kMaxRings ||
       n_rings > idx->ix.max_rings)
     return CRK_E_ARG;
-  ScanRingsParam P;
   memset(&P, 0, sizeof(P));
   P.n_rings = n_rings;
   P.doorbell = doorbell;
@@ -132,6 +132,28 @@ int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rin
     }
     if (tails[r] < heads[r] || tails[r] - heads[r] > rings[r].cap) return CRK_E_ARG;
     P.r[r] = ring_desc(rings[r], heads[r], tails[r]);
+  }
+  return CRK_OK;
+}
+
+// A small index (crk_config.fused_front_max_records) over one ring or a small window: one fused launch.
+bool fused_front(const crk_ctx* c, const crk_index* x, uint32_t n_rings, const uint64_t* heads, const uint64_t* tails,
+                 const uint64_t* doorbell) {
+  uint64_t window = 0;
+  for (uint32_t r = 0; !doorbell && heads && tails && r < n_rings; ++r) window += tails[r] - heads[r];
+  return x->ix.max_records <= c->cfg.fused_front_max_records && x->ix.max_records <= front_small_threads() &&
+         (n_rings == 1 || (!doorbell && window <= c->cfg.fused_front_max_window));
+}
+
+int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
+             const uint64_t* tails, cudaStream_t s, const uint64_t* doorbell = nullptr) {
+  ScanRingsParam P;
+  const int st = scan_param(idx, n_rings, rings, heads, tails, doorbell, P);
+  if (st != CRK_OK) return st;
+  if (fused_front(ctx, idx, n_rings, heads, tails, doorbell)) {  // scan + parse in one launch
+    CK(launch_front_small(idx->ix, ctx->cd, ctx->sc, ctx->d_schemas, P, n_rings, nullptr, nullptr, 0, 0, doorbell,
+                          false, s));
+    return CRK_OK;
   }
   CK(cudaMemsetAsync(idx->ix.xid_hash, 0xff, sizeof(unsigned long long) * ((uint64_t)idx->ix.hash_mask + 1), s));
   CK(launch_frame_scan(idx->ix, P, ctx->cd, s));
@@ -238,6 +260,8 @@ void crk_config_init(crk_config* c) {
   c->mover_run = 8;
   c->mover_tail_tiles = 2;
   c->mover_reserve_ctas = 0;
+  c->fused_front_max_records = 128;
+  c->fused_front_max_window = 1ull << 20;
 }
 
 int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
@@ -693,6 +717,18 @@ int run_serve(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring* rings,
   if (2ull * x->ix.max_records > c->sc.max_jobs) return CRK_E_CAPACITY;
   for (uint32_t r = 0; r < n_rings && r < (uint32_t)kMaxRings; ++r)
     if (!ring_ok(send_rings[r])) return CRK_E_ARG;
+  // small step (an index of at most cfg.fused_front_max_records records; one ring, or at most
+  // cfg.fused_front_max_window bytes of windows): scan, parse and planning fused into one single-CTA
+  // launch, then the mover
+  if (fused_front(c, x, n_rings, heads, tails, doorbell)) {
+    ScanRingsParam P;
+    const int st = scan_param(x, n_rings, rings, heads, tails, doorbell, P);
+    if (st != CRK_OK) return st;
+    CK(launch_front_small(x->ix, c->cd, c->sc, c->d_schemas, P, n_rings, send_rings, send_offs, region_base,
+                          region_bytes, doorbell, true, s));
+    CK(launch_mover(&x->ix, c->cd, c->sc, c->cd.run, c->move_ctas, s));
+    return CRK_OK;
+  }
   int st = run_scan(c, x, n_rings, rings, heads, tails, s, doorbell);
   if (st != CRK_OK) return st;
   if (x->ix.max_records <= kSmallServe) {  // small batch: one planning launch, then the mover

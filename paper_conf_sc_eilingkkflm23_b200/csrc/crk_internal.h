@@ -177,6 +177,14 @@ cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Sc
                                     const crk_ring* send_rings, const uint64_t* send_offs, uint64_t region_base,
                                     uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s);
 
+// Fused front end for small serve steps (k_front.cu): scan + parse + plan_small_block in one CTA; the
+// mover (launch_mover) follows.  rings: validated scan parameters (cursors or doorbell).
+uint32_t front_small_threads();
+cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, const SchemaTable* schemas,
+                               const ScanRingsParam& rings, uint32_t n_rings, const crk_ring* send_rings,
+                               const uint64_t* send_offs, uint64_t region_base, uint64_t region_bytes,
+                               const uint64_t* doorbell, bool plan, cudaStream_t s);
+
 // Persistent server (k_server.cu): one resident CTA of server_threads() threads.
 uint32_t server_threads();
 cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SchemaTable* schemas,

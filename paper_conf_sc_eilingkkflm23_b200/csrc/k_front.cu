@@ -1,0 +1,116 @@
+// Fused front end for small steps: K1 (scan), K3 (parse) and the one-block serve planner in ONE launch
+// of one CTA, followed by the ordinary mover launch (crk_serve); scan + parse only for a small
+// crk_rpc_frame_scan.  A small step (a few records, e.g. one forwarded cudaMemcpy of a few KiB: SURVEY.md
+// §8(d) C1 and the small end of the C3 sweep) is a chain of dependent memory round trips; as five
+// launches (hash clear, scan, parse, plan, mover) each round trip also pays a launch gap.  The device
+// functions are the launched kernels' own (scan_ring_cta, parse_record, plan_small_block), so the index
+// tables, statuses and jobs are identical; the phases hand data to each other inside the CTA, ordered by
+// block barriers.
+#include "k_parse.cuh"
+#include "k_plan.cuh"
+#include "k_scan.cuh"
+
+namespace crk {
+
+namespace {
+
+constexpr uint32_t kFrontThreads = kSmallServe;  // plan_small_block: thread d owns record d
+constexpr uint32_t kFrontWarps = kFrontThreads / 32;
+
+struct FrontParams {
+  IndexDev ix;
+  ConfigDev cfg;
+  Scratch sc;
+  const SchemaTable* schemas;
+  ScanRingsParam rings;  // cursors in r[] or, with rings.doorbell, read here at execution time
+  SendRingsParam send;
+  uint64_t region_base, region_bytes;
+  uint32_t plan;         // 0: scan + parse only (crk_rpc_frame_scan)
+};
+
+__global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontParams P) {
+  __shared__ ScanState S;
+  __shared__ SchemaTable sch;
+  __shared__ __align__(16) uint8_t heads[kFrontWarps][kHeadBuf];
+  __shared__ uint64_t warp_sums[32];
+  __shared__ uint64_t ring_first_pre[kMaxRings];
+  __shared__ uint32_t prefix[kMaxRings + 1];
+  TL_BEGIN(P.cfg, TL_FUSED);
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const IndexDev& ix = P.ix;
+  const uint32_t n_rings = P.rings.n_rings;
+  // ---- setup: schemas, an empty xid table
+  for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
+    reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
+  for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
+  __syncthreads();
+  // ---- K1: each ring in turn by the whole CTA, then dense record numbering
+  for (uint32_t r = 0; r < n_rings; ++r) {
+    RingDesc R = P.rings.r[r];
+    bool bad = false;
+    if (P.rings.doorbell) {
+      R.head = P.rings.doorbell[r];
+      R.tail = P.rings.doorbell[n_rings + r];
+      bad = R.tail < R.head || R.tail - R.head > R.mask + 1;
+      if (bad) R.tail = R.head;
+    }
+    scan_ring_cta(ix, R, bad, r, P.cfg, S);
+  }
+  if (threadIdx.x == 0) dense_numbering(ix, n_rings);
+  __syncthreads();
+  // ---- K3: one warp per record
+  for (uint32_t i = threadIdx.x; i <= n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
+  __syncthreads();
+  const uint32_t total = prefix[n_rings];
+  for (uint32_t d = warp; d < total; d += kFrontWarps) {
+    uint32_t lo = 0, hi = n_rings;  // ring of dense record d
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (prefix[mid] <= d) lo = mid; else hi = mid;
+    }
+    parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane);
+    __syncwarp();
+  }
+  if (!P.plan) {
+    TL_END(P.cfg, TL_FUSED);
+    return;
+  }
+  __syncthreads();
+  // ---- serve planning: statuses, reply offsets, jobs, their tile prefix, mover cursors
+  plan_small_block(ix, P.cfg, P.sc, P.send, P.region_base, P.region_bytes, warp_sums, ring_first_pre);
+  TL_END(P.cfg, TL_FUSED);
+}
+
+}  // namespace
+
+uint32_t front_small_threads() { return kFrontThreads; }
+
+cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, const SchemaTable* schemas,
+                               const ScanRingsParam& rings, uint32_t n_rings, const crk_ring* send_rings,
+                               const uint64_t* send_offs, uint64_t region_base, uint64_t region_bytes,
+                               const uint64_t* doorbell, bool plan, cudaStream_t s) {
+  FrontParams P;
+  memset(&P, 0, sizeof(P));
+  P.ix = ix;
+  P.cfg = cfg;
+  P.sc = sc;
+  P.schemas = schemas;
+  P.rings = rings;
+  P.plan = plan;
+  P.send.n_rings = n_rings;
+  for (uint32_t r = 0; plan && r < n_rings; ++r) {
+    P.send.r[r].base = send_rings[r].base;
+    P.send.r[r].mask = send_rings[r].cap - 1;
+    P.send.off[r] = send_offs ? send_offs[r] : 0;
+  }
+  P.send.doorbell = doorbell;
+  P.region_base = region_base;
+  P.region_bytes = region_bytes;
+  prof_mark(PROF_SCAN, true, s);
+  front_small_kernel<<<1, kFrontThreads, 0, s>>>(P);
+  count_launch();
+  prof_mark(PROF_SCAN, false, s);
+  return cudaGetLastError();
+}
+
+}  // namespace crk

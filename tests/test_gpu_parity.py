@@ -561,10 +561,12 @@ def test_encode_replies_batch_matches_oracle(host, F):
 
 
 MOVER_CONFIGS = [{}, {"mover_tail_tiles": 0, "mover_reserve_ctas": 16},
-                 {"mover_tail_tiles": 64, "mover_run": 1, "tile_bytes": 4096}, {"mover_tail_tiles": 1, "mover_run": 64}]
+                 {"mover_tail_tiles": 64, "mover_run": 1, "tile_bytes": 4096}, {"mover_tail_tiles": 1, "mover_run": 64},
+                 # the fused single-CTA front end (scan + parse + plan in one launch) on the same batch
+                 {"fused_front_max_records": 1024, "fused_front_max_window": 1 << 40}]
 
 
-@pytest.mark.parametrize("host,mover", [(False, m) for m in range(len(MOVER_CONFIGS))] + [(True, 0)])
+@pytest.mark.parametrize("host,mover", [(False, m) for m in range(len(MOVER_CONFIGS))] + [(True, 0), (True, 4)])
 def test_serve_matches_oracle(host, mover):
     cfg = ocfg(F=16384)
     ctx = ctx_for(cfg, **MOVER_CONFIGS[mover])
@@ -652,11 +654,12 @@ def test_ring_copy_and_async_results():
     assert rows[0]["status"] == O.OK and rows[0]["n_records"] == 1 and rows[1]["status"] == O.INCOMPLETE
 
 
-@pytest.mark.parametrize("strict", [True, False])
-def test_serve_cred_bodies_lenient_and_duplicates_match_oracle(strict):
-    """Non-empty cred/verf bodies (args start past the prefetched head), odd pads, lenient mode."""
+@pytest.mark.parametrize("strict,fused", [(True, False), (False, False), (True, True), (False, True)])
+def test_serve_cred_bodies_lenient_and_duplicates_match_oracle(strict, fused):
+    """Non-empty cred/verf bodies (args start past the prefetched head), odd pads, lenient mode; through the
+    separate scan / parse / plan kernels and through the fused single-CTA front end."""
     cfg = ocfg(strict=strict, F=3000)
-    ctx = ctx_for(cfg)
+    ctx = ctx_for(cfg, fused_front_max_records=1024 if fused else 0)
     region = torch.zeros(1 << 20, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
     host_region = np.zeros(1 << 20, np.uint8)
