@@ -396,6 +396,9 @@ def main():
         ctxs = [s.ctx for s in slots]
         del slots
         torch.cuda.empty_cache()
+        # host-link peaks (copy engine, pinned) measured before the rings are allocated (their buffers get
+        # the same placement the rings get) and again after the runs; the roofline takes the better of the two
+        link0 = host_link_peaks(dev)
         P = max(1, args.e2e_pipeline)  # batches in flight for the host-memory runs
         while len(ctxs) < P:
             ctxs.append(crk.Context(local, **ctx_kw))
@@ -455,6 +458,28 @@ def main():
             hslots[0].ep.sends[0].read(0, n0) == hslots[0].ep.dev_sends[0].read(0, n0))
         check_st["ok"] = check_st["ok"] and check_st["host_send_matches_device"]
 
+        def run_mixed(n_steps):
+            # copy engine in, SM zero-copy out: the inbound window is DMA'd into the device ring, the mover
+            # writes the replies straight into the pinned host send rings (no outbound DMA)
+            for k in range(n_steps):
+                s = hslots[k % P]
+                s.in_stream.wait_event(s.ev_served)
+                workload.staged_in(s.ep, s.in_stream)
+                s.ev_in.record(s.in_stream)
+                s.stream.wait_event(s.ev_in)
+                s.idx.serve([(dr, h, t) for dr, (_, h, t) in zip(s.ep.dev_rings, s.ep.rings)], s.ep.sends,
+                            s.ep.offs, s.ep.base, s.ep.region.numel(), stream=s.stream)
+                s.idx.ring_results_async(s.res, stream=s.stream)
+                s.ev_served.record(s.stream)
+            torch.cuda.synchronize()
+
+        run_mixed(max(2, min(args.warmup, 4)))
+        barrier()
+        t0 = time.perf_counter()
+        run_mixed(args.e2e_steps)
+        el_mx = max_over_ranks(time.perf_counter() - t0)
+        check_mx = workload.check_results(hslots[0].idx, ep_h)
+
         def run_e2e(n_steps):
             # step k is launched before the results of step k-1 are read back (device -> host, syncs
             # that slot's stream), so the host read overlaps the next batch
@@ -478,7 +503,10 @@ def main():
         res_bytes = len(ep_h.rings) * 40
         e2e_v = sum_over_ranks(ep_h.payload) * args.e2e_steps / el_max / 1e9
         # live host-link peaks (copy engine, pinned) for the e2e roofline
-        link = host_link_peaks(dev)
+        link1 = host_link_peaks(dev)
+        link = {k: max(link0[k], link1[k]) for k in link0}
+        link["measured"] = "best of two measurements (before allocating the rings, after the runs)"
+        link["before"], link["after"] = link0, link1
         t_link = max(ep_h.wire_in / link["ce_h2d_gbs"], ep_h.reply_wire / link["ce_d2h_gbs"],
                      (ep_h.wire_in + ep_h.reply_wire) / link["ce_bidir_gbs"]) / 1e9
         modes = []
@@ -487,7 +515,10 @@ def main():
                  f"{P} batches in flight", el_max, check_h),
                 (f"copy-engine staged: crk_ring_copy DMAs each receive window into a device ring, crk_serve "
                  f"decodes from HBM into device send rings, crk_ring_copy DMAs the replies back; {P} batches in "
-                 f"flight", el_st, check_st)):
+                 f"flight", el_st, check_st),
+                (f"mixed: crk_ring_copy DMAs each receive window into a device ring, crk_serve decodes from HBM "
+                 f"and the mover writes the replies straight into the pinned host send rings; {P} batches in "
+                 f"flight", el_mx, check_mx)):
             step_s = el_m / args.e2e_steps
             modes.append({"value": round(sum_over_ranks(ep_h.payload) / step_s / 1e9, 3), "unit": "GB/s",
                           "h2d_bytes_per_step": ep_h.wire_in, "d2h_bytes_per_step": ep_h.reply_wire + res_bytes,
@@ -499,7 +530,7 @@ def main():
                           "check": chk})
         modes.sort(key=lambda m: -m["value"] if m["check"]["ok"] else 0)
         e2e = dict(modes[0])
-        e2e["other_mode"] = {k: modes[1][k] for k in ("value", "mode", "ms_per_step", "check")}
+        e2e["other_modes"] = [{k: m[k] for k in ("value", "mode", "ms_per_step", "check")} for m in modes[1:]]
 
     out = {
         "metric": "xdr_memcpy_serve_payload_GBps", "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
