@@ -88,3 +88,31 @@ def test_generator_is_deterministic():
     assert [(r.kind, r.xid, r.size, r.region_off) for s in a for r in s.records] == \
            [(r.kind, r.xid, r.size, r.region_off) for s in b for r in s.records]
     assert gen.c3_payload(12).tobytes() == gen.c3_payload(12).tobytes()
+
+
+def test_ctypes_layouts_match_the_header(tmp_path):
+    """The binding's ctypes mirrors of the public structs have the header's sizes and field offsets (gcc
+    compiles a probe against include/crk.h; no CUDA headers needed)."""
+    import ctypes as C
+    import subprocess
+    structs = {"crk_config": crk.Config, "crk_ring": crk.CRing, "crk_ring_result": crk.RingResult,
+               "crk_index_view": crk.IndexView, "crk_item_req": crk.ItemReq, "crk_item_src": crk.ItemSrc,
+               "crk_reply_req": crk.ReplyReq, "crk_server_bell": crk.ServerBell}
+    lines = ["#include <stdio.h>", "#include <stddef.h>", '#include "crk.h"', "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'  printf("{cname} size %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'  printf("{cname} {f} %zu\\n", offsetof({cname}, {f}));')
+    lines += ["  return 0;", "}"]
+    src = tmp_path / "probe.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "probe"
+    subprocess.run(["gcc", "-std=c11", f"-I{build.ROOT}/include", "-o", str(exe), str(src)], check=True)
+    got = {}
+    for line in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.splitlines():
+        name, field, val = line.split()
+        got[(name, field)] = int(val)
+    for cname, py in structs.items():
+        assert got[(cname, "size")] == C.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
