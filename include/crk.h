@@ -102,9 +102,11 @@ typedef struct {
   uint32_t mover_run;        /* tiles per mover claim, 1..64 (default 8) */
   uint32_t mover_tail_tiles; /* per mover CTA, the last tiles of each queue claimed one at a time, 0..64 (default 2;
                                 shortens the kernel's tail when it runs alone) */
-  uint32_t mover_reserve_ctas; /* mover CTA slots left free (default 0), < half the grid: with several batches in
-                                  flight on other streams, the next batch's scan / parse / plan kernels and the
-                                  start of its mover find room on the GPU while this mover streams */
+  uint32_t mover_reserve_ctas; /* opportunistic mover CTAs (default 0, < half the grid): the last N CTAs of a
+                                  mover launch run only if they start within 10 us of its first CTA (the GPU was
+                                  free: a lone call gets the whole grid); behind another batch's mover (several
+                                  batches in flight on other streams) they exit at once, so the next batch's
+                                  scan / parse / plan kernels find room on the GPU while this mover streams */
   uint32_t fused_front_max_records; /* crk_serve with an index of at most this many records (and one ring, or
                                        at most fused_front_max_window bytes of ring windows) runs scan + parse +
                                        planning as ONE single-CTA launch before the mover (default 128, at most

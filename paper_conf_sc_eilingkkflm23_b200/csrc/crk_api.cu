@@ -288,7 +288,6 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   int occ = cfg.ctas_per_sm ? (int)cfg.ctas_per_sm : mover_occupancy(cfg.tile_bytes, cfg.mover_stages);
   c->move_ctas = c->sms * (occ > 0 ? occ : 1);
   if (2ull * cfg.mover_reserve_ctas >= (uint64_t)c->move_ctas) { delete c; return CRK_E_ARG; }
-  c->move_ctas -= (int)cfg.mover_reserve_ctas;
   ConfigDev& d = c->cd;
   d.F = cfg.frag_payload;
   d.strict = cfg.strict ? 1 : 0;
@@ -304,6 +303,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.stages = cfg.mover_stages;
   d.run = cfg.mover_run;
   d.tail = cfg.mover_tail_tiles;
+  d.reserve = cfg.mover_reserve_ctas;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
   // scratch: one block

@@ -97,18 +97,21 @@ struct Job {              // 64 bytes
 struct Scratch {          // ctx-owned device scratch
   Job* jobs;              // [max_jobs]
   Piece* pieces;          // [2 * max_jobs]
-  uint32_t* counters;     // [8]: 0/2 mover decode/encode run cursors, 3/6 their single-tile tail cursors, 1 n_jobs, 4 queue split, 5 K2 block counter
+  uint32_t* counters;     // [16]: 0/2 mover decode/encode run cursors, 3/6 their single-tile tail cursors, 1 n_jobs,
+                          // 4 queue split, 5 K2 block counter, 8/9 mover launch stamp (sequence, start time)
   uint64_t* lens_pool;    // explicit framing: [2 * max_lens] (lens, then wire starts)
   uint32_t* lens32;       // [max_lens] staging for host-given fragment lengths
   unsigned long long* scan_state;  // decoupled look-back state for K2
   uint64_t* scan_tmp;     // [max_jobs + 2]: sizes -> prefix; [max_jobs + 1] = total
   RingDesc* out_rings;    // [kMaxRings]
   uint32_t max_jobs, max_lens, max_pieces;
+  uint32_t mover_seq;     // host-side count of this context's mover launches (the launch stamp's sequence)
 };
 
 struct ConfigDev {
   uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
   uint32_t scan_threads, stages, run, tail;  // tail: per-CTA single-tile claims at the end of each queue
+  uint32_t reserve, pad_;  // mover CTAs that run only when the launch found the GPU free (crk_config.mover_reserve_ctas)
   uint64_t max_record_bytes;
   unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };

@@ -58,7 +58,43 @@ struct MoveParams {
   const uint32_t* n_jobs_dev;
   const uint64_t* total_tiles;
   uint32_t stage_bytes;    // bytes of one stage buffer (after its header)
+  uint32_t seq;            // this launch's number (launch stamp)
+  uint32_t opp_from;       // CTAs >= opp_from are opportunistic (crk_config.mover_reserve_ctas)
 };
+
+__device__ __forceinline__ uint32_t gtimer32() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return (uint32_t)t;
+}
+// Opportunistic CTAs (the last cfg.reserve of the grid) join only a launch that found the GPU free: the
+// whole grid starts within a few microseconds of CTA 0.  When this mover launches while another batch's
+// mover still holds the SMs (a pipelined server loop), its last CTAs are dispatched only when that mover
+// retires, long after CTA 0 started; they exit at once, so their slots stay free for the next batch's scan /
+// parse / plan kernels.  CTA 0 stamps the launch (sequence, start time) in the context's counters.
+constexpr uint32_t kOppLateNs = 10000;
+__device__ bool mover_cta_runs(const MoveParams& M) {
+  __shared__ uint32_t go;
+  volatile uint32_t* c = M.sc.counters;
+  if (threadIdx.x == 0) {
+    const uint32_t t = gtimer32();
+    uint32_t g = 1;
+    if (blockIdx.x == 0) {
+      c[9] = t;
+      __threadfence();
+      c[8] = M.seq;
+    } else if (blockIdx.x >= M.opp_from) {
+      while (c[8] != M.seq && gtimer32() - t < 2 * kOppLateNs) __nanosleep(256);
+      if (c[8] == M.seq) {
+        __threadfence();
+        g = t - c[9] < kOppLateNs;
+      }
+    }
+    go = g;
+  }
+  __syncthreads();
+  return go != 0;
+}
 
 // ------------------------------------------------------------------------------------------- PTX
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -233,6 +269,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
   const uint32_t kStages = M.cfg.stages;
   const uint32_t stage_stride = (sizeof(StageHdr) + 127) / 128 * 128 + M.stage_bytes;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (!mover_cta_runs(M)) return;
   TL_BEGIN(M.cfg, TL_MOVE);
   if (threadIdx.x == 0) {
     for (uint32_t s = 0; s < kStages; ++s) {
@@ -620,6 +657,8 @@ cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, 
   M.n_jobs_dev = sc.counters + 1;
   M.total_tiles = sc.scan_tmp + sc.max_jobs + 1;
   M.stage_bytes = (1u << cfg.tile_shift) + 32 * kMaxSeg + 32;
+  M.seq = ++sc.mover_seq;
+  M.opp_from = (uint32_t)move_ctas > 2 * cfg.reserve ? (uint32_t)move_ctas - cfg.reserve : (uint32_t)move_ctas;
   const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
   static uint32_t smem_set = 0;  // dynamic shared memory opt-in (per process, grows monotonically)
   if (smem > smem_set) {
