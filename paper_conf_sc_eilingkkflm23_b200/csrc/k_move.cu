@@ -38,7 +38,7 @@ struct Seg {               // 32 bytes
   uint64_t out_a, out_b;   // output range (DEC: dst addresses; ENC: out-ring cursors)
   uint64_t src;            // DEC: ring cursor of the byte for out_a; ENC: V-order address of the byte for out_a
   uint32_t smem_off;       // offset in the stage buffer of the aligned source window (staged only)
-  uint32_t flags;          // bit 0 staged, bits 8-15 kind, bits 16-23 element size
+  uint32_t flags;          // bit 0 staged, bit 1 edge bytes staged too, bits 8-15 kind, bits 16-23 element size
 };
 
 struct StageHdr {
@@ -409,7 +409,13 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
               if (c0 < c1) {  // stage the source window of the interior chunks
                 const uint64_t s0 = g.src + (c0 - r);
                 const uint64_t w0 = s0 & ~15ull, w1 = (s0 + (c1 - c0) + 15) & ~15ull;
-                stage_window(g, pc.R.base, pc.R.mask, true, w0, w1);
+                if (J.esize == 1) {  // bytes: widen the window over the edge bytes (at most 16 B each side)
+                  const uint64_t wa = g.src & ~15ull, wb = (g.src + (sb - r) + 15) & ~15ull;
+                  stage_window(g, pc.R.base, pc.R.mask, true, wa, wb);
+                  if (g.flags & 1) { g.smem_off += (uint32_t)(w0 - wa); g.flags |= 2; }
+                } else {
+                  stage_window(g, pc.R.base, pc.R.mask, true, w0, w1);
+                }
               }
               r = sb;
             }
@@ -437,7 +443,13 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
               if (c0 < c1) {
                 const uint64_t s0 = src + (c0 - g.out_a);
                 const uint64_t w0 = s0 & ~15ull, w1 = (s0 + (c1 - c0) + 15) & ~15ull;
-                stage_window(g, nullptr, 0, false, w0, w1);
+                if (es == 1) {  // bytes: widen over the edge bytes (16-byte granules never cross a page)
+                  const uint64_t wa = src & ~15ull, wb = (src + (g.out_b - g.out_a) + 15) & ~15ull;
+                  stage_window(g, nullptr, 0, false, wa, wb);
+                  if (g.flags & 1) { g.smem_off += (uint32_t)(w0 - wa); g.flags |= 2; }
+                } else {
+                  stage_window(g, nullptr, 0, false, w0, w1);
+                }
               }
             }
             return true;
@@ -489,13 +501,15 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
             }
             const uint64_t s0 = S.src + (c0 - S.out_a);
             staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, nullptr, es, true);
-            // edge bytes
+            // edge bytes (from the stage when the producer widened the window over them)
             const uint64_t ea = min(S.out_b, c0), eb = max(S.out_a, c1);
             const uint32_t ne = (uint32_t)((ea - S.out_a) + (S.out_b - eb));
             if (T.tid < ne) {
               const uint64_t x = T.tid < ea - S.out_a ? S.out_a + T.tid : eb + (T.tid - (ea - S.out_a));
               uint8_t v;
-              if (es == 1) {
+              if (S.flags & 2) {
+                v = buf[(int64_t)S.smem_off + (int64_t)(S.src + (x - S.out_a) - (s0 & ~15ull))];
+              } else if (es == 1) {
                 v = ring_byte(H.R, S.src + (x - S.out_a));
               } else {
                 DecCtx c;
@@ -526,8 +540,17 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
             const uint64_t c0 = (S.out_a + 15) & ~15ull, c1 = S.out_b & ~15ull;
             const uint64_t s0 = S.src + (c0 - S.out_a);
             staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, &H.R, es, false);
-            enc_bytes(T, c, S.out_a - c.start, min(S.out_b, c0) - c.start);
-            enc_bytes(T, c, max(S.out_a, c1) - c.start, S.out_b - c.start);
+            if (S.flags & 2) {  // edge bytes of plain data, from the widened stage window
+              const uint64_t ea = min(S.out_b, c0), eb = max(S.out_a, c1);
+              const uint32_t ne = (uint32_t)((ea - S.out_a) + (S.out_b - eb));
+              if (T.tid < ne) {
+                const uint64_t x = T.tid < ea - S.out_a ? S.out_a + T.tid : eb + (T.tid - (ea - S.out_a));
+                H.R.base[x & H.R.mask] = buf[(int64_t)S.smem_off + (int64_t)(S.src + (x - S.out_a) - (s0 & ~15ull))];
+              }
+            } else {
+              enc_bytes(T, c, S.out_a - c.start, min(S.out_b, c0) - c.start);
+              enc_bytes(T, c, max(S.out_a, c1) - c.start, S.out_b - c.start);
+            }
           }
         }
       }
