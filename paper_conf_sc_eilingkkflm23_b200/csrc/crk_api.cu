@@ -161,8 +161,9 @@ int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rin
   return CRK_OK;
 }
 
-int move(crk_ctx* ctx, const IndexDev* ix, uint32_t bound, cudaStream_t s, uint64_t out_bytes_bound = 0) {
-  CK(launch_plan_and_move(ix, ctx->cd, ctx->sc, bound, out_bytes_bound, ctx->sms, ctx->move_ctas, s));
+int move(crk_ctx* ctx, const IndexDev* ix, uint32_t bound, cudaStream_t s, uint64_t out_bytes_bound = 0,
+         bool planned = false) {
+  CK(launch_plan_and_move(ix, ctx->cd, ctx->sc, bound, out_bytes_bound, ctx->sms, ctx->move_ctas, s, planned));
   return CRK_OK;
 }
 
@@ -214,8 +215,8 @@ int encode_reply(crk_ctx* ctx, uint32_t xid, const void* src, uint64_t count, ui
   j.out_ring = 0;
   P.n_jobs = 1;
   *wire_bytes = wire;
-  CK(launch_put_enc_jobs(ctx->sc, P, ring_desc(out, 0, 0), s));
-  return move(ctx, nullptr, 1, s, wire);
+  CK(launch_put_enc_jobs(ctx->sc, ctx->cd, P, ring_desc(out, 0, 0), s));
+  return move(ctx, nullptr, 1, s, wire, true);
 }
 
 int decode_item_one(crk_ctx* ctx, crk_index* idx, uint32_t xid, uint32_t arg_no, uint32_t kind, void* dst,
@@ -234,7 +235,7 @@ int decode_item_one(crk_ctx* ctx, crk_index* idx, uint32_t xid, uint32_t arg_no,
   r.count = count_dev;
   r.status = status_dev;
   CK(launch_resolve_items(idx->ix, ctx->cd, ctx->sc, 1, nullptr, &r, s));
-  return move(ctx, &idx->ix, 1, s, max_count * es + 1);
+  return move(ctx, &idx->ix, 1, s, max_count * es + 1, true);
 }
 
 }  // namespace
@@ -531,7 +532,7 @@ int crk_xdr_decode_memcpy_h2d(crk_ctx* c, crk_index* x, uint32_t xid, void* dst,
   r.copied = copied_dev;
   cudaStream_t s = (cudaStream_t)stream;
   CK(launch_resolve_h2d(x->ix, c->cd, c->sc, 1, nullptr, nullptr, nullptr, nullptr, nullptr, &r, s));
-  return move(c, &x->ix, 1, s, dst_bytes + 1);
+  return move(c, &x->ix, 1, s, dst_bytes + 1, true);
 }
 
 int crk_xdr_decode_memcpy_h2d_batch(crk_ctx* c, crk_index* x, uint32_t n, const uint32_t* xids, void* const* dsts,
@@ -703,8 +704,8 @@ int crk_rpc_encode_call(crk_ctx* c, uint32_t xid, uint32_t proc, const crk_item_
   j.out_end = out_off + wire;
   P.n_jobs = 1;
   *wire_bytes = wire;
-  CK(launch_put_enc_jobs(c->sc, P, ring_desc(out, 0, 0), s));
-  return move(c, nullptr, 1, s, wire);
+  CK(launch_put_enc_jobs(c->sc, c->cd, P, ring_desc(out, 0, 0), s));
+  return move(c, nullptr, 1, s, wire, true);
 }
 
 }  // extern "C"

@@ -157,7 +157,9 @@ struct EncJobParam {
   Job jobs[2];
   Piece pieces[kMaxPieces];
 };
-cudaError_t launch_put_enc_jobs(Scratch& sc, const EncJobParam& p, const RingDesc& out, cudaStream_t s);
+// One job (n_jobs == 1) is planned in place: the mover follows directly (launch_plan_and_move planned=true).
+cudaError_t launch_put_enc_jobs(Scratch& sc, const ConfigDev& cfg, const EncJobParam& p, const RingDesc& out,
+                                cudaStream_t s);
 cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const uint32_t* xids,
                                   const void* const* srcs, const uint64_t* bytes, const int32_t* errs,
                                   const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
@@ -168,8 +170,10 @@ cudaError_t launch_replies_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, c
                                 cudaStream_t s);
 // Plans tiles for jobs [0, n_jobs) (n_jobs from counters[1] <= max_jobs_bound) and runs the mover.
 // out_bytes_bound (0 = unknown) caps the mover grid for small requests.
+// planned: the jobs' tile prefix and cursors were already written (single-request kernels).
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
-                                 uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s);
+                                 uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s,
+                                 bool planned = false);
 int mover_occupancy(uint32_t tile_bytes, uint32_t stages);
 cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
                          cudaStream_t s);

@@ -637,12 +637,13 @@ uint32_t mover_smem_bytes(uint32_t tile_bytes, uint32_t kStages) {
 }
 
 cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t max_jobs_bound,
-                                 uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s) {
+                                 uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s, bool planned) {
   uint64_t* tiles = sc.scan_tmp;  // [max_jobs + 1]
   uint64_t* total = sc.scan_tmp + sc.max_jobs + 1;
   const uint32_t* n_jobs_dev = sc.counters + 1;
   cudaError_t e;
-  if (max_jobs_bound <= kSmallJobs) {
+  if (planned) {
+  } else if (max_jobs_bound <= kSmallJobs) {
     plan_small_kernel<<<1, 256, 0, s>>>(sc, cfg, tiles, total, n_jobs_dev);
     count_launch();
     if ((e = cudaGetLastError()) != cudaSuccess) return e;

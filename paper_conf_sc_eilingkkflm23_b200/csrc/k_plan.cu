@@ -41,6 +41,7 @@ __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint3
     sc.jobs[i] = job;
     *st_out = st;
     if (cp_out) *cp_out = m;
+    if (use_single) plan_single_job(sc, cfg, job);  // n == 1: no planning launch
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
 }
@@ -71,6 +72,7 @@ __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uin
     sc.jobs[i] = job;
     *r.status = st;
     if (r.count) *r.count = cnt;
+    if (use_single) plan_single_job(sc, cfg, job);  // n == 1: no planning launch
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
 }
@@ -123,12 +125,13 @@ __global__ void __launch_bounds__(kSmallServe) serve_plan_small_kernel(IndexDev 
   TL_END(cfg, TL_PLAN);
 }
 
-__global__ void put_enc_jobs_kernel(Scratch sc, EncJobParam p, RingDesc out) {
+__global__ void put_enc_jobs_kernel(Scratch sc, ConfigDev cfg, EncJobParam p, RingDesc out) {
   if (threadIdx.x == 0) {
     for (uint32_t j = 0; j < p.n_jobs; ++j) sc.jobs[j] = p.jobs[j];
     sc.out_rings[0] = out;
     sc.counters[1] = p.n_jobs;
     sc.counters[4] = p.n_jobs;
+    if (p.n_jobs == 1) plan_single_job(sc, cfg, p.jobs[0]);  // no planning launch
   }
   for (uint32_t i = threadIdx.x; i < p.n_pieces; i += blockDim.x) sc.pieces[i] = p.pieces[i];
 }
@@ -345,8 +348,9 @@ cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Sc
   return cudaGetLastError();
 }
 
-cudaError_t launch_put_enc_jobs(Scratch& sc, const EncJobParam& p, const RingDesc& out, cudaStream_t s) {
-  put_enc_jobs_kernel<<<1, 64, 0, s>>>(sc, p, out);
+cudaError_t launch_put_enc_jobs(Scratch& sc, const ConfigDev& cfg, const EncJobParam& p, const RingDesc& out,
+                                cudaStream_t s) {
+  put_enc_jobs_kernel<<<1, 64, 0, s>>>(sc, cfg, p, out);
   count_launch();
   return cudaGetLastError();
 }

@@ -128,6 +128,19 @@ __device__ __forceinline__ Job serve_reply_job(const IndexDev& ix, const ConfigD
   return job;
 }
 
+// The mover plan of a single job, written by the thread that built it (single-request calls skip the
+// separate planning launch): tile prefix [0] = 0, total tiles, queue cursors reset.
+__device__ __forceinline__ void plan_single_job(const Scratch& sc, const ConfigDev& cfg, const Job& j) {
+  const uint64_t t = (j.type == JOB_NONE || j.out_end <= j.out_start)
+                         ? 0 : ((j.out_end - 1) >> cfg.tile_shift) - (j.out_start >> cfg.tile_shift) + 1;
+  sc.scan_tmp[0] = 0;
+  sc.scan_tmp[sc.max_jobs + 1] = t;
+  sc.counters[0] = 0;
+  sc.counters[2] = 0;
+  sc.counters[3] = 0;
+  sc.counters[6] = 0;
+}
+
 struct SendRingsParam {
   uint32_t n_rings;
   RingDesc r[kMaxRings];

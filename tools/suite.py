@@ -95,6 +95,20 @@ def c1(ctx):
 
     lat_ms = timed(one, 200)
     ok = bool(torch.equal(dst, data) and torch.equal(out, ints) and (st == 0).all())
+    # the same three calls captured once as a CUDA graph and replayed: device-side latency without the
+    # Python / ctypes issue cost of the loop above (which bounds it when launches are this short)
+    g = torch.cuda.CUDAGraph()
+    cs = torch.cuda.Stream()
+    cs.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(cs):
+        one(0)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=cs):
+            one(0)
+    torch.cuda.current_stream().wait_stream(cs)
+    dst.zero_(); out.zero_(); st.fill_(-1)
+    lat_graph_ms = timed(lambda _: g.replay(), 200)
+    ok &= bool(torch.equal(dst, data) and torch.equal(out, ints) and (st == 0).all())
     # 131,072 back-to-back records
     n = 131072
     big = crk.Ring.device(next_pow2(n * w + 4096))
@@ -124,7 +138,7 @@ def c1(ctx):
 
     bms = timed(batch, 5, warm=1)
     ok2 = bool((sts == 0).all() and torch.equal(dsts[n - 1], data) and torch.equal(outs[12345], ints))
-    return {"latency_us": round(lat_ms * 1e3, 2), "ok": ok,
+    return {"latency_us": round(lat_ms * 1e3, 2), "latency_graph_us": round(lat_graph_ms * 1e3, 2), "ok": ok,
             "note": "one record: crk_rpc_frame_scan (scan+parse) + crk_xdr_decode_opaque + crk_xdr_decode_array_i32",
             "batch_records": n, "batch_ms": round(bms, 3), "records_per_s": round(n / bms * 1e3),
             "batch_payload_gbs": round(n * 8192 / bms / 1e6, 1), "batch_ok": ok2}
