@@ -129,3 +129,50 @@ def test_server_capacity_limits():
     ring, send = crk.Ring.device(1 << 12), crk.Ring.device(1 << 12)
     with pytest.raises(crk.CrkError):
         crk.Server(ctx.index(1, 1 << 12, 2048), [ring], [send], 0, 0)  # > 1024 records
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_serve_steps_across_the_wrap_match_oracle(fused):
+    """The same multi-step stream through crk_serve launches (windows and send cursors crossing the ring
+    wrap, error records, a truncated window), with the separate scan / parse / plan kernels and with the
+    fused single-CTA front end."""
+    F = 4096
+    cfg = ocfg(F=F, user={33: [O.K_U32, O.K_I32_VAR]})
+    ctx = ctx_for(cfg, fused_front_max_records=1024 if fused else 0, fused_front_max_window=1 << 30)
+    n_rings, cap, scap = 3, 1 << 18, 1 << 18
+    region_bytes = 1 << 20
+    region = torch.zeros(region_bytes, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    g = gen.rng(0x5F)
+    host_region = gen.random_bytes(0x5F5F, region_bytes).copy()
+    region.copy_(torch.from_numpy(host_region))
+    rings = [crk.Ring.device(cap) for _ in range(n_rings)]
+    sends = [crk.Ring.device(scap) for _ in range(n_rings)]
+    idx = ctx.index(n_rings, 1 << 12, 3 * 64)
+    tails = [cap - 5000 + 97 * r for r in range(n_rings)]
+    send_offs = [scap - 3000 + 11 * r for r in range(n_rings)]
+    for step in range(8):
+        heads = list(tails)
+        for r in range(n_rings):
+            w = batch(g, step, r, base, region_bytes, host_region, cfg, F)
+            rings[r].write(tails[r], w)
+            tails[r] += len(w)
+        if step == 5:
+            tails[1] -= 3
+        before = [ring_bytes(r) for r in rings]
+        idx.serve([(rg, h, t) for rg, h, t in zip(rings, heads, tails)], sends, send_offs, base, region_bytes)
+        torch.cuda.synchronize()
+        want = O.serve([(b, h, t) for b, h, t in zip(before, heads, tails)], cfg, host_region, base,
+                       [scap] * n_rings, send_offs, max_frags_per_ring=(1 << 12) // n_rings, max_records_per_ring=64)
+        res = idx.ring_results(n_rings)
+        for r in range(n_rings):
+            assert res[r]["status"] == want["scan_status"][r], (step, r, res[r])
+            assert res[r]["consumed"] == want["consumed"][r], (step, r)
+            assert res[r]["reply_bytes"] == want["reply_bytes"][r], (step, r)
+            n = want["reply_bytes"][r]
+            exp = bytes(np.roll(want["send"][r], -(send_offs[r] % scap))[:n])
+            assert sends[r].read(send_offs[r], n) == exp, (step, r)
+        assert np.array_equal(region.cpu().numpy(), host_region), step
+        for r in range(n_rings):
+            tails[r] = want["consumed"][r] if step == 5 and r == 1 else tails[r]
+            send_offs[r] += want["reply_bytes"][r]
