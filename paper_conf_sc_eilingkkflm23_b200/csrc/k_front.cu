@@ -77,7 +77,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   }
   __syncthreads();
   // ---- serve planning: statuses, reply offsets, jobs, their tile prefix, mover cursors
-  plan_small_block(ix, P.cfg, P.sc, P.send, P.region_base, P.region_bytes, warp_sums, ring_first_pre);
+  plan_small_block(ix, P.cfg, P.sc, P.send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix);
   TL_END(P.cfg, TL_FUSED);
 }
 

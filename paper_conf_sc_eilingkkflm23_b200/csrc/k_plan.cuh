@@ -172,11 +172,13 @@ __device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_su
 // Small batches (<= kSmallServe records): statuses, reply offsets, decode and encode jobs, their tile
 // prefix and the mover cursors, by one block of kSmallServe threads (thread d owns record d).
 // warp_sums (32) and ring_first_pre (kMaxRings) are the block's shared scratch.  Used by the
-// single-block planning kernel and by the persistent server.
+// single-block planning kernel, the fused front end and the persistent server; the latter two pass the
+// dense record prefix they already hold in shared memory (prefix_s, n_rings + 1 entries), which saves the
+// dependent loads of the record total and of each record's ring bounds.
 __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
                                  uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
-                                 uint64_t* ring_first_pre) {
-  const uint32_t total = *ix.total;
+                                 uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr) {
+  const uint32_t total = prefix_s ? prefix_s[S.n_rings] : *ix.total;
   const uint32_t d = threadIdx.x;
   for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
   int st = CRK_OK;
@@ -187,8 +189,8 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   if (d < total) {
     ring = ix.p_ring[d];
     serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
-    first = ix.rec_prefix[ring];
-    end = ix.rec_prefix[ring + 1];
+    first = prefix_s ? prefix_s[ring] : ix.rec_prefix[ring];
+    end = prefix_s ? prefix_s[ring + 1] : ix.rec_prefix[ring + 1];
     w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   }
   uint64_t tot;

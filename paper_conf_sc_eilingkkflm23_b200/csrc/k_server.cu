@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     TL_END(P.cfg, 2);
     if (threadIdx.x == 0) B->t_phase_ns[2] = gtimer();
     // ---- serve planning (statuses, reply offsets, jobs)
-    plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre);
+    plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix);
     phase_sync();
     TL_END(P.cfg, 3);
     if (threadIdx.x == 0) B->t_phase_ns[3] = gtimer();
