@@ -308,7 +308,10 @@ def copy_to_host(dev_ptr: int, nbytes: int) -> np.ndarray:
 def config(**kw) -> Config:
     c = Config()
     lib().crk_config_init(C.byref(c))
+    names = {f for f, _ in Config._fields_}
     for k, v in kw.items():
+        if k not in names:  # a ctypes Structure would silently keep a misspelt field as a Python attribute
+            raise KeyError(f"crk_config has no field {k!r}")
         setattr(c, k, v)
     return c
 

@@ -116,3 +116,9 @@ def test_ctypes_layouts_match_the_header(tmp_path):
         assert got[(cname, "size")] == C.sizeof(py), cname
         for f, _ in py._fields_:
             assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
+
+
+def test_config_rejects_unknown_fields(L):
+    with pytest.raises(KeyError):
+        crk.config(mover_reserve=16)  # misspelt: the field is mover_reserve_ctas
+    assert crk.config(mover_reserve_ctas=16).mover_reserve_ctas == 16
