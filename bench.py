@@ -316,6 +316,7 @@ def main():
         # CTAs retire staggered, handing SMs over to the next mover gradually)
         ctx_kw.setdefault("mover_reserve_ctas", 16)
         ctx_kw.setdefault("mover_tail_tiles", 0)
+        ctx_kw.setdefault("mover_run", 32)  # 1 MiB claims: fewer job / fragment-window loads per byte
     stream = torch.cuda.current_stream(dev)
     slots = []
     for i in range(P):
@@ -549,7 +550,7 @@ def main():
                                          "frac": round(alg_bytes / (ms_max / 1e3) / 1e9 / hbm_peak, 4),
                                          "how": "mover algorithmic bytes per step / ms_per_step of the pipelined "
                                                 "timed region (a lower bound: the step also holds scan/parse/plan)"},
-                     "mover_config": {k: ctx_kw.get(k) for k in ("mover_reserve_ctas", "mover_tail_tiles")}},
+                     "mover_config": {k: ctx_kw.get(k) for k in ("mover_reserve_ctas", "mover_tail_tiles", "mover_run")}},
         "wire_gbs": round(sum_over_ranks(ep.wire_in + ep.reply_wire) / (ms_max / 1e3) / 1e9, 2),
         "pipeline": P, "serial_ms_per_step": round(serial_ms, 4),
         "serial_value": round(payload_all / (serial_ms / 1e3) / 1e9, 2),
