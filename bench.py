@@ -49,6 +49,8 @@ def parse_args():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
     p.add_argument("--ctx", default="", help="crk_config overrides, e.g. scan_threads=128,tile_bytes=32768")
+    p.add_argument("--direction", default="mixed", choices=["mixed", "h2d", "d2h"],
+                   help="C5 call mix: 50/50 (default), HtoD-only or DtoH-only memcpys")
     return p.parse_args()
 
 
@@ -261,9 +263,14 @@ def run_reference(args):
         "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
 
 
+H2D_FRAC = {"mixed": 0.5, "h2d": 1.0, "d2h": 0.0}
+
+
 def workload_config(args):
+    mix = {"mixed": "50/50 HtoD/DtoH", "h2d": "HtoD only", "d2h": "DtoH only"}[args.direction]
     return {"workload": f"C5 endpoint per GPU: {args.streams} client streams x {args.payload_mib} MiB memcpy payload "
-                        f"(ONC RPC CALLs, sizes log-uniform 4 KiB-16 MiB, 50/50 HtoD/DtoH, F=64 KiB fragments)",
+                        f"(ONC RPC CALLs, sizes log-uniform 4 KiB-16 MiB, {mix}, F=64 KiB fragments)",
+            "direction": args.direction,
             "streams_per_gpu": args.streams, "payload_per_gpu_bytes": args.streams * args.payload_mib * MiB,
             "frag_payload": 65536, "l2": "inputs larger than L2 (rings + region > 2 GiB per GPU)",
             "parallelism": f"{args.gpus} independent endpoints, no collective"}
@@ -322,7 +329,7 @@ def main():
     for i in range(P):
         ctx_i = crk.Context(local, **ctx_kw)
         ep_i = workload.c5_endpoint(ctx_i, rank, dev, n_streams=args.streams,
-                                    payload_per_stream=args.payload_mib * MiB)
+                                    payload_per_stream=args.payload_mib * MiB, h2d_frac=H2D_FRAC[args.direction])
         idx_i = ctx_i.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
         slots.append(workload.Slot(ctx_i, idx_i, ep_i, torch.cuda.Stream(dev) if P > 1 else stream))
     ep = slots[0].ep
@@ -406,7 +413,8 @@ def main():
         hslots = []
         for i in range(P):
             ep_i = workload.c5_endpoint(ctxs[i], rank, dev, n_streams=args.streams,
-                                        payload_per_stream=args.payload_mib * MiB, host_rings=True, staged=True)
+                                        payload_per_stream=args.payload_mib * MiB, host_rings=True, staged=True,
+                                        h2d_frac=H2D_FRAC[args.direction])
             idx_i = ctxs[i].index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
             hslots.append(workload.Slot(ctxs[i], idx_i, ep_i, torch.cuda.Stream(dev) if P > 1 else stream))
             hslots[-1].res = crk.PinnedResults(args.streams)

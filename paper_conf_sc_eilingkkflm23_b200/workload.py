@@ -52,10 +52,12 @@ class Endpoint:
 
 def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: int = 16,
                 payload_per_stream: int = 64 * MiB, host_rings: bool = False, misalign: bool = False,
-                staged: bool = False) -> Endpoint:
+                staged: bool = False, h2d_frac: float = 0.5) -> Endpoint:
+    """h2d_frac: share of HtoD calls (0.5 = the mixed 50/50 stream; 1.0 / 0.0 = HtoD-only / DtoH-only,
+    SURVEY.md §8(d) C5's three directions)."""
+    budget = payload_per_stream if h2d_frac >= 1.0 else payload_per_stream - payload_per_stream // 16
     streams, region_bytes = gen.c5_endpoint(rank, n_streams=n_streams, payload_per_stream=payload_per_stream,
-                                            h2d_budget=payload_per_stream - payload_per_stream // 16,
-                                            misalign=misalign)
+                                            h2d_budget=budget, misalign=misalign, h2d_frac=h2d_frac)
     region = torch.zeros(region_bytes + 256, dtype=torch.uint8, device=device)
     ep = Endpoint(ctx, rank, streams, region)
     F = ctx.cfg.frag_payload
