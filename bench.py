@@ -45,6 +45,7 @@ def parse_args():
     p.add_argument("--e2e-steps", type=int, default=100)
     p.add_argument("--pipeline", type=int, default=3, help="batches in flight (server loop slots)")
     p.add_argument("--e2e-pipeline", type=int, default=3, help="batches in flight for the host-memory runs")
+    p.add_argument("--e2e-copy-streams", type=int, default=1, help="streams per direction for the staged ring DMAs")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -422,6 +423,8 @@ def main():
 
         for s in hslots:  # inbound and outbound DMA get their own streams so the two directions never
             s.in_stream, s.out_stream = torch.cuda.Stream(dev), torch.cuda.Stream(dev)  # wait on each other
+            s.in_aux = [torch.cuda.Stream(dev) for _ in range(args.e2e_copy_streams - 1)]
+            s.out_aux = [torch.cuda.Stream(dev) for _ in range(args.e2e_copy_streams - 1)]
             s.ev_in, s.ev_served, s.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
             s.ev_out.record(s.out_stream)
             s.ev_served.record(s.stream)
@@ -435,7 +438,7 @@ def main():
             for k in range(n_steps):
                 s = hslots[k % P]
                 s.in_stream.wait_event(s.ev_served)
-                workload.staged_in(s.ep, s.in_stream)
+                workload.staged_in(s.ep, s.in_stream, s.in_aux)
                 s.ev_in.record(s.in_stream)
                 s.stream.wait_event(s.ev_in)
                 s.stream.wait_event(s.ev_out)
@@ -446,12 +449,12 @@ def main():
                     ps = pend.pop(0)
                     ps.ev_served.synchronize()
                     ps.out_stream.wait_event(ps.ev_served)
-                    workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream)
+                    workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream, ps.out_aux)
                     ps.ev_out.record(ps.out_stream)
             for ps in pend:
                 ps.ev_served.synchronize()
                 ps.out_stream.wait_event(ps.ev_served)
-                workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream)
+                workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream, ps.out_aux)
                 ps.ev_out.record(ps.out_stream)
             torch.cuda.synchronize()
 

@@ -133,10 +133,31 @@ def staged_in_and_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResult
     staged_serve(idx, ep, results, stream)
 
 
-def staged_in(ep: Endpoint, stream):
-    """DMA each host receive window into its device ring."""
-    for (hr, h, t), dr in zip(ep.rings, ep.dev_rings):
-        crk.ring_copy(dr, hr, h, t, stream=stream)
+def _fan_out(stream, aux):
+    """Streams for a step's ring copies: `stream` plus the auxiliary streams, which start after
+    everything already queued on `stream`."""
+    if not aux:
+        return [stream]
+    ev = torch.cuda.Event()
+    ev.record(stream)
+    for a in aux:
+        a.wait_event(ev)
+    return [stream] + list(aux)
+
+
+def _fan_in(stream, aux):
+    for a in aux or ():
+        ev = torch.cuda.Event()
+        ev.record(a)
+        stream.wait_event(ev)
+
+
+def staged_in(ep: Endpoint, stream, aux=None):
+    """DMA each host receive window into its device ring (ring r on streams[r % n] with aux streams)."""
+    ss = _fan_out(stream, aux)
+    for r, ((hr, h, t), dr) in enumerate(zip(ep.rings, ep.dev_rings)):
+        crk.ring_copy(dr, hr, h, t, stream=ss[r % len(ss)])
+    _fan_in(stream, aux)
 
 
 def staged_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResults", stream):
@@ -146,12 +167,14 @@ def staged_serve(idx: crk.Index, ep: Endpoint, results: "crk.PinnedResults", str
     idx.ring_results_async(results, stream=stream)
 
 
-def staged_out(ep: Endpoint, rows: list, stream):
+def staged_out(ep: Endpoint, rows: list, stream, aux=None):
     """Second half: DMA each ring's reply bytes (now known on the host) back to the host send ring."""
+    ss = _fan_out(stream, aux)
     for r, (hs, ds, off) in enumerate(zip(ep.sends, ep.dev_sends, ep.offs)):
         n = rows[r]["reply_bytes"]
         if n:
-            crk.ring_copy(hs, ds, off, off + n, stream=stream)
+            crk.ring_copy(hs, ds, off, off + n, stream=ss[r % len(ss)])
+    _fan_in(stream, aux)
 
 
 def check_results(idx: crk.Index, ep: Endpoint) -> dict:
