@@ -44,3 +44,35 @@ def test_bind_numa_without_node_leaves_affinity(tmp_path, monkeypatch):
     (d / "numa_node").write_text("-1\n")
     assert P.bind_numa(0, sysfs=str(tmp_path))["numa_node"] == -1
     assert os.sched_getaffinity(0) == before
+
+
+def test_bench_defaults_meet_the_timing_contract(monkeypatch):
+    """bench.py with no flags: N=1, >= 3 warm-up steps, the C5 mixed workload, inputs beyond L2."""
+    import sys
+    import bench
+    monkeypatch.setattr(sys, "argv", ["bench.py"])
+    a = bench.parse_args()
+    assert a.gpus == 1 and a.warmup >= 3 and a.steps >= 10 and a.impl == "crk" and a.direction == "mixed"
+    cfg = bench.workload_config(a)
+    assert cfg["direction"] == "mixed" and "50/50" in cfg["workload"] and "L2" in cfg["l2"]
+    assert cfg["payload_per_gpu_bytes"] == 16 * 64 * (1 << 20)
+    assert bench.H2D_FRAC == {"mixed": 0.5, "h2d": 1.0, "d2h": 0.0}
+
+
+def test_c5_direction_mixes():
+    """gen.c5_endpoint's call mix: h2d_frac 1 / 0 gives HtoD-only / DtoH-only streams; 0.5 keeps the
+    default draws (the mixed stream is the same whatever the other mixes do)."""
+    from paper_conf_sc_eilingkkflm23_b200 import gen
+    MiB = 1 << 20
+    only_h, _ = gen.c5_endpoint(0, n_streams=2, payload_per_stream=8 * MiB, h2d_budget=8 * MiB, h2d_frac=1.0)
+    only_d, _ = gen.c5_endpoint(0, n_streams=2, payload_per_stream=8 * MiB, h2d_frac=0.0)
+    mixed, _ = gen.c5_endpoint(0, n_streams=2, payload_per_stream=8 * MiB)
+    mixed2, _ = gen.c5_endpoint(0, n_streams=2, payload_per_stream=8 * MiB, h2d_frac=0.5)
+    assert all(r.kind == gen.PROC_H2D for s in only_h for r in s.records)
+    assert all(r.kind == gen.PROC_D2H for s in only_d for r in s.records)
+    kinds = {r.kind for s in mixed for r in s.records}
+    assert kinds == {gen.PROC_H2D, gen.PROC_D2H}
+    assert [(r.kind, r.size, r.xid) for s in mixed for r in s.records] == \
+           [(r.kind, r.size, r.xid) for s in mixed2 for r in s.records]
+    for streams in (only_h, only_d, mixed):
+        assert all(sum(r.size for r in s.records) == 8 * MiB for s in streams)
