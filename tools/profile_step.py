@@ -25,10 +25,11 @@ def main():
     ap.add_argument("--host", action="store_true")
     ap.add_argument("--streams", type=int, default=16)
     ap.add_argument("--payload-mib", type=int, default=64)
+    ap.add_argument("--ctx", default="", help="crk_config overrides, e.g. mover_run=32,mover_reserve_ctas=16")
     a = ap.parse_args()
     build.build()
     dev = torch.device("cuda:0")
-    ctx = crk.Context(0)
+    ctx = crk.Context(0, **{k: int(v, 0) for k, v in (kv.split("=") for kv in a.ctx.split(",") if kv)})
     ep = workload.c5_endpoint(ctx, 0, dev, n_streams=a.streams, payload_per_stream=a.payload_mib << 20,
                               host_rings=a.host)
     idx = ctx.index(max_rings=a.streams, max_frags=1 << 20, max_records=1 << 14)
