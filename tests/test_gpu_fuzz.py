@@ -52,10 +52,12 @@ def mutate(g, wires):
     return bytes(w)
 
 
-@pytest.mark.parametrize("strict", [True, False])
-def test_mutated_streams_match_oracle(strict):
+@pytest.mark.parametrize("strict,fused", [(True, False), (False, False), (True, True), (False, True)])
+def test_mutated_streams_match_oracle(strict, fused):
+    """fused: the same batches through the single-CTA fused front end (scan + parse + plan in one launch)."""
     cfg = ocfg(strict=strict, F=1024, user={40: [O.K_U32, O.K_OPAQUE_VAR]})
-    ctx = ctx_for(cfg, max_record_bytes=1 << 14)
+    ctx = ctx_for(cfg, max_record_bytes=1 << 14, fused_front_max_records=1024 if fused else 0,
+                  fused_front_max_window=1 << 30)
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
     g = gen.rng(2024 + strict)
