@@ -324,7 +324,6 @@ def main():
         # CTAs retire staggered, handing SMs over to the next mover gradually)
         ctx_kw.setdefault("mover_reserve_ctas", 16)
         ctx_kw.setdefault("mover_tail_tiles", 0)
-        ctx_kw.setdefault("mover_run", 32)  # 1 MiB claims: fewer job / fragment-window loads per byte
     stream = torch.cuda.current_stream(dev)
     slots = []
     for i in range(P):

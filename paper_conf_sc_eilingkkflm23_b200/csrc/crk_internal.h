@@ -82,15 +82,15 @@ struct Job {              // 64 bytes
   uint32_t type;          // JOB_*
   uint32_t esize;         // DEC: element size
   uint32_t rec;           // DEC: dense record id
-  uint32_t n_pieces;      // ENC
+  uint32_t n_pieces;      // ENC: pieces; DEC: the record's fragment count
   uint64_t out_start;     // DEC: dst address; ENC: out-ring cursor of the record's first header byte
   uint64_t out_end;       // exclusive (DEC: dst + nbytes; ENC: out_start + wire size)
   uint64_t loff;          // DEC: logical offset of the first byte; ENC: logical length of the record
-  uint32_t piece0;        // ENC: first piece in the piece pool
-  uint32_t F;             // ENC: fragment payload (0 -> explicit fragment table)
+  uint32_t piece0;        // ENC: first piece in the piece pool; DEC: the record's first fragment (absolute)
+  uint32_t F;             // ENC: fragment payload (0 -> explicit fragment table); DEC: first fragment's length
   uint32_t lens0;         // ENC with explicit framing: first entry in the lens / wire-start pool
   uint32_t n_lens;
-  uint32_t out_ring;      // ENC: index into the out-ring table
+  uint32_t out_ring;      // ENC: index into the out-ring table; DEC: the record's ring
   uint32_t pad_;
 };
 

@@ -161,7 +161,8 @@ struct ProdCache {
 };
 
 // Loads job j (and its pieces / ring / record) into the producer cache; the whole warp calls it.
-__device__ __forceinline__ void producer_load_job(ProdCache& pc, const MoveParams& M, uint32_t j, uint32_t lane) {
+__device__ __forceinline__ void producer_load_job(ProdCache& pc, const MoveParams& M, uint32_t j, uint32_t lane,
+                                                  const RingDesc* ring_s) {
   if (lane < sizeof(Job) / 4)
     reinterpret_cast<uint32_t*>(&pc.job)[lane] = reinterpret_cast<const uint32_t*>(M.sc.jobs + j)[lane];
   __syncwarp();
@@ -170,13 +171,11 @@ __device__ __forceinline__ void producer_load_job(ProdCache& pc, const MoveParam
     for (uint32_t i = lane; i < J.n_pieces * (sizeof(Piece) / 4); i += 32)
       reinterpret_cast<uint32_t*>(pc.pieces)[i] = reinterpret_cast<const uint32_t*>(M.sc.pieces + J.piece0)[i];
     if (lane == 0) pc.R = M.sc.out_rings[J.out_ring];
-  } else if (J.type == JOB_DEC && lane == 0) {
-    const uint32_t slot = M.ix.p_slot[J.rec], ring = M.ix.p_ring[J.rec];
-    pc.R = M.ix.rings[ring];
-    pc.frag0 = M.ix.rec_frag0[slot];
-    pc.nfrags = M.ix.rec_nfrags[slot];
-    pc.rec_len = M.ix.rec_len[slot];
-    pc.F0 = M.ix.frag_hdr[pc.frag0] & 0x7fffffffu;
+  } else if (J.type == JOB_DEC && lane == 0) {  // the record's coordinates travel in the job (dec_job)
+    pc.R = ring_s[J.out_ring];
+    pc.frag0 = J.piece0;
+    pc.nfrags = J.n_pieces;
+    pc.F0 = J.F;
     pc.wn = 0;
     pc.hint = 0;
   }
@@ -198,6 +197,23 @@ __device__ __forceinline__ void producer_frag(const ProdCache& pc, const MovePar
 // the next kMaxSeg fragments.  The whole warp calls it; lane 0's answer is returned to every lane.
 __device__ uint32_t producer_frag_window(ProdCache& pc, const MoveParams& M, uint64_t off, uint32_t lane) {
   uint32_t k0 = 0;
+  if (pc.wn == 0 && pc.F0) {
+    // fresh job: fill the window around the uniform-stride guess in one round trip, so the search below
+    // runs from shared memory (greedy F framing puts offset off in fragment off / F0 exactly)
+    const uint32_t n = pc.nfrags;
+    const uint64_t gs = off / pc.F0;
+    const uint32_t g = gs < n ? (uint32_t)gs : n - 1;
+    const uint32_t base = g > 0 ? g - 1 : 0, cnt = min(kWin, n - base);
+    for (uint32_t i = lane; i < cnt; i += 32) {
+      const uint64_t q = (uint64_t)pc.frag0 + base + i;
+      pc.lstart[i] = M.ix.frag_lstart[q];
+      pc.phys[i] = M.ix.frag_phys[q];
+      pc.hdr[i] = M.ix.frag_hdr[q];
+    }
+    __syncwarp();
+    if (lane == 0) { pc.wk0 = base; pc.wn = cnt; pc.hint = g; }
+    __syncwarp();
+  }
   if (lane == 0) {
     auto holds = [&](uint32_t k) {
       uint64_t ls, ph;
@@ -295,6 +311,10 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
     // a window of kWin fragment entries is refilled by the whole warp in one round trip, so a tile's
     // descriptor costs no dependent global loads in the common case.
     __shared__ ProdCache pc;
+    __shared__ RingDesc ring_s[kMaxRings];  // the index's ring descriptors (decode jobs name their ring)
+    if (M.ix.rings)
+      for (uint32_t i = lane; i < M.ix.max_rings && i < (uint32_t)kMaxRings; i += 32) ring_s[i] = M.ix.rings[i];
+    __syncwarp();
     uint32_t k = 0, claims = 0;
     for (;;) {
       uint64_t t0 = ~0ull, t1 = 0;
@@ -340,7 +360,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
           pnext = j + 1 < n_jobs ? M.prefix[j + 1] : ~0ull;
           fresh = true;
         }
-        if (fresh) producer_load_job(pc, M, j, lane);
+        if (fresh) producer_load_job(pc, M, j, lane, ring_s);
         const Job& J = pc.job;
         const uint64_t t = tile - pj;
         const uint64_t A = J.out_start >> shf;

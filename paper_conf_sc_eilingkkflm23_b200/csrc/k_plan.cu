@@ -33,7 +33,7 @@ __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint3
         else {
           m = (cfg.strict || nb <= size) ? nb : size;
           if (cap < m) { st = CRK_E_PTR; m = 0; }
-          else job = dec_job(dst, m, ix.p_off[(uint64_t)d * kMaxItems + 1], d, 1);
+          else job = dec_job(ix, dst, m, ix.p_off[(uint64_t)d * kMaxItems + 1], d, 1);
         }
       }
     }
@@ -66,7 +66,7 @@ __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uin
         st = CRK_E_SIZE;
       } else {
         cnt = ix.p_count[b];
-        job = dec_job((uint64_t)r.dst, cnt * es, ix.p_off[b], d, es);
+        job = dec_job(ix, (uint64_t)r.dst, cnt * es, ix.p_off[b], d, es);
       }
     }
     sc.jobs[i] = job;

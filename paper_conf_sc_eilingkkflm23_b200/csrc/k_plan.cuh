@@ -36,7 +36,11 @@ __device__ __forceinline__ uint64_t wire_of(uint64_t Ll, uint32_t F) {
   return Ll + 4 * nfr;
 }
 
-__device__ __forceinline__ Job dec_job(uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec, uint32_t es) {
+// A decode job carries its record's fragment-table coordinates (first fragment, count, ring, first
+// fragment length), so the mover's producer resolves a fresh job with one load instead of a chain of
+// record-table loads.
+__device__ __forceinline__ Job dec_job(const IndexDev& ix, uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec,
+                                       uint32_t es) {
   Job j{};
   j.type = nbytes ? JOB_DEC : JOB_NONE;
   j.esize = es;
@@ -44,6 +48,14 @@ __device__ __forceinline__ Job dec_job(uint64_t dst, uint64_t nbytes, uint64_t l
   j.out_start = dst;
   j.out_end = dst + nbytes;
   j.loff = loff;
+  if (nbytes) {
+    const uint32_t slot = ix.p_slot[rec];
+    const uint32_t f0 = ix.rec_frag0[slot];
+    j.piece0 = f0;
+    j.n_pieces = ix.rec_nfrags[slot];
+    j.out_ring = ix.p_ring[rec];
+    j.F = ix.frag_hdr[f0] & 0x7fffffffu;
+  }
   return j;
 }
 
@@ -82,7 +94,7 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
     const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
     if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
     else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
-    else { err = 0; job = dec_job(ptr, m, o1, d, 1); }
+    else { err = 0; job = dec_job(ix, ptr, m, o1, d, 1); }
     Ll = 28;
   } else if (st == CRK_OK && proc == cfg.proc_d2h) {
     const uint64_t ptr = v0, size = v1;
