@@ -8,12 +8,16 @@ log-uniform 4 KiB-16 MiB, 50/50 HtoD/DtoH, 64 MiB of payload per stream = 1 GiB 
 sums (K2), CALL parse (K3), HtoD opaque scatter into device memory (K4) and DtoH reply encode into the
 send rings (K6), i.e. every §8(a) row the memcpy path has.
 
-  value : payload GB/s (1e9 B/s) with rings and send rings resident in HBM (inputs > L2: 1 GiB of rings)
-  e2e   : the same through the C ABI with the rings in pinned host memory (zero-copy over PCIe: the
-          kernels read the CALLs from host memory and write the replies to host memory) plus a
-          device->host read of the per-ring results every step
-  roofline: the mover kernel (K4/K6) against the measured HBM copy bandwidth
-  cpu_baseline: the oracle (oracle/, plain C, one core) on a bounded sample of the same workload
+  value : payload GB/s (1e9 B/s) with rings and send rings resident in HBM (inputs > L2: 1 GiB of rings),
+          3 batches in flight
+  e2e   : the same through the C ABI with the receive and send rings in pinned host memory, plus a
+          device->host read of the per-ring results every step; the fastest of three modes (copy-engine
+          staged, mixed, zero-copy), each measured, against the host link measured in the same run
+  roofline: the mover kernel (K4/K6) against the measured HBM copy bandwidth (per launch, and over the
+          timed region)
+  cpu_baseline: the oracle (oracle/, plain C) on a bounded sample of the same workload: one core, one
+          thread per core, and Cricket-style (pageable buffer + cudaMemcpy)
+  --direction h2d|d2h: the HtoD-only / DtoH-only call mixes of the same endpoint
 
 Launch: python bench.py [--gpus N --steps K --warmup W]; N > 1 under torch.distributed.run (one rank per
 GPU, NCCL only for the barrier and the max-over-ranks of the timings; the data path has no collective).
