@@ -316,9 +316,9 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   const size_t sz[] = {sizeof(Job) * (size_t)sc.max_jobs, sizeof(Piece) * (size_t)sc.max_pieces, 64,
                        sizeof(uint64_t) * 2 * (size_t)sc.max_lens, sizeof(uint32_t) * (size_t)sc.max_lens,
                        sizeof(unsigned long long) * scan_blocks, sizeof(uint64_t) * ((size_t)sc.max_jobs + 2),
-                       sizeof(RingDesc) * kMaxRings, sizeof(SchemaTable)};
-  size_t total = 0, off[9];
-  for (int i = 0; i < 9; ++i) { off[i] = total; total += (sz[i] + 255) & ~(size_t)255; }
+                       sizeof(RingDesc) * kMaxRings, sizeof(SchemaTable), sizeof(uint32_t) * (size_t)sc.max_jobs};
+  size_t total = 0, off[10];
+  for (int i = 0; i < 10; ++i) { off[i] = total; total += (sz[i] + 255) & ~(size_t)255; }
   cudaError_t e = cudaMalloc(&c->block, total);
   if (e != cudaSuccess) { delete c; return cuda_fail(e); }
   char* b = (char*)c->block;
@@ -331,6 +331,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   sc.scan_tmp = (uint64_t*)(b + off[6]);
   sc.out_rings = (RingDesc*)(b + off[7]);
   c->d_schemas = (SchemaTable*)(b + off[8]);
+  sc.run_job = (uint32_t*)(b + off[9]);
   e = cudaMemset(c->block, 0, total);
   if (e == cudaSuccess) e = cudaMemcpy(c->d_schemas, &c->host_schemas, sizeof(SchemaTable), cudaMemcpyHostToDevice);
   if (e != cudaSuccess) { cudaFree(c->block); delete c; return cuda_fail(e); }

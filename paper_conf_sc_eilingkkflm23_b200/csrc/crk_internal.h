@@ -98,12 +98,14 @@ struct Scratch {          // ctx-owned device scratch
   Job* jobs;              // [max_jobs]
   Piece* pieces;          // [2 * max_jobs]
   uint32_t* counters;     // [16]: 0/2 mover decode/encode run cursors, 3/6 their single-tile tail cursors, 1 n_jobs,
-                          // 4 queue split, 5 K2 block counter, 8/9 mover launch stamp (sequence, start time)
+                          // 4 queue split, 5 K2 block counter, 8/9 mover launch stamp (sequence, start time),
+                          // 12 queue-0 runs in run_job, 13 run_job valid for the next mover launch
   uint64_t* lens_pool;    // explicit framing: [2 * max_lens] (lens, then wire starts)
   uint32_t* lens32;       // [max_lens] staging for host-given fragment lengths
   unsigned long long* scan_state;  // decoupled look-back state for K2
   uint64_t* scan_tmp;     // [max_jobs + 2]: sizes -> prefix; [max_jobs + 1] = total
   RingDesc* out_rings;    // [kMaxRings]
+  uint32_t* run_job;      // [max_jobs]: the job holding each mover run's first tile (queue 0 runs, then queue 1)
   uint32_t max_jobs, max_lens, max_pieces;
   uint32_t mover_seq;     // host-side count of this context's mover launches (the launch stamp's sequence)
 };
@@ -176,7 +178,7 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
                                  bool planned = false);
 int mover_occupancy(uint32_t tile_bytes, uint32_t stages);
 cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
-                         cudaStream_t s);
+                         cudaStream_t s, bool use_map = false);
 // Serve planning for small batches (index max_records <= kSmallServe): statuses, reply offsets, decode
 // and encode jobs, their tile prefix and the mover cursors in one single-block kernel.
 constexpr uint32_t kSmallServe = 1024;

@@ -59,6 +59,7 @@ struct MoveParams {
   const uint64_t* total_tiles;
   uint32_t stage_bytes;    // bytes of one stage buffer (after its header)
   uint32_t seq;            // this launch's number (launch stamp)
+  uint32_t use_map;        // a run_map_kernel ran for this launch (counters[13] says whether its map applies)
   uint32_t opp_from;       // CTAs >= opp_from are opportunistic (crk_config.mover_reserve_ctas)
 };
 
@@ -303,6 +304,8 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
   // runs of cfg.run tiles amortise claims on big batches; a batch with fewer than two runs per CTA is
   // claimed tile by tile so it spreads over the grid
   const uint32_t kRun = total >= 2ull * gridDim.x * M.cfg.run ? M.cfg.run : 1u;
+  const bool map_ok = M.use_map && kRun > 1 && M.sc.counters[13] != 0;
+  const uint32_t map_r0 = map_ok ? M.sc.counters[12] : 0;
 
   if (warp == 0) {
     // ------------------------------------------------ producer
@@ -318,6 +321,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
     uint32_t k = 0, claims = 0;
     for (;;) {
       uint64_t t0 = ~0ull, t1 = 0;
+      uint32_t run_idx = ~0u;  // index of the claimed run in run_job (when the map applies)
       if (lane == 0) {
         const uint32_t pref = (claims + blockIdx.x) & 1;
         for (int tries = 0; tries < 2 && t0 == ~0ull; ++tries) {
@@ -329,9 +333,11 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
             const uint64_t tail = (uint64_t)M.cfg.tail * gridDim.x;
             const uint64_t cut = (kRun > 1 && hi - lo > tail) ? lo + (hi - lo - tail) / kRun * kRun : lo;
             uint64_t t = ~0ull;
-            if (cut > lo) t = lo + (uint64_t)kRun * atomicAdd(M.sc.counters + (q ? 2 : 0), 1u);
+            uint32_t ri = 0;
+            if (cut > lo) { ri = atomicAdd(M.sc.counters + (q ? 2 : 0), 1u); t = lo + (uint64_t)kRun * ri; }
             if (t < cut) {
               t0 = t; t1 = min(cut, t + kRun);
+              if (map_ok) run_idx = (q ? map_r0 : 0) + ri;
             } else {
               t = cut + atomicAdd(M.sc.counters + (q ? 6 : 3), 1u);
               if (t < hi) { t0 = t; t1 = t + 1; }
@@ -350,7 +356,15 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
         mbar_arrive(&full[s]);
         break;
       }
-      uint32_t j = find_job(M.prefix, n_jobs, t0, lane);
+      uint32_t j;
+      run_idx = __shfl_sync(0xffffffffu, run_idx, 0);
+      if (run_idx != ~0u) {  // the planner's run -> job map: one load instead of the prefix search
+        uint32_t jj = 0;
+        if (lane == 0) jj = M.sc.run_job[run_idx];
+        j = __shfl_sync(0xffffffffu, jj, 0);
+      } else {
+        j = find_job(M.prefix, n_jobs, t0, lane);
+      }
       uint64_t pj = M.prefix[j], pnext = j + 1 < n_jobs ? M.prefix[j + 1] : ~0ull;
       bool fresh = true;
       for (uint64_t tile = t0; tile < t1; ++tile, ++k) {
@@ -583,6 +597,40 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
   TL_END(M.cfg, TL_MOVE);
 }
 
+// The run -> job map of the next mover launch (grid CTAs, runs of `run` tiles, cfg.tail tail tiles per CTA):
+// the run boundaries are the mover's own (queue 0 = decode jobs from tile 0, queue 1 = encode jobs from the
+// split, runs up to the queue's single-tile tail region); each thread maps one run by binary search over
+// the tile prefix.  counters[12] = queue-0 run count, counters[13] = 1 when the map applies.
+__global__ void run_map_kernel(Scratch sc, ConfigDev cfg, uint32_t grid, uint32_t run, const uint64_t* prefix,
+                               const uint32_t* n_jobs_dev, const uint64_t* total_tiles) {
+  const uint64_t total = *total_tiles;
+  const uint32_t n_jobs = *n_jobs_dev;
+  const uint32_t n_split = sc.counters[4] < n_jobs ? sc.counters[4] : n_jobs;
+  const uint64_t split = n_split < n_jobs ? prefix[n_split] : total;
+  const uint32_t kRun = total >= 2ull * grid * run ? run : 1u;
+  const uint64_t tail = (uint64_t)cfg.tail * grid;
+  auto runs_of = [&](uint64_t lo, uint64_t hi) -> uint64_t {
+    const uint64_t cut = (kRun > 1 && hi - lo > tail) ? lo + (hi - lo - tail) / kRun * kRun : lo;
+    return (cut - lo) / kRun;
+  };
+  const uint64_t r0 = split > 0 ? runs_of(0, split) : 0, r1 = total > split ? runs_of(split, total) : 0;
+  const bool ok = kRun > 1 && r0 + r1 <= sc.max_jobs;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    sc.counters[12] = (uint32_t)r0;
+    sc.counters[13] = ok ? 1u : 0u;
+  }
+  if (!ok) return;
+  for (uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; r < r0 + r1; r += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t t = r < r0 ? r * kRun : split + (r - r0) * kRun;
+    uint32_t lo = 0, hi = n_jobs;  // last j with prefix[j] <= t (zero-tile jobs share a prefix value)
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (prefix[mid] <= t) lo = mid; else hi = mid;
+    }
+    sc.run_job[r] = lo;
+  }
+}
+
 // tiles per job: output range cut at tile_bytes-aligned boundaries
 __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, const uint32_t* n_jobs_dev) {
   const uint32_t n = *n_jobs_dev;
@@ -684,13 +732,20 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
       if (tiles_max < (uint64_t)move_ctas) move_ctas = (int)tiles_max;
     }
   }
-  return launch_mover(ix, cfg, sc, run, move_ctas, s);
+  bool use_map = false;
+  if (!planned && run > 1) {  // the run -> job map for this launch's run boundaries
+    run_map_kernel<<<(uint32_t)sms * 2, 256, 0, s>>>(sc, cfg, (uint32_t)move_ctas, run, tiles, n_jobs_dev, total);
+    count_launch();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    use_map = true;
+  }
+  return launch_mover(ix, cfg, sc, run, move_ctas, s, use_map);
 }
 
 // The mover over already-planned jobs: tile prefix in scan_tmp[0..n_jobs), total tiles at
 // scan_tmp[max_jobs + 1], job count in counters[1], queue split in counters[4], cursors reset.
 cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
-                         cudaStream_t s) {
+                         cudaStream_t s, bool use_map) {
   cudaError_t e;
   MoveParams M;
   if (ix) M.ix = *ix; else memset(&M.ix, 0, sizeof(M.ix));
@@ -702,6 +757,7 @@ cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, 
   M.total_tiles = sc.scan_tmp + sc.max_jobs + 1;
   M.stage_bytes = (1u << cfg.tile_shift) + 32 * kMaxSeg + 32;
   M.seq = ++sc.mover_seq;
+  M.use_map = use_map ? 1u : 0u;
   M.opp_from = (uint32_t)move_ctas > 2 * cfg.reserve ? (uint32_t)move_ctas - cfg.reserve : (uint32_t)move_ctas;
   const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
   static uint32_t smem_set = 0;  // dynamic shared memory opt-in (per process, grows monotonically)
