@@ -562,11 +562,15 @@ def test_encode_replies_batch_matches_oracle(host, F):
 
 MOVER_CONFIGS = [{}, {"mover_tail_tiles": 0, "mover_reserve_ctas": 16},
                  {"mover_tail_tiles": 64, "mover_run": 1, "tile_bytes": 4096}, {"mover_tail_tiles": 1, "mover_run": 64},
+                 # small tiles and short runs: the batch holds >= 2 runs per CTA, so run_map_kernel's run -> job
+                 # map drives the claims (with and without the single-tile tail region)
+                 {"tile_bytes": 4096, "mover_run": 2, "mover_tail_tiles": 0},
+                 {"tile_bytes": 4096, "mover_run": 2, "mover_tail_tiles": 1, "mover_reserve_ctas": 16},
                  # the fused single-CTA front end (scan + parse + plan in one launch) on the same batch
                  {"fused_front_max_records": 1024, "fused_front_max_window": 1 << 40}]
 
 
-@pytest.mark.parametrize("host,mover", [(False, m) for m in range(len(MOVER_CONFIGS))] + [(True, 0), (True, 4)])
+@pytest.mark.parametrize("host,mover", [(False, m) for m in range(len(MOVER_CONFIGS))] + [(True, 0), (True, 6)])
 def test_serve_matches_oracle(host, mover):
     cfg = ocfg(F=16384)
     ctx = ctx_for(cfg, **MOVER_CONFIGS[mover])
