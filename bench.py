@@ -321,37 +321,18 @@ def main():
     # A server loop keeps `pipeline` batches in flight: each slot is a (context, index, stream, batch
     # buffers) set, so the front end (scan / parse / plan) of batch k+1 runs while the mover of batch k
     # streams bytes.  Step k is served by slot k % pipeline; every step is one full pass over its batch.
+    # workload.run_pipelined / StagedLoop are the loops timed here; tests/test_gpu_bench_parity.py runs the
+    # same functions on the same configuration and compares every byte with the oracle.
     P = max(1, args.pipeline)
-    if P > 1:
-        # with batches in flight the mover leaves 16 CTA slots free, so the next batch's front-end
-        # kernels and the start of its mover overlap this one, and claims whole runs to the end (its
-        # CTAs retire staggered, handing SMs over to the next mover gradually)
-        ctx_kw.setdefault("mover_reserve_ctas", 16)
-        ctx_kw.setdefault("mover_tail_tiles", 0)
+    ctx_kw = workload.pipelined_ctx_kw(ctx_kw, P)
     stream = torch.cuda.current_stream(dev)
-    slots = []
-    for i in range(P):
-        ctx_i = crk.Context(local, **ctx_kw)
-        ep_i = workload.c5_endpoint(ctx_i, rank, dev, n_streams=args.streams,
-                                    payload_per_stream=args.payload_mib * MiB, h2d_frac=H2D_FRAC[args.direction])
-        idx_i = ctx_i.index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
-        slots.append(workload.Slot(ctx_i, idx_i, ep_i, torch.cuda.Stream(dev) if P > 1 else stream))
+    slots = workload.build_slots(local, rank, dev, P, ctx_kw, n_streams=args.streams,
+                                 payload_per_stream=args.payload_mib * MiB, h2d_frac=H2D_FRAC[args.direction],
+                                 default_stream=stream)
     ep = slots[0].ep
 
     def run(n_steps):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for s in slots:
-            s.stream.wait_event(e0)
-        for k in range(n_steps):
-            s = slots[k % P]
-            workload.serve_step(s.idx, s.ep, stream=s.stream)
-        for s in slots:
-            ev = torch.cuda.Event()
-            ev.record(s.stream)
-            stream.wait_event(ev)
-        e1.record(stream)
-        return e0, e1
+        return workload.run_pipelined(slots, stream, n_steps)
 
     # ---- device-resident timed region (value)
     run(max(args.warmup, P))
@@ -412,54 +393,12 @@ def main():
         # the same placement the rings get) and again after the runs; the roofline takes the better of the two
         link0 = host_link_peaks(dev)
         P = max(1, args.e2e_pipeline)  # batches in flight for the host-memory runs
-        while len(ctxs) < P:
-            ctxs.append(crk.Context(local, **ctx_kw))
-        hslots = []
-        for i in range(P):
-            ep_i = workload.c5_endpoint(ctxs[i], rank, dev, n_streams=args.streams,
-                                        payload_per_stream=args.payload_mib * MiB, host_rings=True, staged=True,
-                                        h2d_frac=H2D_FRAC[args.direction])
-            idx_i = ctxs[i].index(max_rings=args.streams, max_frags=1 << 20, max_records=1 << 14)
-            hslots.append(workload.Slot(ctxs[i], idx_i, ep_i, torch.cuda.Stream(dev) if P > 1 else stream))
-            hslots[-1].res = crk.PinnedResults(args.streams)
+        hslots = workload.build_slots(local, rank, dev, P, ctx_kw, n_streams=args.streams,
+                                      payload_per_stream=args.payload_mib * MiB, h2d_frac=H2D_FRAC[args.direction],
+                                      host_rings=True, staged=True, ctxs=ctxs, default_stream=stream)
         ep_h = hslots[0].ep
-
-        for s in hslots:  # inbound and outbound DMA get their own streams so the two directions never
-            s.in_stream, s.out_stream = torch.cuda.Stream(dev), torch.cuda.Stream(dev)  # wait on each other
-            s.in_aux = [torch.cuda.Stream(dev) for _ in range(args.e2e_copy_streams - 1)]
-            s.out_aux = [torch.cuda.Stream(dev) for _ in range(args.e2e_copy_streams - 1)]
-            s.ev_in, s.ev_served, s.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
-            s.ev_out.record(s.out_stream)
-            s.ev_served.record(s.stream)
-
-        def run_staged(n_steps):
-            # copy-engine mode, per slot: inbound DMA (in_stream, after the slot's previous serve has read
-            # its device rings) -> serve from HBM (stream, after the previous reply DMA has drained the
-            # device send rings) -> reply DMA (out_stream, queued by the host once the reply sizes are
-            # known).  Inbound DMA of later batches never waits behind a reply DMA.
-            pend = []
-            for k in range(n_steps):
-                s = hslots[k % P]
-                s.in_stream.wait_event(s.ev_served)
-                workload.staged_in(s.ep, s.in_stream, s.in_aux)
-                s.ev_in.record(s.in_stream)
-                s.stream.wait_event(s.ev_in)
-                s.stream.wait_event(s.ev_out)
-                workload.staged_serve(s.idx, s.ep, s.res, s.stream)
-                s.ev_served.record(s.stream)
-                pend.append(s)
-                if len(pend) >= P:
-                    ps = pend.pop(0)
-                    ps.ev_served.synchronize()
-                    ps.out_stream.wait_event(ps.ev_served)
-                    workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream, ps.out_aux)
-                    ps.ev_out.record(ps.out_stream)
-            for ps in pend:
-                ps.ev_served.synchronize()
-                ps.out_stream.wait_event(ps.ev_served)
-                workload.staged_out(ps.ep, ps.res.rows(), ps.out_stream, ps.out_aux)
-                ps.ev_out.record(ps.out_stream)
-            torch.cuda.synchronize()
+        loop = workload.StagedLoop(hslots, dev, args.e2e_copy_streams)
+        run_staged, run_mixed, run_e2e = loop.run, loop.run_mixed, loop.run_zero_copy
 
         run_staged(max(2, min(args.warmup, 4)))
         barrier()
@@ -473,40 +412,12 @@ def main():
             hslots[0].ep.sends[0].read(0, n0) == hslots[0].ep.dev_sends[0].read(0, n0))
         check_st["ok"] = check_st["ok"] and check_st["host_send_matches_device"]
 
-        def run_mixed(n_steps):
-            # copy engine in, SM zero-copy out: the inbound window is DMA'd into the device ring, the mover
-            # writes the replies straight into the pinned host send rings (no outbound DMA)
-            for k in range(n_steps):
-                s = hslots[k % P]
-                s.in_stream.wait_event(s.ev_served)
-                workload.staged_in(s.ep, s.in_stream)
-                s.ev_in.record(s.in_stream)
-                s.stream.wait_event(s.ev_in)
-                s.idx.serve([(dr, h, t) for dr, (_, h, t) in zip(s.ep.dev_rings, s.ep.rings)], s.ep.sends,
-                            s.ep.offs, s.ep.base, s.ep.region.numel(), stream=s.stream)
-                s.idx.ring_results_async(s.res, stream=s.stream)
-                s.ev_served.record(s.stream)
-            torch.cuda.synchronize()
-
         run_mixed(max(2, min(args.warmup, 4)))
         barrier()
         t0 = time.perf_counter()
         run_mixed(args.e2e_steps)
         el_mx = max_over_ranks(time.perf_counter() - t0)
         check_mx = workload.check_results(hslots[0].idx, ep_h)
-
-        def run_e2e(n_steps):
-            # step k is launched before the results of step k-1 are read back (device -> host, syncs
-            # that slot's stream), so the host read overlaps the next batch
-            for k in range(n_steps):
-                s = hslots[k % P]
-                workload.serve_step(s.idx, s.ep, stream=s.stream)
-                if k >= P - 1:
-                    p_ = hslots[(k - P + 1) % P]
-                    p_.idx.ring_results(len(p_.ep.rings), stream=p_.stream)
-            for k in range(max(0, n_steps - P + 1), n_steps):
-                p_ = hslots[k % P]
-                p_.idx.ring_results(len(p_.ep.rings), stream=p_.stream)
 
         run_e2e(max(2, min(args.warmup, 4)))
         barrier()

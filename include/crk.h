@@ -201,7 +201,8 @@ int crk_rpc_frame_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk
  * status_dev / copied_dev: dev int32 / uint64 slots (copied_dev may be NULL). */
 int crk_xdr_decode_memcpy_h2d(crk_ctx* ctx, crk_index* idx, uint32_t xid, void* dst, uint64_t dst_bytes,
                               int32_t* status_dev, uint64_t* copied_dev, crk_stream_t stream);
-/* n requests at once; xids, dsts, dst_bytes, statuses, copied are dev arrays of length n. */
+/* n requests at once; xids, dsts, dst_bytes, statuses, copied are dev arrays of length n.  A request whose
+ * checks pass but whose dst is NULL with a non-empty payload gets CRK_E_ARG (after E_PTR) and copies nothing. */
 int crk_xdr_decode_memcpy_h2d_batch(crk_ctx* ctx, crk_index* idx, uint32_t n, const uint32_t* xids,
                                     void* const* dsts, const uint64_t* dst_bytes, int32_t* statuses,
                                     uint64_t* copied, crk_stream_t stream);
@@ -226,7 +227,9 @@ int crk_xdr_decode_array_f64(crk_ctx*, crk_index*, uint32_t xid, uint32_t arg_no
 int crk_xdr_decode_opaque(crk_ctx*, crk_index*, uint32_t xid, uint32_t arg_no, void* dst, uint64_t max_count,
                           uint64_t* count_dev, int32_t* status_dev, crk_stream_t);
 
-/* Generic batch: one request per element (device array of n). */
+/* Generic batch: one request per element (device array of n).  Per-request checks in order: E_XID, wire
+ * status, E_ARG (arg_no / kind), E_SIZE (count > max_count), then E_ARG for a NULL dst with count > 0 or a
+ * dst not aligned to the element size (the single-request calls reject those synchronously). */
 typedef struct {
   uint32_t xid, arg_no, kind, pad_;
   void* dst;

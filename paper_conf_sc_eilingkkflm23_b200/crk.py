@@ -140,6 +140,7 @@ def lib():
             "crk_profile_enable": (C.c_int, [C.c_int]),
             "crk_profile_read": (C.c_int, [C.POINTER(C.c_double), C.POINTER(u32)]),
             "crk_version": (C.c_char_p, []),
+            "crk_debug_counters": (C.c_int, [vp, C.POINTER(u32)]),  # diagnostic, not in include/crk.h
         }
         for t in ("i32", "u32", "i64", "u64", "f32", "f64"):
             sig[f"crk_xdr_decode_array_{t}"] = (C.c_int, [vp, vp, u32, u32, vp, u64, vp, vp, vp])
@@ -340,6 +341,12 @@ class Context:
             self.close()
         except Exception:
             pass
+
+    def debug_counters(self) -> list[int]:
+        """Diagnostic: the context's 16 scratch counters (synchronises the device)."""
+        out = (C.c_uint32 * 16)()
+        _check(lib().crk_debug_counters(self.h, out), "crk_debug_counters")
+        return list(out)
 
     def register_schema(self, proc: int, items):
         arr = (u32 * max(1, len(items)))(*items)

@@ -818,6 +818,18 @@ void crk_graph_destroy(crk_graph* G) {
   delete G;
 }
 
+// Diagnostic (not in the public header): copies the context's 16 scratch counters (crk_internal.h Scratch::
+// counters) to host memory after synchronising the device; tests read counters[13] (the mover's run -> job
+// map applied) with it.
+extern "C" int crk_debug_counters(crk_ctx* c, uint32_t* host16) {
+  if (!c || !host16) return CRK_E_ARG;
+  DeviceGuard g(c->device);
+  if (cudaDeviceSynchronize() != cudaSuccess) return CRK_E_CUDA;
+  if (cudaMemcpy(host16, c->sc.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost) != cudaSuccess)
+    return CRK_E_CUDA;
+  return CRK_OK;
+}
+
 #ifdef CRK_TIMELINE
 // Diagnostic build only: kernels of this context stamp [min start, max end] per stage into dev_buf
 // (TL_STAGES x 2 u64, device memory; nullptr turns it off).

@@ -177,6 +177,8 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
                                  uint64_t out_bytes_bound, int sms, int move_ctas, cudaStream_t s,
                                  bool planned = false);
 int mover_occupancy(uint32_t tile_bytes, uint32_t stages);
+constexpr int kMaxDevices = 64;
+cudaError_t ensure_mover_smem(uint32_t smem);  // per-device dynamic shared memory opt-in, raise-only
 cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, uint32_t run, int move_ctas,
                          cudaStream_t s, bool use_map = false);
 // Serve planning for small batches (index max_records <= kSmallServe): statuses, reply offsets, decode

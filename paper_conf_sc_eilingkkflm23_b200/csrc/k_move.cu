@@ -20,6 +20,8 @@
 // segment walk done by the consumers with direct 16-byte global loads and warp-shuffle realignment.
 // Two tile queues (decode jobs, encode jobs) are claimed alternately so a serve step keeps both PCIe
 // directions busy when the rings live in host memory.
+#include <mutex>
+
 #include "k_move.cuh"
 
 namespace crk {
@@ -88,7 +90,8 @@ __device__ bool mover_cta_runs(const MoveParams& M) {
       while (c[8] != M.seq && gtimer32() - t < 2 * kOppLateNs) __nanosleep(256);
       if (c[8] == M.seq) {
         __threadfence();
-        g = t - c[9] < kOppLateNs;
+        g = (int32_t)(t - c[9]) < (int32_t)kOppLateNs;  // signed: a CTA that read the timer before CTA 0
+                                                        // stamped it started with the launch
       }
     }
     go = g;
@@ -759,13 +762,13 @@ cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, 
   M.seq = ++sc.mover_seq;
   M.use_map = use_map ? 1u : 0u;
   M.opp_from = (uint32_t)move_ctas > 2 * cfg.reserve ? (uint32_t)move_ctas - cfg.reserve : (uint32_t)move_ctas;
+  // Reserved CTAs compare against the launch stamp of the same launch (sequence M.seq).  A captured graph
+  // replays one baked M.seq, so a replay could read the previous replay's stamp: no reserve under capture.
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &cap) == cudaSuccess && cap != cudaStreamCaptureStatusNone)
+    M.opp_from = (uint32_t)move_ctas;
   const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
-  static uint32_t smem_set = 0;  // dynamic shared memory opt-in (per process, grows monotonically)
-  if (smem > smem_set) {
-    e = cudaFuncSetAttribute(mover_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    smem_set = smem;
-  }
+  if ((e = ensure_mover_smem(smem)) != cudaSuccess) return e;
   prof_mark(PROF_MOVE, true, s);
   mover_kernel<<<move_ctas, kMoverThreads, smem, s>>>(M);
   count_launch();
@@ -773,11 +776,27 @@ cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, 
   return cudaGetLastError();
 }
 
-// CTAs per SM the mover can keep resident for a tile size (sets the dynamic shared memory limit).
+// The mover's dynamic shared memory opt-in is a per-device attribute of the kernel.  It is kept per device
+// and only ever raised (under a lock), so a context created later with smaller tiles never lowers the
+// limit another context's launches rely on, and each device gets its own opt-in.
+cudaError_t ensure_mover_smem(uint32_t smem) {
+  static std::mutex mu;
+  static uint32_t set[kMaxDevices] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lk(mu);
+  if (smem <= set[dev]) return cudaSuccess;
+  e = cudaFuncSetAttribute(mover_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) set[dev] = smem;
+  return e;
+}
+
+// CTAs per SM the mover can keep resident for a tile size (raises the dynamic shared memory limit).
 int mover_occupancy(uint32_t tile_bytes, uint32_t stages) {
   const uint32_t smem = mover_smem_bytes(tile_bytes, stages);
-  if (cudaFuncSetAttribute(mover_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-    return 0;
+  if (ensure_mover_smem(smem) != cudaSuccess) return 0;
   int n = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, mover_kernel, kMoverThreads, smem);
   return n;

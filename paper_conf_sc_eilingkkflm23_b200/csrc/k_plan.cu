@@ -33,6 +33,7 @@ __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint3
         else {
           m = (cfg.strict || nb <= size) ? nb : size;
           if (cap < m) { st = CRK_E_PTR; m = 0; }
+          else if (m && !dst) { st = CRK_E_ARG; m = 0; }  // a NULL destination for a non-empty payload
           else job = dec_job(ix, dst, m, ix.p_off[(uint64_t)d * kMaxItems + 1], d, 1);
         }
       }
@@ -64,6 +65,8 @@ __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uin
         st = CRK_E_ARG;
       } else if (ix.p_count[b] > r.max_count) {
         st = CRK_E_SIZE;
+      } else if ((ix.p_count[b] && !r.dst) || ((uint64_t)r.dst % es) != 0) {
+        st = CRK_E_ARG;  // NULL or misaligned destination: the element swap works in element lanes
       } else {
         cnt = ix.p_count[b];
         job = dec_job(ix, (uint64_t)r.dst, cnt * es, ix.p_off[b], d, es);

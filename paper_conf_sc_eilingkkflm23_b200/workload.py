@@ -120,6 +120,132 @@ class Slot:
     idx: crk.Index
     ep: Endpoint
     stream: torch.cuda.Stream
+    res: "crk.PinnedResults | None" = None
+
+
+# Mover settings of the pipelined server loop (bench.py's timed configuration): with batches in flight the
+# mover leaves 16 CTA slots free, so the next batch's front-end kernels and the start of its mover overlap
+# this one, and claims whole runs to the end (its CTAs retire staggered, handing SMs over gradually).
+PIPELINE_CTX = {"mover_reserve_ctas": 16, "mover_tail_tiles": 0}
+INDEX_SHAPE = dict(max_frags=1 << 20, max_records=1 << 14)  # per endpoint (16 rings): > kSmallServe records
+
+
+def pipelined_ctx_kw(ctx_kw: dict, pipeline: int) -> dict:
+    kw = dict(ctx_kw)
+    if pipeline > 1:
+        for k, v in PIPELINE_CTX.items():
+            kw.setdefault(k, v)
+    return kw
+
+
+def build_slots(device_index: int, rank: int, device: torch.device, pipeline: int, ctx_kw: dict,
+                n_streams: int = 16, payload_per_stream: int = 64 * MiB, h2d_frac: float = 0.5,
+                host_rings: bool = False, staged: bool = False, ctxs: list | None = None,
+                default_stream=None) -> list[Slot]:
+    """The `pipeline` slots of a server loop, each with its own context, index, stream and C5 endpoint
+    (bench.py's device-resident loop; host_rings / staged for its end-to-end modes)."""
+    slots = []
+    for i in range(pipeline):
+        ctx = ctxs[i] if ctxs and i < len(ctxs) else crk.Context(device_index, **ctx_kw)
+        ep = c5_endpoint(ctx, rank, device, n_streams=n_streams, payload_per_stream=payload_per_stream,
+                         host_rings=host_rings, staged=staged, h2d_frac=h2d_frac)
+        idx = ctx.index(max_rings=n_streams, **INDEX_SHAPE)
+        st = torch.cuda.Stream(device) if pipeline > 1 or default_stream is None else default_stream
+        slots.append(Slot(ctx, idx, ep, st, crk.PinnedResults(n_streams) if host_rings else None))
+    return slots
+
+
+def run_pipelined(slots: list[Slot], stream, n_steps: int, step_fn=None):
+    """bench.py's server loop: step k is served by slot k % P on the slot's stream, so up to P batches are in
+    flight.  Returns CUDA events recorded on `stream` before the first and after the last step."""
+    P = len(slots)
+    step_fn = step_fn or (lambda s: serve_step(s.idx, s.ep, stream=s.stream))
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for s in slots:
+        s.stream.wait_event(e0)
+    for k in range(n_steps):
+        step_fn(slots[k % P])
+    for s in slots:
+        ev = torch.cuda.Event()
+        ev.record(s.stream)
+        stream.wait_event(ev)
+    e1.record(stream)
+    return e0, e1
+
+
+class StagedLoop:
+    """Copy-engine e2e mode (host rings): per slot, inbound DMA (in_stream, after the slot's previous serve
+    has read its device rings) -> serve from HBM (stream, after the previous reply DMA has drained the device
+    send rings) -> reply DMA (out_stream, queued by the host once the reply sizes are known).  Inbound DMA
+    of later batches never waits behind a reply DMA."""
+
+    def __init__(self, slots: list[Slot], device: torch.device, copy_streams: int = 1):
+        self.slots = slots
+        for s in slots:
+            s.in_stream, s.out_stream = torch.cuda.Stream(device), torch.cuda.Stream(device)
+            s.in_aux = [torch.cuda.Stream(device) for _ in range(copy_streams - 1)]
+            s.out_aux = [torch.cuda.Stream(device) for _ in range(copy_streams - 1)]
+            s.ev_in, s.ev_served, s.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
+            s.ev_out.record(s.out_stream)
+            s.ev_served.record(s.stream)
+
+    @staticmethod
+    def _drain(ps: Slot):
+        ps.ev_served.synchronize()
+        ps.out_stream.wait_event(ps.ev_served)
+        staged_out(ps.ep, ps.res.rows(), ps.out_stream, ps.out_aux)
+        ps.ev_out.record(ps.out_stream)
+
+    def run(self, n_steps: int):
+        P, pend = len(self.slots), []
+        for k in range(n_steps):
+            s = self.slots[k % P]
+            s.in_stream.wait_event(s.ev_served)
+            staged_in(s.ep, s.in_stream, s.in_aux)
+            s.ev_in.record(s.in_stream)
+            s.stream.wait_event(s.ev_in)
+            s.stream.wait_event(s.ev_out)
+            staged_serve(s.idx, s.ep, s.res, s.stream)
+            s.ev_served.record(s.stream)
+            pend.append(s)
+            if len(pend) >= P:
+                self._drain(pend.pop(0))
+        for ps in pend:
+            self._drain(ps)
+        torch.cuda.synchronize()
+
+    def run_mixed(self, n_steps: int):
+        """Copy engine in, SM zero-copy out: the inbound window is DMA'd into the device ring, the mover writes
+        the replies straight into the pinned host send rings (no outbound DMA)."""
+        P = len(self.slots)
+        for k in range(n_steps):
+            s = self.slots[k % P]
+            s.in_stream.wait_event(s.ev_served)
+            staged_in(s.ep, s.in_stream)
+            s.ev_in.record(s.in_stream)
+            s.stream.wait_event(s.ev_in)
+            s.idx.serve([(dr, h, t) for dr, (_, h, t) in zip(s.ep.dev_rings, s.ep.rings)], s.ep.sends,
+                        s.ep.offs, s.ep.base, s.ep.region.numel(), stream=s.stream)
+            s.idx.ring_results_async(s.res, stream=s.stream)
+            s.ev_served.record(s.stream)
+        torch.cuda.synchronize()
+
+    def run_zero_copy(self, n_steps: int):
+        """Zero-copy: the kernels read the CALL rings from and write the reply rings to pinned host memory.
+        Step k is launched before the results of step k-1 are read back (device -> host, syncs that slot's
+        stream), so the host read overlaps the next batch."""
+        P = len(self.slots)
+        for k in range(n_steps):
+            s = self.slots[k % P]
+            serve_step(s.idx, s.ep, stream=s.stream)
+            if k >= P - 1:
+                p_ = self.slots[(k - P + 1) % P]
+                p_.idx.ring_results(len(p_.ep.rings), stream=p_.stream)
+        for k in range(max(0, n_steps - P + 1), n_steps):
+            p_ = self.slots[k % P]
+            p_.idx.ring_results(len(p_.ep.rings), stream=p_.stream)
+        torch.cuda.synchronize()
 
 
 def serve_step(idx: crk.Index, ep: Endpoint, stream=None):

@@ -604,13 +604,19 @@ def test_serve_matches_oracle(host, mover):
         sends.append(make_ring(1 << 23, host))
         offs.append(777 * s.stream)
     region.copy_(torch.from_numpy(host_region))
-    idx = ctx.index(4, 1 << 14, 1 << 10)
+    # the run -> job map configs need the multi-kernel planning path: an index above kSmallServe (1024)
+    # records, otherwise the one-block planner plans the jobs and the mover claims through find_job
+    map_cfg = MOVER_CONFIGS[mover].get("mover_run") == 2
+    max_records = 1 << 11 if map_cfg else 1 << 10
+    idx = ctx.index(4, 1 << 14, max_records)
     idx.serve(rings, sends, offs, base, region_bytes + 64)
     torch.cuda.synchronize()
+    if map_cfg:
+        assert ctx.debug_counters()[13] == 1, "the mover did not claim through the run -> job map"
     T = idx.tables(4)
     ring_bytes = [ring_np(r[0]) for r in rings]
     want = O.serve([(rb, h, t) for rb, (_, h, t) in zip(ring_bytes, rings)], cfg, host_region, base,
-                   [1 << 23] * 4, offs, max_frags_per_ring=(1 << 14) // 4, max_records_per_ring=(1 << 10) // 4)
+                   [1 << 23] * 4, offs, max_frags_per_ring=(1 << 14) // 4, max_records_per_ring=max_records // 4)
     assert np.array_equal(region.cpu().numpy(), host_region)
     P = T["parsed"]
     assert [r["status"] for r in want["records"]] == list(P["serve_status"])
@@ -800,3 +806,43 @@ def test_serve_graph_replays_with_doorbell_cursors():
     torch.cuda.synchronize()
     assert idx.ring_results(1)[0]["status"] == O.E_ARG
     graph.close()
+
+
+def test_batch_requests_reject_null_and_misaligned_dst():
+    """batched requests check their destinations like the single-request calls do (include/crk.h:
+    NULL dst with a non-empty payload, or a typed dst not aligned to the element size -> E_ARG, nothing
+    written) instead of faulting or byte-swapping across element lanes."""
+    cfg = ocfg(user={33: [O.K_I32_VAR, O.K_F64_VAR, O.K_OPAQUE_VAR]})
+    ctx = ctx_for(cfg)
+    ring = make_ring(1 << 16)
+    a = np.arange(9, dtype=np.int32)
+    b = np.arange(3, dtype=np.float64)
+    wire = (O.encode_call(1, 33, [(O.K_I32_VAR, a), (O.K_F64_VAR, b), (O.K_OPAQUE_VAR, b"")], cfg)
+            + O.encode_call(2, gen.PROC_H2D, [(O.K_U64, 0), (O.K_OPAQUE_VAR, b"abcdef"), (O.K_U64, 6)], cfg))
+    tail = place(ring, wire, 0)
+    idx = ctx.index(1, 64, 16)
+    idx.frame_scan([(ring, 0, tail)])
+    out = torch.zeros(256, dtype=torch.uint8, device="cuda")
+    st = torch.full((6,), 99, dtype=torch.int32, device="cuda")
+    p = out.data_ptr()
+    reqs = [(1, 0, O.K_I32_VAR, p + 2, 9, None, st.data_ptr()),        # misaligned int32 dst
+            (1, 1, O.K_F64_VAR, p + 4, 3, None, st.data_ptr() + 4),    # misaligned double dst
+            (1, 0, O.K_I32_VAR, 0, 9, None, st.data_ptr() + 8),        # NULL dst, 9 elements
+            (1, 2, O.K_OPAQUE_VAR, 0, 0, None, st.data_ptr() + 12),    # NULL dst, empty opaque: fine
+            (1, 1, O.K_F64_VAR, p + 64, 3, None, st.data_ptr() + 16)]  # aligned: decoded
+    keep = idx.decode_items_batch(reqs)
+    torch.cuda.synchronize()
+    assert st.cpu().tolist()[:5] == [O.E_ARG, O.E_ARG, O.E_ARG, O.OK, O.OK]
+    got = out.cpu().numpy()
+    assert not got[:64].any()  # nothing written by the rejected requests
+    assert got[64:88].tobytes() == b.tobytes()
+    del keep
+    xids = torch.tensor([2, 2], dtype=torch.int32, device="cuda")
+    dsts = torch.tensor([0, p + 100], dtype=torch.int64, device="cuda")
+    caps = torch.tensor([6, 6], dtype=torch.int64, device="cuda")
+    sts = torch.full((2,), 99, dtype=torch.int32, device="cuda")
+    cps = torch.full((2,), 99, dtype=torch.int64, device="cuda")
+    idx.decode_memcpy_h2d_batch(xids, dsts, caps, sts, cps)
+    torch.cuda.synchronize()
+    assert sts.cpu().tolist() == [O.E_ARG, O.OK] and cps.cpu().tolist() == [0, 6]
+    assert out.cpu().numpy()[100:106].tobytes() == b"abcdef"
