@@ -107,11 +107,13 @@ typedef struct {
                                   free: a lone call gets the whole grid); behind another batch's mover (several
                                   batches in flight on other streams) they exit at once, so the next batch's
                                   scan / parse / plan kernels find room on the GPU while this mover streams */
-  uint32_t fused_front_max_records; /* crk_serve with an index of at most this many records (and one ring, or
-                                       at most fused_front_max_window bytes of ring windows) runs scan + parse +
-                                       planning as ONE single-CTA launch before the mover (default 128, at most
-                                       1024 takes effect; 0 = always separate kernels) */
-  uint32_t pad0_;
+  uint32_t fused_front_max_records; /* crk_serve with an index of at most this many records (and at most
+                                       fused_front_max_window bytes of ring windows; with scan_chunking = 1 also
+                                       any single ring) runs scan + parse + planning as ONE single-CTA launch
+                                       before the mover (default 128, at most 1024 takes effect; 0 = always
+                                       separate kernels) */
+  uint32_t scan_chunking;    /* 0 (default): windows of at least 2 chunks (>= 512 KiB) are scanned by the chunked
+                                multi-CTA scan (one CTA per chunk); 1: always one CTA per ring */
   uint64_t fused_front_max_window; /* default 1 MiB (one CTA scans the rings in turn) */
 } crk_config;
 

@@ -45,7 +45,7 @@ class Config(C.Structure):
                 ("scan_stride_guess", C.c_uint32), ("tile_bytes", C.c_uint32), ("max_jobs", C.c_uint32),
                 ("ctas_per_sm", C.c_uint32), ("scan_threads", C.c_uint32), ("mover_stages", C.c_uint32),
                 ("mover_run", C.c_uint32), ("mover_tail_tiles", C.c_uint32), ("mover_reserve_ctas", C.c_uint32),
-                ("fused_front_max_records", C.c_uint32), ("pad0_", C.c_uint32), ("fused_front_max_window", C.c_uint64)]
+                ("fused_front_max_records", C.c_uint32), ("scan_chunking", C.c_uint32), ("fused_front_max_window", C.c_uint64)]
 
 
 class CRing(C.Structure):
@@ -141,6 +141,8 @@ def lib():
             "crk_profile_read": (C.c_int, [C.POINTER(C.c_double), C.POINTER(u32)]),
             "crk_version": (C.c_char_p, []),
             "crk_debug_counters": (C.c_int, [vp, C.POINTER(u32)]),  # diagnostic, not in include/crk.h
+            "crk_debug_index_stats": (C.c_int, [vp, C.POINTER(u32)]),  # diagnostic, not in include/crk.h
+            "crk_debug_index_ms": (C.c_int, [vp, C.POINTER(vp), C.POINTER(u32)]),  # diagnostic
         }
         for t in ("i32", "u32", "i64", "u64", "f32", "f64"):
             sig[f"crk_xdr_decode_array_{t}"] = (C.c_int, [vp, vp, u32, u32, vp, u64, vp, vp, vp])
@@ -479,6 +481,13 @@ class Index:
         """Captures one server step reading its cursors from `doorbell` (a device uint64 tensor or a
         HostBuffer of 3 * n_rings uint64: heads | tails | send offsets)."""
         return ServeGraph(self, rings, send_rings, region_base, region_bytes, doorbell)
+
+    def scan_stats(self) -> dict:
+        """Diagnostic: rings this index's scans resolved with the chunked multi-CTA scan, and rings that fell
+        back to the one-CTA scan (totals since creation; synchronises the device)."""
+        out = (C.c_uint32 * 4)()
+        _check(lib().crk_debug_index_stats(self.h, out), "crk_debug_index_stats")
+        return {"chunked": out[0], "fallback": out[1]}
 
     def ring_results(self, n: int | None = None, stream=None) -> list[dict]:
         n = self.n_rings if n is None else n

@@ -1,6 +1,7 @@
 // The C ABI (include/crk.h): argument checks, scratch ownership and launch sequences.  No byte of the
 // data path is touched here; every step runs in the kernels of k_scan / k_parse / k_prefix / k_plan /
 // k_move.
+#include <algorithm>
 #include <atomic>
 #include <cstdio>
 #include <cstdlib>
@@ -137,12 +138,15 @@ int scan_param(crk_index* idx, uint32_t n_rings, const crk_ring* rings, const ui
 }
 
 // A small index (crk_config.fused_front_max_records) over one ring or a small window: one fused launch.
+// A window long enough for the chunked multi-CTA scan (k_mscan.cu) goes to the separate kernels even on one
+// ring: the single CTA of the fused front end would walk its whole header chain alone.
 bool fused_front(const crk_ctx* c, const crk_index* x, uint32_t n_rings, const uint64_t* heads, const uint64_t* tails,
                  const uint64_t* doorbell) {
   uint64_t window = 0;
   for (uint32_t r = 0; !doorbell && heads && tails && r < n_rings; ++r) window += tails[r] - heads[r];
+  const bool chunkable = !doorbell && c->cfg.scan_chunking == 0 && window > c->cfg.fused_front_max_window;
   return x->ix.max_records <= c->cfg.fused_front_max_records && x->ix.max_records <= front_small_threads() &&
-         (n_rings == 1 || (!doorbell && window <= c->cfg.fused_front_max_window));
+         !chunkable && (n_rings == 1 || (!doorbell && window <= c->cfg.fused_front_max_window));
 }
 
 int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
@@ -273,7 +277,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   if (cfg.frag_payload == 0 || cfg.frag_payload > 0x7fffffffu || !pow2(cfg.tile_bytes) || cfg.tile_bytes < 1024 ||
       cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 64 ||
       cfg.scan_threads > 1024 || (cfg.scan_threads & 63) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
-      cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64)
+      cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64 || cfg.scan_chunking > 1)
     return CRK_E_ARG;
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -305,6 +309,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.run = cfg.mover_run;
   d.tail = cfg.mover_tail_tiles;
   d.reserve = cfg.mover_reserve_ctas;
+  d.no_chunked_scan = cfg.scan_chunking == 1 ? 1u : 0u;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
   // scratch: one block
@@ -391,6 +396,10 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
   while (hs < 2ull * R) hs <<= 1;
   ix.hash_mask = (uint32_t)(hs - 1);
   const uint64_t MI = (uint64_t)R * kMaxItems;
+  // chunked-scan scratch (k_mscan.cu): enough chunks for the index's fragment capacity at ~16 fragments per
+  // chunk, 64 .. 2048
+  const uint32_t CC = std::min<uint32_t>(2048u, std::max<uint32_t>(64u, F / 16));
+  ix.ms.chunk_cap = CC;
   const size_t sz[] = {
       sizeof(RingDesc) * max_rings, sizeof(crk_ring_result) * max_rings, sizeof(uint32_t) * (max_rings + 1), 4, 4,
       8 * (size_t)F, 8 * (size_t)F, 4 * (size_t)F,                              // frags
@@ -398,7 +407,9 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
       4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R,  // parsed scalars
       4 * MI, 8 * MI, 8 * MI, 8 * MI,                                           // items
       4 * (size_t)R, 4 * (size_t)R, 8 * (size_t)R, 8 * (size_t)R,               // serve
-      8 * (size_t)hs};
+      8 * (size_t)hs,
+      sizeof(uint2) * (size_t)CC * kCand * kLogCap, sizeof(ChainSum) * (size_t)CC * kCand,  // chunked scan
+      sizeof(ChunkState) * (size_t)CC, sizeof(ChunkStop) * (size_t)CC, sizeof(RingPlan) * max_rings, 16};
   constexpr int N = sizeof(sz) / sizeof(sz[0]);
   size_t total = 0, off[N];
   for (int i = 0; i < N; ++i) { off[i] = total; total += (sz[i] + 255) & ~(size_t)255; }
@@ -433,8 +444,16 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
   ix.s_reply_off = (uint64_t*)(b + off[i++]);
   ix.s_reply_wire = (uint64_t*)(b + off[i++]);
   ix.xid_hash = (unsigned long long*)(b + off[i++]);
+  ix.ms.log = (uint2*)(b + off[i++]);
+  ix.ms.sums = (ChainSum*)(b + off[i++]);
+  ix.ms.state = (ChunkState*)(b + off[i++]);
+  ix.ms.stops = (ChunkStop*)(b + off[i++]);
+  ix.ms.plan = (RingPlan*)(b + off[i++]);
+  ix.ms.stats = (uint32_t*)(b + off[i++]);
   e = cudaMemset(x->block, 0, total);
   if (e == cudaSuccess) e = cudaMemset(ix.xid_hash, 0xff, 8 * (size_t)hs);
+  for (uint32_t r = 0; e == cudaSuccess && r < max_rings; ++r)  // no stop recorded
+    e = cudaMemset(&ix.ms.plan[r].stop_key, 0xff, sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMallocHost(&x->host_res, sizeof(crk_ring_result) * max_rings);
   if (e != cudaSuccess) { cudaFree(x->block); delete x; return cuda_fail(e); }
   *out = x;
@@ -816,6 +835,29 @@ void crk_graph_destroy(crk_graph* G) {
   cudaGraphExecDestroy(G->exec);
   cudaGraphDestroy(G->graph);
   delete G;
+}
+
+// Diagnostic (not in the public header): the chunked scan's totals for this index (rings resolved by the
+// chunked scan, rings that fell back to the one-CTA scan) after synchronising the device.
+extern "C" int crk_debug_index_stats(crk_index* x, uint32_t* host4) {
+  if (!x || !host4) return CRK_E_ARG;
+  DeviceGuard g(x->device);
+  if (cudaDeviceSynchronize() != cudaSuccess) return CRK_E_CUDA;
+  if (cudaMemcpy(host4, x->ix.ms.stats, 16, cudaMemcpyDeviceToHost) != cudaSuccess) return CRK_E_CUDA;
+  return CRK_OK;
+}
+
+// Diagnostic (not in the public header): device pointers of the chunked scan's scratch (sums, state, stops,
+// plan, log) and its chunk capacity, for inspection tools.
+extern "C" int crk_debug_index_ms(crk_index* x, void** ptrs5, uint32_t* chunk_cap) {
+  if (!x || !ptrs5 || !chunk_cap) return CRK_E_ARG;
+  ptrs5[0] = x->ix.ms.sums;
+  ptrs5[1] = x->ix.ms.state;
+  ptrs5[2] = x->ix.ms.stops;
+  ptrs5[3] = x->ix.ms.plan;
+  ptrs5[4] = x->ix.ms.log;
+  *chunk_cap = x->ix.ms.chunk_cap;
+  return CRK_OK;
 }
 
 // Diagnostic (not in the public header): copies the context's 16 scratch counters (crk_internal.h Scratch::

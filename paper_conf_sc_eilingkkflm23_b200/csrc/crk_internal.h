@@ -30,6 +30,46 @@ struct RingDesc {
   uint64_t head, tail;
 };
 
+// ---- chunked scan of long windows (k_mscan.cu): per-index scratch --------------------------------
+constexpr uint32_t kCand = 4;       // candidate chains walked per chunk
+constexpr uint32_t kLogCap = 512;   // headers logged per chain
+struct alignas(16) ChainSum {       // one candidate chain of one chunk (64 bytes)
+  uint64_t start, exit;             // its first header; the cursor after its last logged header
+  uint64_t r0_after, sum_after;     // after its last last-fragment header: next record start, lengths since
+  uint64_t sum_total;               // sum of all logged lengths
+  uint32_t n, nlast;                // logged headers, of which last fragments
+  int32_t idx_last;                 // log index of the last last-fragment header (-1: none)
+  uint32_t kind;                    // CH_* (k_mscan.cu)
+  uint64_t pad_;
+};
+static_assert(sizeof(ChainSum) == 64, "ChainSum is read as four 16-byte words");
+struct ChunkState {                 // the walk state at a chunk's true entry (written by the resolver)
+  uint64_t p, r0, sum;
+  uint32_t nf, nr, f0;
+  int32_t chosen;                   // candidate chain holding the true chain, -1: no header starts here
+  uint32_t skip;                    // log entries of that chain before the true entry (a false start fed it)
+  uint32_t pad_;
+};
+struct ChunkStop {                  // outcome of a check that failed in this chunk's emission
+  uint64_t consumed;
+  int32_t status;
+  uint32_t nr, kept, pad_;
+};
+struct RingPlan {                   // per ring of the index
+  uint32_t ticket_a, ticket_b, fallback, pad_;
+  unsigned long long stop_key;      // min over failing hops of (fragment number << 24 | chunk), ~0 = none
+  crk_ring_result end;              // the outcome when no check fails (end of the chain)
+};
+struct MultiScanDev {
+  uint32_t chunk_cap;               // chunks one launch can hold
+  uint2* log;                       // [chunk_cap * kCand * kLogCap]: (cursor - chunk start, header)
+  ChainSum* sums;                   // [chunk_cap * kCand]
+  ChunkState* state;                // [chunk_cap]
+  ChunkStop* stops;                 // [chunk_cap]
+  RingPlan* plan;                   // [max_rings]
+  uint32_t* stats;                  // [4] diagnostic totals: rings resolved chunked, rings that fell back
+};
+
 // Device-resident tables of one index (pointers into one cudaMalloc block).
 struct IndexDev {
   uint32_t max_rings, frags_per_ring, recs_per_ring, max_records;
@@ -61,6 +101,7 @@ struct IndexDev {
   uint64_t* s_reply_off;
   uint64_t* s_reply_wire;
   unsigned long long* xid_hash;  // (xid << 32 | dense id), empty = ~0
+  MultiScanDev ms;               // chunked scan scratch
 };
 
 // ---- mover jobs ----------------------------------------------------------------------------------
@@ -113,7 +154,8 @@ struct Scratch {          // ctx-owned device scratch
 struct ConfigDev {
   uint32_t F, strict, prog, vers, proc_h2d, proc_d2h, guess, tile_shift;
   uint32_t scan_threads, stages, run, tail;  // tail: per-CTA single-tile claims at the end of each queue
-  uint32_t reserve, pad_;  // mover CTAs that run only when the launch found the GPU free (crk_config.mover_reserve_ctas)
+  uint32_t reserve;         // mover CTAs that run only when the launch found the GPU free (crk_config.mover_reserve_ctas)
+  uint32_t no_chunked_scan; // crk_config.scan_chunking == 1: one CTA per ring always
   uint64_t max_record_bytes;
   unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };
@@ -128,6 +170,12 @@ struct ScanRingsParam {
 };
 
 cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s);
+// Chunked multi-CTA scan of long windows (k_mscan.cu): chunk_plan fills an opaque parameter block
+// (chunk_param_bytes()) and returns false when every ring is short enough for the one-CTA scan.
+bool chunk_plan(const IndexDev& ix, const ScanRingsParam& p, int sms, void* out_param);
+size_t chunk_param_bytes();
+uint32_t chunk_plan_chunks(const void* param);
+cudaError_t launch_chunk_scan(const IndexDev& ix, const void* param, const ConfigDev& cfg, cudaStream_t s);
 cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const ConfigDev& cfg, uint32_t n_rings,
                          int sms, cudaStream_t s);
 // Exclusive scan of n u64 values in place; total (may be null) gets the sum.  n read from n_dev if

@@ -1,5 +1,7 @@
 // K1 kernel: one CTA per ring runs scan_ring_cta (k_scan.cuh); the last CTA to finish numbers the
 // records densely across rings.
+#include <vector>
+
 #include "k_scan.cuh"
 
 namespace crk {
@@ -45,12 +47,25 @@ extern "C" int crk_debug_scan_trace(unsigned long long* out, uint32_t* counts, i
 }
 #endif
 
+// Long windows (explicit cursors) take the chunked multi-CTA scan (k_mscan.cu); short ones, and windows
+// published through a doorbell at execution time, the one-CTA-per-ring scan.
 cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const ConfigDev& cfg, cudaStream_t s) {
+  static thread_local std::vector<unsigned char> chunk_param;
+  chunk_param.resize(chunk_param_bytes());
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   prof_mark(PROF_SCAN, true, s);
-  frame_scan_kernel<<<p.n_rings, cfg.scan_threads, 0, s>>>(ix, p, cfg);
-  count_launch();
+  cudaError_t e;
+  if (!cfg.no_chunked_scan && chunk_plan(ix, p, sms, chunk_param.data())) {
+    e = launch_chunk_scan(ix, chunk_param.data(), cfg, s);
+  } else {
+    frame_scan_kernel<<<p.n_rings, cfg.scan_threads, 0, s>>>(ix, p, cfg);
+    count_launch();
+    e = cudaGetLastError();
+  }
   prof_mark(PROF_SCAN, false, s);
-  return cudaGetLastError();
+  return e;
 }
 
 }  // namespace crk

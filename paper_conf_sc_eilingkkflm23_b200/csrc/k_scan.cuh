@@ -118,16 +118,108 @@ __device__ __forceinline__ void prefetch_l2(const RingDesc& R, uint64_t c, uint3
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(R.base + o), "r"(n) : "memory");
 }
 
+// The index work for a batch of consecutive chain hops, one per lane (lane k = hop k at cursor myq with
+// header myh; hop 0 is at W.p, each next hop at the previous one's cursor + 4 + length): for the first
+// n_take hops, the closed forms of or_frame_scan's loop -- segmented prefix sums of the lengths (logical
+// starts), record boundaries -- and its checks in its order (E_FRAG -> INCOMPLETE -> index capacity),
+// all with warp scans, then the fragment / record index entries of the hops before the first failing
+// one.  On a failure the outcome is recorded in W (stop) and its hop number returned; otherwise W
+// advances past hop n_take - 1 (and the predictors follow its headers) and -1 is returned.  Used by the
+// chase pass below and by the chunked scan's emission (k_mscan.cu), whose hops come from a log.
+__device__ int take_hops(const Env& E, Walk& W, uint32_t lane, uint32_t n_take, uint64_t myq, uint32_t myh) {
+  const uint64_t tail = E.R.tail;
+  const uint32_t vmask = n_take >= 32 ? kFull : (1u << n_take) - 1;
+  const bool v = lane < n_take;
+  const uint64_t len = v ? (uint64_t)(myh & 0x7fffffffu) : 0ull;
+  const uint32_t last = v ? myh >> 31 : 0u;
+  const uint32_t lastm = __ballot_sync(kFull, last);
+  const uint32_t startm = ((lastm << 1) | (W.p == W.r0 ? 1u : 0u)) & vmask;
+  const bool start = (startm >> lane) & 1;
+  uint64_t P = len;  // inclusive prefix of lengths over the batch
+#pragma unroll
+  for (uint32_t o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(kFull, P, o);
+    if (lane >= o) P += y;
+  }
+  const uint64_t Ex = P - len;
+  const uint32_t below = startm & (lane == 31 ? kFull : (2u << lane) - 1);
+  const int j = below ? 31 - __clz(below) : -1;  // this hop's record began at hop j of the batch
+  const uint64_t Ej = __shfl_sync(kFull, Ex, j < 0 ? 0 : j);
+  const uint64_t qj = __shfl_sync(kFull, myq, j < 0 ? 0 : j);
+  const uint64_t send = j >= 0 ? P - Ej : W.sum + P;  // logical end of this fragment in its record
+  const uint64_t rbeg = j >= 0 ? qj : W.r0;
+  const uint32_t f0 = j >= 0 ? W.nf + (uint32_t)j : W.f0;
+  const uint32_t nrec = W.nr + __popc(lastm & ((1u << lane) - 1));
+  uint32_t code = STOP_NONE;
+  if (v) {
+    if (send > E.max_record_bytes) code = STOP_FRAG;
+    else if (myq + 4 + len > tail) code = STOP_INCOMPLETE;
+    else if (W.nf + lane >= E.FC || (start && nrec >= E.RC)) code = STOP_CAP;
+  }
+  const uint32_t failm = __ballot_sync(kFull, code != STOP_NONE);
+  const uint32_t tf = failm ? __ffs(failm) - 1 : 32u;
+  const uint32_t n_acc = tf < n_take ? tf : n_take;
+  if (lane < n_acc) {
+    const uint64_t fs = E.fbase + W.nf + lane;
+    E.ix.frag_phys[fs] = myq + 4;
+    E.ix.frag_lstart[fs] = send - len;
+    E.ix.frag_hdr[fs] = myh;
+    // (nrec < RC always holds for a walk that checks every record start; a chunk of the chunked scan that
+    // starts inside a record after an earlier chunk's capacity stop must still stay inside the slice)
+    if (last && nrec < E.RC) {
+      const uint64_t rs = E.rbase + nrec;
+      E.ix.rec_begin[rs] = start ? myq : rbeg;
+      E.ix.rec_len[rs] = send;
+      E.ix.rec_frag0[rs] = (uint32_t)(E.fbase + f0);
+      E.ix.rec_nfrags[rs] = W.nf + lane - f0 + 1;
+    }
+  }
+  if (tf < n_take) {  // hop tf's check failed: the outcome is recorded there
+    const uint32_t c = __shfl_sync(kFull, code, tf);
+    const uint32_t nr_t = __shfl_sync(kFull, nrec, tf);
+    const bool st_t = (startm >> tf) & 1;
+    W.consumed = st_t ? __shfl_sync(kFull, myq, tf) : __shfl_sync(kFull, rbeg, tf);
+    W.kept = st_t ? W.nf + tf : __shfl_sync(kFull, f0, tf);
+    W.nr = nr_t;
+    W.status = c == STOP_FRAG ? CRK_E_FRAG : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
+             : (nr_t > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
+    W.stop = true;
+    return (int)tf;
+  }
+  if (n_acc) {  // advance the state to after hop n_acc - 1 and update the predictors
+    const uint32_t L = n_acc - 1, am = n_acc >= 32 ? kFull : (1u << n_acc) - 1;
+    const uint64_t qL = __shfl_sync(kFull, myq, L), lenL = __shfl_sync(kFull, len, L);
+    const uint64_t sendL = __shfl_sync(kFull, send, L), rbegL = __shfl_sync(kFull, rbeg, L);
+    const uint32_t f0L = __shfl_sync(kFull, f0, L), nrecL = __shfl_sync(kFull, nrec, L);
+    const uint32_t hL = __shfl_sync(kFull, myh, L);
+    const uint32_t singlem = __ballot_sync(kFull, start && last) & am, nonlastm = ~lastm & am;
+    if (singlem) W.hp1 = __shfl_sync(kFull, myh, 31 - __clz(singlem));
+    if (nonlastm) W.hp0 = __shfl_sync(kFull, myh, 31 - __clz(nonlastm));
+    W.p = qL + 4 + lenL;
+    W.nf += n_acc;
+    if (hL >> 31) {
+      W.nr = nrecL + 1;
+      W.r0 = W.p;
+      W.sum = 0;
+      W.f0 = W.nf;
+    } else {
+      W.nr = nrecL;
+      W.sum = sendL;
+      W.r0 = rbegL;
+      W.f0 = f0L;
+    }
+  }
+  return -1;
+}
+
 // Chase pass: the serial walk of the chain, for framing no predictor follows.  It runs in batches of 32
 // hops.  The walk itself carries only the chain (p -> p + 4 + len(be32(p))): every lane follows it
-// (broadcast loads) and lane k keeps hop k's cursor and header.  All per-header work -- the checks in
-// or_frame_scan's order E_FRAG -> INCOMPLETE -> capacity, the segmented prefix sum of lengths (logical
-// starts), record boundaries, the index writes -- is then done for the 32 hops at once with warp scans,
-// so a hop costs one load latency.  Hops past a failing header are walked but discarded (reads stay
-// inside the ring).  Once a pass is long (an irregular stream), the TMA prefetches the ring ahead of
-// the walk into L2 (kPfLead bytes ahead), so header reads hit L2 instead of HBM / the host link.
-// Stops after kChase headers, at a stop, or at two equal consecutive headers (a regular run the
-// predictors can take over again).
+// (broadcast loads) and lane k keeps hop k's cursor and header.  All per-header work is then take_hops
+// for the 32 hops at once, so a hop costs one load latency.  Hops past a failing header are walked but
+// discarded (reads stay inside the ring).  Once a pass is long (an irregular stream), the TMA prefetches
+// the ring ahead of the walk into L2 (kPfLead bytes ahead), so header reads hit L2 instead of HBM / the
+// host link.  Stops after kChase headers, at a stop, or at two equal consecutive headers (a regular run
+// the predictors can take over again).
 #ifndef CRK_PF_LEAD
 #define CRK_PF_LEAD (1ull << 20)  // prefetch frontier lead over the walk (bytes; 0 = no prefetch)
 #endif
@@ -165,90 +257,12 @@ __device__ void chase(const Env& E, Walk& W, uint32_t lane) {
       hw = h;
     }
     SCAN_TRACE(lane == 0, 2, n);
-    // ---- per-hop closed forms (lane k = hop k)
-    const uint32_t vmask = n == 32 ? kFull : (1u << n) - 1;
-    const bool v = lane < n;
-    const uint64_t len = v ? (uint64_t)(myh & 0x7fffffffu) : 0ull;
-    const uint32_t last = v ? myh >> 31 : 0u;
-    const uint32_t lastm = __ballot_sync(kFull, last);
-    const uint32_t startm = ((lastm << 1) | (W.p == W.r0 ? 1u : 0u)) & vmask;
-    const bool start = (startm >> lane) & 1;
-    uint64_t P = len;  // inclusive prefix of lengths over the batch
-#pragma unroll
-    for (uint32_t o = 1; o < 32; o <<= 1) {
-      const uint64_t y = __shfl_up_sync(kFull, P, o);
-      if (lane >= o) P += y;
-    }
-    const uint64_t Ex = P - len;
-    const uint32_t below = startm & (lane == 31 ? kFull : (2u << lane) - 1);
-    const int j = below ? 31 - __clz(below) : -1;  // this hop's record began at hop j of the batch
-    const uint64_t Ej = __shfl_sync(kFull, Ex, j < 0 ? 0 : j);
-    const uint64_t qj = __shfl_sync(kFull, myq, j < 0 ? 0 : j);
-    const uint64_t send = j >= 0 ? P - Ej : W.sum + P;  // logical end of this fragment in its record
-    const uint64_t rbeg = j >= 0 ? qj : W.r0;
-    const uint32_t f0 = j >= 0 ? W.nf + (uint32_t)j : W.f0;
-    const uint32_t nrec = W.nr + __popc(lastm & ((1u << lane) - 1));
-    uint32_t code = STOP_NONE;
-    if (v) {
-      if (send > E.max_record_bytes) code = STOP_FRAG;
-      else if (myq + 4 + len > tail) code = STOP_INCOMPLETE;
-      else if (W.nf + lane >= E.FC || (start && nrec >= E.RC)) code = STOP_CAP;
-    }
-    const uint32_t failm = __ballot_sync(kFull, code != STOP_NONE);
     const uint32_t hprev = __shfl_up_sync(kFull, myh, 1);
-    const uint32_t eqm = __ballot_sync(kFull, v && myh == (lane ? hprev : prev));
-    const uint32_t tf = failm ? __ffs(failm) - 1 : 32u, te = eqm ? __ffs(eqm) - 1 : 32u;
-    const bool fail_stop = tf < n && tf <= te;
-    const uint32_t n_acc = fail_stop ? tf : (te < n ? te + 1 : n);
-    if (lane < n_acc) {
-      const uint64_t fs = E.fbase + W.nf + lane;
-      E.ix.frag_phys[fs] = myq + 4;
-      E.ix.frag_lstart[fs] = send - len;
-      E.ix.frag_hdr[fs] = myh;
-      if (last) {
-        const uint64_t rs = E.rbase + nrec;
-        E.ix.rec_begin[rs] = start ? myq : rbeg;
-        E.ix.rec_len[rs] = send;
-        E.ix.rec_frag0[rs] = (uint32_t)(E.fbase + f0);
-        E.ix.rec_nfrags[rs] = W.nf + lane - f0 + 1;
-      }
-    }
-    if (fail_stop) {  // hop tf's check failed: the outcome is recorded there
-      const uint32_t c = __shfl_sync(kFull, code, tf);
-      const uint32_t nr_t = __shfl_sync(kFull, nrec, tf);
-      const bool st_t = (startm >> tf) & 1;
-      W.consumed = st_t ? __shfl_sync(kFull, myq, tf) : __shfl_sync(kFull, rbeg, tf);
-      W.kept = st_t ? W.nf + tf : __shfl_sync(kFull, f0, tf);
-      W.nr = nr_t;
-      W.status = c == STOP_FRAG ? CRK_E_FRAG : c == STOP_INCOMPLETE ? CRK_INCOMPLETE
-               : (nr_t > 0 ? CRK_INCOMPLETE : CRK_E_CAPACITY);
-      W.stop = true;
-      return;
-    }
-    if (n_acc) {  // advance the state to after hop n_acc - 1 and update the predictors
-      const uint32_t L = n_acc - 1, am = n_acc == 32 ? kFull : (1u << n_acc) - 1;
-      const uint64_t qL = __shfl_sync(kFull, myq, L), lenL = __shfl_sync(kFull, len, L);
-      const uint64_t sendL = __shfl_sync(kFull, send, L), rbegL = __shfl_sync(kFull, rbeg, L);
-      const uint32_t f0L = __shfl_sync(kFull, f0, L), nrecL = __shfl_sync(kFull, nrec, L);
-      const uint32_t hL = __shfl_sync(kFull, myh, L);
-      const uint32_t singlem = __ballot_sync(kFull, start && last) & am, nonlastm = ~lastm & am;
-      if (singlem) W.hp1 = __shfl_sync(kFull, myh, 31 - __clz(singlem));
-      if (nonlastm) W.hp0 = __shfl_sync(kFull, myh, 31 - __clz(nonlastm));
-      W.p = qL + 4 + lenL;
-      W.nf += n_acc;
-      if (hL >> 31) {
-        W.nr = nrecL + 1;
-        W.r0 = W.p;
-        W.sum = 0;
-        W.f0 = W.nf;
-      } else {
-        W.nr = nrecL;
-        W.sum = sendL;
-        W.r0 = rbegL;
-        W.f0 = f0L;
-      }
-      prev = hL;
-    }
+    const uint32_t eqm = __ballot_sync(kFull, lane < n && myh == (lane ? hprev : prev));
+    const uint32_t te = eqm ? __ffs(eqm) - 1 : 32u;
+    const uint32_t n_take = te < n ? te + 1 : n;
+    if (take_hops(E, W, lane, n_take, myq, myh) >= 0) return;
+    if (n_take) prev = __shfl_sync(kFull, myh, n_take - 1);
     if (te < n) return;  // two equal headers: back to the speculative rounds
     if (n < 32) {        // no readable header at W.p: the window ends here
       const bool st = W.p == W.r0;

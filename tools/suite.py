@@ -329,6 +329,7 @@ def c4(ctx, irregular):
                                        for o, s in zip(outs, srcs))
     return {"records": len(calls), "items": len(reqs), "payload_bytes": total, "wire": cur, "ms": round(ms, 3),
             "scan_ms": round(ms_scan, 3), "frags": int(idx.ring_results(1)[0]["n_frags"]),
+            "scan_stats": idx.scan_stats(),
             "decode_gbs": round(total / ms / 1e6, 1), "ok": ok}
 
 
