@@ -364,6 +364,30 @@ def main():
     prof = crk.profile_read()
     crk.profile_enable(False)
     serial_ms = max_over_ranks(f0.elapsed_time(f1) / n_serial)
+    # The same batch served alone by a context with the library defaults (the chunked multi-CTA scan for
+    # long windows, the whole grid for the mover): a single batch's latency and its stage shares.
+    ctx_l = crk.Context(local)
+    idx_l = ctx_l.index(max_rings=args.streams, **workload.INDEX_SHAPE)
+    for _ in range(3):
+        workload.serve_step(idx_l, s0.ep, stream=s0.stream)
+    torch.cuda.synchronize()
+    crk.profile_enable(True)
+    f0.record(s0.stream)
+    for _ in range(n_serial):
+        workload.serve_step(idx_l, s0.ep, stream=s0.stream)
+    f1.record(s0.stream)
+    torch.cuda.synchronize()
+    prof_l = crk.profile_read()
+    crk.profile_enable(False)
+    lone = {"ms_per_step": round(max_over_ranks(f0.elapsed_time(f1) / n_serial), 4),
+            "stages_ms_per_step": {k: round(v[0] / max(1, v[1]), 4) for k, v in prof_l.items()},
+            "stage_share": {k: round(v[0] / max(1e-9, sum(x[0] for x in prof_l.values())), 4)
+                            for k, v in prof_l.items()},
+            "scan_stats": idx_l.scan_stats(),
+            "config": "library defaults (chunked multi-CTA scan of long windows, whole-grid mover), one batch "
+                      "at a time"}
+    lone["value"] = round(sum_over_ranks(ep.payload) / (lone["ms_per_step"] / 1e3) / 1e9, 2)
+    del idx_l, ctx_l
 
     # roofline of the dominant kernel (the mover): algorithmic HBM bytes per launch / its event time
     mv_ms, mv_n = prof["move"]
@@ -477,7 +501,7 @@ def main():
                                                 "timed region (a lower bound: the step also holds scan/parse/plan)"},
                      "mover_config": {k: ctx_kw.get(k) for k in ("mover_reserve_ctas", "mover_tail_tiles", "mover_run")}},
         "wire_gbs": round(sum_over_ranks(ep.wire_in + ep.reply_wire) / (ms_max / 1e3) / 1e9, 2),
-        "pipeline": P, "serial_ms_per_step": round(serial_ms, 4),
+        "pipeline": P, "serial_ms_per_step": round(serial_ms, 4), "lone_batch": lone,
         "serial_value": round(payload_all / (serial_ms / 1e3) / 1e9, 2),
         "stages_ms_per_step": {k: round(v[0] / max(1, v[1]), 4) for k, v in prof.items()},
         "stage_share": stage_share,

@@ -123,10 +123,13 @@ class Slot:
     res: "crk.PinnedResults | None" = None
 
 
-# Mover settings of the pipelined server loop (bench.py's timed configuration): with batches in flight the
-# mover leaves 16 CTA slots free, so the next batch's front-end kernels and the start of its mover overlap
-# this one, and claims whole runs to the end (its CTAs retire staggered, handing SMs over gradually).
-PIPELINE_CTX = {"mover_reserve_ctas": 16, "mover_tail_tiles": 0}
+# Settings of the pipelined server loop (bench.py's timed configuration): with batches in flight the mover
+# leaves 16 CTA slots free, so the next batch's front-end kernels and the start of its mover overlap this one,
+# and claims whole runs to the end (its CTAs retire staggered, handing SMs over gradually).  The front end
+# uses the one-CTA-per-ring scan there: it runs inside those 16 free slots while the previous batch's mover
+# streams, whereas the chunked scan needs ~2 CTAs on every SM and would wait for the mover to leave
+# (measured: 0.374 vs 0.335 ms per C5 step).  A batch served alone (latency) takes the chunked scan.
+PIPELINE_CTX = {"mover_reserve_ctas": 16, "mover_tail_tiles": 0, "scan_chunking": 1}
 INDEX_SHAPE = dict(max_frags=1 << 20, max_records=1 << 14)  # per endpoint (16 rings): > kSmallServe records
 
 

@@ -72,7 +72,7 @@ def test_bench_pipelined_loop_matches_oracle(direction):
     import bench
     dev = torch.device("cuda:0")
     ctx_kw = workload.pipelined_ctx_kw({}, P)
-    assert ctx_kw == {"mover_reserve_ctas": 16, "mover_tail_tiles": 0}
+    assert ctx_kw == {"mover_reserve_ctas": 16, "mover_tail_tiles": 0, "scan_chunking": 1}
     frac = bench.H2D_FRAC[direction]
     slots = workload.build_slots(0, 0, dev, P, ctx_kw, n_streams=16, payload_per_stream=64 * MiB, h2d_frac=frac,
                                  default_stream=torch.cuda.current_stream(dev))
