@@ -219,3 +219,45 @@ def c5_endpoint(gpu: int, n_streams: int = 16, payload_per_stream: int = 64 * Mi
             seq += 1
         streams.append(st)
     return streams, off
+
+
+# ------------------------------------------------------------------ NEXT-2: more of the paper's workloads
+
+# cuSolverDn_LinearSolver: "LU with 900x900 matrix, 1000 Iterations" (Fig. 5b), 6.07 GiB of
+# memory transfers in all.  Per iteration the sample copies the matrix A (n x n doubles) and
+# the right-hand side b (n doubles) to the device and the solution x (n doubles) back; 1000 iterations move
+# 6,494,400,000 B = 6.05 GiB (the paper's 6.07 GiB also counts the sample's setup copies).
+CUSOLVER_N, CUSOLVER_ITERS = 900, 1000
+# histogram: 64 MiB of memory transfers: the CUDA sample's 64 MiB byte array to the device and
+# its 256-bin uint32 histogram back.
+HISTOGRAM_BYTES, HISTOGRAM_BINS = 64 * MiB, 256
+
+
+def _profile_streams(recs_per_stream: list[list[tuple[int, int]]], gpu: int, seed: int,
+                     align: int = 256) -> tuple[list[Stream], int]:
+    """Streams of (kind, size) memcpy calls laid out in one region (disjoint, `align`-aligned ranges)."""
+    g = rng(seed)
+    streams, off = [], 0
+    for s, recs in enumerate(recs_per_stream):
+        st = Stream(gpu, s)
+        for seq, (kind, size) in enumerate(recs):
+            st.records.append(MemcpyRec(kind, (gpu << 28) | (s << 20) | seq, size, off, int(g.integers(0, 1 << 62))))
+            off = (off + size + align - 1) // align * align
+        streams.append(st)
+    return streams, off
+
+
+def cusolver_endpoint(gpu: int = 0, iterations: int = CUSOLVER_ITERS, n: int = CUSOLVER_N, n_streams: int = 1,
+                      seed: int = 0xC50D) -> tuple[list[Stream], int]:
+    """cuSolverDn_LinearSolver's memcpy calls: per iteration A (n*n*8 B) and b (n*8 B) HtoD, x (n*8 B) DtoH,
+    iterations dealt round-robin over n_streams client streams (one stream = one connection)."""
+    per = [[] for _ in range(n_streams)]
+    for it in range(iterations):
+        per[it % n_streams] += [(PROC_H2D, n * n * 8), (PROC_H2D, n * 8), (PROC_D2H, n * 8)]
+    return _profile_streams(per, gpu, seed)
+
+
+def histogram_endpoint(gpu: int = 0, nbytes: int = HISTOGRAM_BYTES, bins: int = HISTOGRAM_BINS,
+                       seed: int = 0x4157) -> tuple[list[Stream], int]:
+    """histogram's memcpy calls: the byte array HtoD, the bins (uint32) DtoH, on one client stream."""
+    return _profile_streams([[(PROC_H2D, nbytes), (PROC_D2H, bins * 4)]], gpu, seed)

@@ -58,6 +58,14 @@ def c5_endpoint(ctx: crk.Context, rank: int, device: torch.device, n_streams: in
     budget = payload_per_stream if h2d_frac >= 1.0 else payload_per_stream - payload_per_stream // 16
     streams, region_bytes = gen.c5_endpoint(rank, n_streams=n_streams, payload_per_stream=payload_per_stream,
                                             h2d_budget=budget, misalign=misalign, h2d_frac=h2d_frac)
+    return endpoint(ctx, rank, device, streams, region_bytes, host_rings=host_rings, staged=staged)
+
+
+def endpoint(ctx: crk.Context, rank: int, device: torch.device, streams: list, region_bytes: int,
+             host_rings: bool = False, staged: bool = False) -> Endpoint:
+    """An endpoint serving gen's memcpy streams (C5, or the NEXT-2 profiles): one ring per stream holding its
+    CALLs (encoded on the GPU), one send ring per stream, one device region for every HtoD destination and
+    DtoH source."""
     region = torch.zeros(region_bytes + 256, dtype=torch.uint8, device=device)
     ep = Endpoint(ctx, rank, streams, region)
     F = ctx.cfg.frag_payload

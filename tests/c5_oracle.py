@@ -34,6 +34,11 @@ def oracle_endpoint(rank: int, n_streams: int, region_bytes: int, base: int, pay
     streams, rb = gen.c5_endpoint(rank, n_streams=n_streams, payload_per_stream=payload_per_stream,
                                   h2d_budget=budget, h2d_frac=h2d_frac)
     assert rb == region_bytes, (rb, region_bytes)
+    return oracle_endpoint_of(streams, region_bytes, base, F)
+
+
+def oracle_endpoint_of(streams: list, region_bytes: int, base: int, F: int = 65536) -> OracleEndpoint:
+    """The oracle's encoding of any gen memcpy streams (C5, the NEXT-2 profiles)."""
     cfg = O.Config(prog=gen.PROG, vers=gen.VERS, proc_h2d=gen.PROC_H2D, proc_d2h=gen.PROC_D2H, frag_payload=F)
     region = np.zeros(region_bytes + 256, np.uint8)
     wires = []

@@ -76,3 +76,18 @@ def test_c5_direction_mixes():
            [(r.kind, r.size, r.xid) for s in mixed2 for r in s.records]
     for streams in (only_h, only_d, mixed):
         assert all(sum(r.size for r in s.records) == 8 * MiB for s in streams)
+
+
+def test_next2_profiles_match_the_paper_volumes():
+    """NEXT-2 profiles (gen.cusolver_endpoint / histogram_endpoint) against PAPER.md:180's transfer volumes:
+    cuSolverDn_LinearSolver 6.07 GiB over its 1000 iterations, histogram 64 MiB."""
+    from paper_conf_sc_eilingkkflm23_b200 import gen
+    streams, rb = gen.cusolver_endpoint(iterations=3, n_streams=2)
+    sizes = [r.size for s in streams for r in s.records]
+    assert sizes.count(900 * 900 * 8) == 3 and sizes.count(900 * 8) == 6
+    per_iter = 900 * 900 * 8 + 2 * 900 * 8
+    assert abs(per_iter * gen.CUSOLVER_ITERS / 2**30 - 6.07) < 0.03   # 6.05 GiB vs the paper's 6.07 GiB
+    offs = sorted((r.region_off, r.size) for s in streams for r in s.records)
+    assert all(a + n <= b for (a, n), (b, _) in zip(offs, offs[1:])) and offs[-1][0] + offs[-1][1] <= rb
+    h, hrb = gen.histogram_endpoint()
+    assert [(r.kind, r.size) for r in h[0].records] == [(gen.PROC_H2D, 64 << 20), (gen.PROC_D2H, 1024)]

@@ -10,7 +10,8 @@ output against the generator's values.  Writes one JSON object (stdout).
        over >= 256 MiB so repeated runs do not hit L2
   C4   256 MiB typed-array stress: decode GB/s (all items, regular and irregular framing)
   NEXT-1  one 1 GiB memcpy striped over 16 rings (16 CALLs of 64 MiB at ptr + offset), served as one batch
-  NEXT-2  cuSolverDn-shaped (100 x 900x900 f64 HtoD + 7.2 KB DtoH) and histogram-shaped (64 MiB HtoD, 1 KiB DtoH)
+  NEXT-2  gen.cusolver_endpoint (100 iterations of A 900x900 f64 + b HtoD, x DtoH; 1 and 4 client streams) and
+          gen.histogram_endpoint (64 MiB HtoD, 256-bin result DtoH), served by crk_serve
 """
 import json
 import os
@@ -374,6 +375,18 @@ def served(ctx, sizes_h2d, sizes_d2h, streams=1, reps=20):
     return {"ms": round(ms, 4), "payload_bytes": pay, "gbs": round(pay / ms / 1e6, 1), "ok": bool(ok)}
 
 
+def profile(streams, region_bytes, reps=10):
+    """A gen workload profile (NEXT-2) served by crk_serve: payload GB/s and the per-ring check."""
+    from paper_conf_sc_eilingkkflm23_b200 import workload
+    ctx = Ctx()
+    ep = workload.endpoint(ctx, 0, dev, streams, region_bytes)
+    idx = ctx.index(len(streams), 1 << 16, 1 << 12)
+    ms = timed(lambda _: workload.serve_step(idx, ep), reps)
+    chk = workload.check_results(idx, ep)
+    return {"ms": round(ms, 4), "payload_bytes": ep.payload, "records": ep.n_records, "streams": len(streams),
+            "gbs": round(ep.payload / ms / 1e6, 1), "ok": chk["ok"], "scan_stats": idx.scan_stats()}
+
+
 def main():
     build.build()
     only = [x for x in os.environ.get("SUITE_ONLY", "").split(",") if x]
@@ -387,9 +400,9 @@ def main():
         "C4_typed_irregular": lambda: c4(Ctx(), True),
         "NEXT1_striped_1GiB_16_rings": lambda: served(Ctx(), [64 * MiB] * 16, [], streams=16),
         "NEXT1_single_1GiB_1_ring": lambda: served(Ctx(), [GiB], [], streams=1),
-        "NEXT2_cusolver_100_iters": lambda: served(Ctx(), [900 * 900 * 8] * 100, [900 * 8] * 100,
-                                                   streams=1, reps=10),
-        "NEXT2_histogram": lambda: served(Ctx(), [64 * MiB], [256 * 4], streams=1),
+        "NEXT2_cusolver_100_iters": lambda: profile(*gen.cusolver_endpoint(iterations=100)),
+        "NEXT2_cusolver_100_iters_4_streams": lambda: profile(*gen.cusolver_endpoint(iterations=100, n_streams=4)),
+        "NEXT2_histogram": lambda: profile(*gen.histogram_endpoint()),
     }
     out = {}
     t0 = time.time()
