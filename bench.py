@@ -51,6 +51,8 @@ def parse_args():
     p.add_argument("--e2e-pipeline", type=int, default=3, help="batches in flight for the host-memory runs")
     p.add_argument("--e2e-copy-streams", type=int, default=1, help="streams per direction for the staged ring DMAs")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-sweep", action="store_true", help="skip the C3 / C2 host-link sweeps")
+    p.add_argument("--sweep-log2", default="12-30", help="C3 sweep sizes as log2 range, e.g. 12-30")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
     p.add_argument("--ctx", default="", help="crk_config overrides, e.g. scan_threads=128,tile_bytes=32768")
@@ -481,6 +483,13 @@ def main():
         modes.sort(key=lambda m: -m["value"] if m["check"]["ok"] else 0)
         e2e = dict(modes[0])
         e2e["other_modes"] = [{k: m[k] for k in ("value", "mode", "ms_per_step", "check")} for m in modes[1:]]
+        del hslots, loop, ep_h
+        torch.cuda.empty_cache()
+    sweep = None
+    if not args.no_sweep:
+        if e2e is None:
+            link = host_link_peaks(dev)
+        sweep = run_sweep(args, dev, link)
 
     out = {
         "metric": "xdr_memcpy_serve_payload_GBps", "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
@@ -510,6 +519,7 @@ def main():
         "gpu_launches": launches, "check": check, "host_numa": numa,
         "clocks": clk.summary(),
         "e2e": e2e,
+        "sweep": sweep,
     }
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(args, args.cpu_seconds)
@@ -518,6 +528,68 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def run_sweep(args, dev, link) -> dict:
+    """The paper-shaped host-link sweeps through pinned host rings (PAPER.md:232-236
+    bandwidthTest, PAPER.md:180 matrixMul): per size and direction, end-to-end GB/s of copy-engine staged (ce) and
+    zero-copy (zc) serving, the faster one, and its wire bytes as a fraction of the measured copy-engine link in
+    that direction (`link`, measured in this run).  workload.LinkSweep documents what one call includes."""
+    import torch
+    from paper_conf_sc_eilingkkflm23_b200 import gen, workload
+    lo, hi = (int(x) for x in args.sweep_log2.split("-"))
+    sizes = list(range(lo, hi + 1))
+    sw = workload.LinkSweep(dev.index, dev, max_n=1 << max(max(sizes), 21))
+    main = torch.cuda.current_stream(dev)
+    points = []
+    for lg in sizes:
+        n = 1 << lg
+        payload = torch.from_numpy(gen.c3_payload(lg)).to(dev)
+        runs = min(400, max(10, -(-(1 << 30) // n)))  # >= 10 runs (PAPER.md:232), ~1 GiB moved when affordable
+        pt = {"log2n": lg, "bytes": n, "runs": runs}
+        for direction, peak in (("h2d", link["ce_h2d_gbs"]), ("d2h", link["ce_d2h_gbs"])):
+            sw.prepare(n, direction, payload)
+            res = {}
+            for mode in ("ce", "zc"):
+                sw.run(mode, 3, main)
+                ms = sw.run(mode, runs, main)
+                wire = sw.slots[0].w_in if direction == "h2d" else sw.slots[0].w_out
+                wg = wire * runs / ms / 1e6
+                res[mode] = {"gbs": round(n * runs / ms / 1e6, 3), "wire_gbs": round(wg, 3),
+                             "us_per_call": round(ms * 1e3 / runs, 2), "frac": round(wg / peak, 4),
+                             "ok": sw.check(payload)}
+            best = max(res, key=lambda m: res[m]["gbs"] if res[m]["ok"] else -1)
+            pt[direction] = {"best": best, "gbs": res[best]["gbs"], "frac": res[best]["frac"],
+                             "ok": res["ce"]["ok"] and res["zc"]["ok"], **res}
+        points.append(pt)
+        del payload
+    cutoff = None
+    for pt in reversed(points):
+        if pt["h2d"]["frac"] >= 0.8 and pt["d2h"]["frac"] >= 0.8:
+            cutoff = pt["bytes"]
+        else:
+            break
+    # C2: the matrixMul batch (two HtoD CALLs, one DtoH) served as one step
+    sw.prepare_c2()
+    w_in, w_out = sw.slots[0].w_in, sw.slots[0].w_out
+    bound_ms = max(w_in / link["ce_h2d_gbs"], w_out / link["ce_d2h_gbs"], (w_in + w_out) / link["ce_bidir_gbs"]) / 1e6
+    c2 = {"payload_bytes": 2_048_000, "wire_in": w_in, "wire_out": w_out, "link_bound_us": round(bound_ms * 1e3, 2)}
+    for mode in ("ce", "zc"):
+        sw.run(mode, 5, main)
+        ms = sw.run(mode, 200, main) / 200
+        c2[mode] = {"us_per_batch": round(ms * 1e3, 2), "gbs": round(2_048_000 / ms / 1e6, 3),
+                    "frac": round(bound_ms / ms, 4), "ok": sw.check(None)}
+    c2["best"] = max(("ce", "zc"), key=lambda m: c2[m]["gbs"] if c2[m]["ok"] else -1)
+    del sw
+    torch.cuda.empty_cache()
+    return {"c3": points, "c2_matrixMul": c2,
+            "cutoff_bytes_frac_ge_0.8": cutoff,
+            "link": {k: link[k] for k in ("ce_h2d_gbs", "ce_d2h_gbs", "ce_bidir_gbs")},
+            "how": "one memcpy CALL per run (bandwidthTest), 2 calls in flight; ce = crk_ring_copy in + crk_serve from "
+                   "HBM + crk_ring_copy out; zc = crk_serve on the pinned rings; each run includes the host->device "
+                   "copy of its CALL and the device->host copy of its REPLY; CUDA events around all runs of a size; "
+                   "frac = wire bytes in that direction / time / measured copy-engine link (C2: link-bound time / "
+                   "time)"}
 
 
 def host_link_peaks(dev, nbytes: int = 512 * MiB) -> dict:

@@ -223,6 +223,13 @@ class HostBuffer:
             pass
 
 
+class _HostView:
+    """Part of a HostBuffer (keeps the buffer alive); `.np` views the part."""
+
+    def __init__(self, buf, np_view):
+        self.buf, self.np = buf, np_view
+
+
 @dataclass
 class Ring:
     """A ring: `cap` (power of two >= 256) bytes of device memory or pinned mapped host memory."""
@@ -247,11 +254,19 @@ class Ring:
     def c(self) -> CRing:
         return CRing(self.base, self.cap)
 
+    def sub(self, offset: int, cap: int) -> "Ring":
+        """A ring over bytes [offset, offset + cap) of this one's memory (offset 256-aligned, cap a power of two)."""
+        assert offset % 256 == 0 and offset + cap <= self.cap and cap & (cap - 1) == 0
+        if isinstance(self.owner, torch.Tensor):
+            return Ring(self.base + offset, cap, self.owner[offset:offset + cap])
+        view = _HostView(self.owner, self.host_view()[offset:offset + cap])
+        return Ring(self.base + offset, cap, view)
+
     def tensor(self) -> torch.Tensor | None:
         return self.owner if isinstance(self.owner, torch.Tensor) else None
 
     def host_view(self) -> np.ndarray | None:
-        return self.owner.np if isinstance(self.owner, HostBuffer) else None
+        return self.owner.np if isinstance(self.owner, (HostBuffer, _HostView)) else None
 
     def read(self, cursor: int, n: int) -> bytes:
         """Bytes [cursor, cursor + n) with wrap (host-side inspection, for tests)."""

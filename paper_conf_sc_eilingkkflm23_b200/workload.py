@@ -328,3 +328,146 @@ def check_results(idx: crk.Index, ep: Endpoint) -> dict:
             ok &= bool(torch.equal(ep.region[r.region_off:r.region_off + r.size], want))
             sampled += 1
     return dict(ok=bool(ok), sampled_h2d_records=sampled)
+
+
+# ------------------------------------------------------------------ host-link sweeps (C3, C2) through host rings
+
+class LinkSweep:
+    """bandwidthTest-shaped end-to-end runs through pinned host rings:
+    one memcpy CALL of n bytes per run, HtoD (the CALL carries the payload; the 32-byte REPLY goes back) or DtoH
+    (a 64-byte CALL; the framed payload REPLY goes back), `slots` calls in flight (consecutive calls alternate
+    between slots, so one call's copies overlap the previous call's kernels).  Two ways to serve a call:
+      ce: crk_ring_copy DMAs the receive window into a device ring, crk_serve runs from HBM into a device send
+          ring, crk_ring_copy DMAs the reply bytes out (copy engines for the host link);
+      zc: crk_serve reads the pinned receive ring and writes the pinned send ring over the link (zero-copy).
+    Every run includes the host -> device copy of its CALL and the device -> host copy of its REPLY; the times
+    are CUDA events on the launching streams around all runs of a size."""
+
+    def __init__(self, device_index: int, device: torch.device, max_n: int = 1 << 30, slots: int = 2, **ctx_kw):
+        # one context per slot: a context's scratch serves one call at a time (include/crk.h)
+        ctxs = [crk.Context(device_index, **ctx_kw) for _ in range(slots)]
+        self.ctx, self.dev, F = ctxs[0], device, ctxs[0].cfg.frag_payload
+        self.big = next_pow2(max_n + 64 + 4 * (max_n // F + 2))  # a ring for the larger side of any call
+        self.slots = []
+        for ctx in ctxs:
+            sl = type("SweepSlot", (), {})()
+            sl.ctx = ctx
+            sl.host_big = crk.Ring.host(self.big)
+            sl.host_small = crk.Ring.host(4096)
+            sl.dev_big = crk.Ring.device(self.big, device)
+            sl.dev_small = crk.Ring.device(4096, device)
+            sl.region = torch.zeros(max_n + 256, dtype=torch.uint8, device=device)
+            sl.idx = ctx.index(1, (max_n >> 15) + 64, 16)
+            sl.stream, sl.in_s, sl.out_s = (torch.cuda.Stream(device) for _ in range(3))
+            sl.ev_in, sl.ev_served, sl.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
+            self.slots.append(sl)
+
+    def _sub(self, ring: crk.Ring, cap: int) -> crk.Ring:
+        return ring.sub(0, cap)
+
+    def prepare(self, n: int, direction: str, payload: torch.Tensor):
+        """Encodes the CALL of each slot (setup, outside the timed region): HtoD carries `payload`, DtoH reads it
+        from the slot's region."""
+        F = self.ctx.cfg.frag_payload
+        self.n, self.direction = n, direction
+        for i, sl in enumerate(self.slots):
+            base = sl.region.data_ptr()
+            if direction == "h2d":
+                stage = self._sub(sl.dev_big, self.big)
+                w = sl.ctx.encode_call(0x5E0000 + i, gen.PROC_H2D, [(crk.K_U64, base), (crk.K_OPAQUE_VAR, payload),
+                                                                     (crk.K_U64, n)], stage, 0)
+                torch.cuda.synchronize(self.dev)
+                crk.ring_copy(sl.host_big, sl.dev_big, 0, w)
+                sl.rx_host, sl.rx_dev, sl.w_in = sl.host_big, sl.dev_big, w
+                sl.tx_host, sl.tx_dev, sl.w_out = sl.host_small, sl.dev_small, crk.wire_size_d2h(0, 1, F)
+            else:
+                sl.region[:n].copy_(payload)
+                w = sl.ctx.encode_call(0x5D0000 + i, gen.PROC_D2H, [(crk.K_U64, base), (crk.K_U64, n)], sl.dev_small, 0)
+                torch.cuda.synchronize(self.dev)
+                crk.ring_copy(sl.host_small, sl.dev_small, 0, w)
+                sl.rx_host, sl.rx_dev, sl.w_in = sl.host_small, sl.dev_small, w
+                sl.tx_host, sl.tx_dev, sl.w_out = sl.host_big, sl.dev_big, crk.wire_size_d2h(n, 0, F)
+            sl.ev_served.record(sl.stream)
+            sl.ev_out.record(sl.out_s)
+        torch.cuda.synchronize(self.dev)
+
+    def prepare_c2(self):
+        """The matrixMul batch: A (409,600 B of 1.0f) and B (819,200 B of 0.01f)
+        HtoD and C (819,200 B of 3.2f) DtoH, three CALLs served as one batch; wire in 1,229,060 B, out 819,348 B."""
+        F = self.ctx.cfg.frag_payload
+        A, B, Cm = (torch.from_numpy(x.view(np.uint8).copy()).to(self.dev) for x in gen.c2_matrices())
+        self.direction, self.c2 = "c2", (A, B, Cm)
+        half = self.big // 2
+        for i, sl in enumerate(self.slots):
+            base = sl.region.data_ptr()
+            offA, offB, offC = 0, 409_600, 409_600 + 819_200
+            sl.region[offC:offC + Cm.numel()].copy_(Cm)
+            rx_dev, tx_dev = sl.dev_big.sub(0, 1 << 21), sl.dev_big.sub(half, 1 << 20)
+            rx_host, tx_host = sl.host_big.sub(0, 1 << 21), sl.host_big.sub(half, 1 << 20)
+            w = 0
+            for xid, kind, items in ((0xC2A, gen.PROC_H2D, [(crk.K_U64, base + offA), (crk.K_OPAQUE_VAR, A),
+                                                            (crk.K_U64, A.numel())]),
+                                     (0xC2B, gen.PROC_H2D, [(crk.K_U64, base + offB), (crk.K_OPAQUE_VAR, B),
+                                                            (crk.K_U64, B.numel())]),
+                                     (0xC2C, gen.PROC_D2H, [(crk.K_U64, base + offC), (crk.K_U64, Cm.numel())])):
+                w += sl.ctx.encode_call(xid, kind, items, rx_dev, w)
+            torch.cuda.synchronize(self.dev)
+            crk.ring_copy(rx_host, rx_dev, 0, w)
+            sl.rx_host, sl.rx_dev, sl.w_in = rx_host, rx_dev, w
+            sl.tx_host, sl.tx_dev = tx_host, tx_dev
+            sl.w_out = 2 * crk.wire_size_d2h(0, 1, F) + crk.wire_size_d2h(Cm.numel(), 0, F)
+            sl.ev_served.record(sl.stream)
+            sl.ev_out.record(sl.out_s)
+        torch.cuda.synchronize(self.dev)
+
+    def run(self, mode: str, runs: int, main) -> float:
+        """`runs` calls in `mode` ("ce" / "zc"); returns device ms over all of them (events on `main`)."""
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(main)
+        for sl in self.slots:
+            for st in (sl.stream, sl.in_s, sl.out_s):
+                st.wait_event(e0)
+        for k in range(runs):
+            sl = self.slots[k % len(self.slots)]
+            base, nb = sl.region.data_ptr(), sl.region.numel()
+            if mode == "ce":
+                sl.in_s.wait_event(sl.ev_served)
+                crk.ring_copy(sl.rx_dev, sl.rx_host, 0, sl.w_in, stream=sl.in_s)
+                sl.ev_in.record(sl.in_s)
+                sl.stream.wait_event(sl.ev_in)
+                sl.stream.wait_event(sl.ev_out)
+                sl.idx.serve([(sl.rx_dev, 0, sl.w_in)], [sl.tx_dev], [0], base, nb, stream=sl.stream)
+                sl.ev_served.record(sl.stream)
+                sl.out_s.wait_event(sl.ev_served)
+                crk.ring_copy(sl.tx_host, sl.tx_dev, 0, sl.w_out, stream=sl.out_s)
+                sl.ev_out.record(sl.out_s)
+            else:
+                sl.idx.serve([(sl.rx_host, 0, sl.w_in)], [sl.tx_host], [0], base, nb, stream=sl.stream)
+        for sl in self.slots:
+            for st in (sl.stream, sl.in_s, sl.out_s):
+                ev = torch.cuda.Event()
+                ev.record(st)
+                main.wait_event(ev)
+        e1.record(main)
+        torch.cuda.synchronize(self.dev)
+        return e0.elapsed_time(e1)
+
+    def check(self, payload: torch.Tensor) -> bool:
+        """Every slot's last call served OK: HtoD destinations == payload; DtoH: the reply's size and, past its
+        first fragment header and the 32-byte REPLY prefix, the payload's first bytes."""
+        ok = True
+        for sl in self.slots:
+            r = sl.idx.ring_results(1)[0]
+            ok &= r["status"] == crk.OK and r["reply_bytes"] == sl.w_out
+            if self.direction == "c2":
+                A, B, Cm = self.c2
+                ok &= bool(torch.equal(sl.region[:A.numel()], A)) and bool(
+                    torch.equal(sl.region[409_600:409_600 + B.numel()], B))
+                # C's reply follows the two 32-byte HtoD replies: its payload starts 36 bytes in
+                ok &= sl.tx_host.read(64 + 36, 1024) == bytes(Cm[:1024].cpu().numpy())
+            elif self.direction == "h2d":
+                ok &= bool(torch.equal(sl.region[:self.n], payload))
+            else:
+                k = min(self.n, 1024)
+                ok &= sl.tx_host.read(36, k) == bytes(payload[:k].cpu().numpy())
+        return bool(ok)

@@ -16,6 +16,10 @@
 #include <vector>
 #include <algorithm>
 #include <string>
+#include <atomic>
+#include <chrono>
+#include <cstring>
+#include <thread>
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { \
   fprintf(stderr, "CUDA %s at %s:%d: %s\n", #x, __FILE__, __LINE__, cudaGetErrorString(e)); exit(1);} } while (0)
@@ -124,7 +128,82 @@ static Stat time_it(F f, double bytes, int warm = 3, int reps = 10) {
   return summarize(ms, bytes);
 }
 
+// All-GPUs-at-once mode (the 8-GPU roofline is the CONCURRENTLY measured aggregate, not
+// 8x one GPU): one host thread per device, each with its own pinned buffers (allocated by that thread after it
+// has bound to its device), a spin barrier before every measurement, copy-engine H2D, D2H and both at once on
+// all devices together.  Per device: GB/s from its own CUDA events; aggregate: all bytes / the wall-clock span
+// from the barrier to the last device's completion.
+static void concurrent(int ngpu, size_t n, int reps) {
+  std::atomic<int> arrived{0};
+  std::atomic<int> gen{0};
+  auto barrier = [&](int parties) {
+    const int g = gen.load();
+    if (arrived.fetch_add(1) + 1 == parties) { arrived.store(0); gen.fetch_add(1); }
+    else while (gen.load() == g) std::this_thread::yield();
+  };
+  struct Res { double h2d, d2h, bi; };
+  std::vector<Res> res(ngpu);
+  double wall[3] = {0, 0, 0};
+  std::vector<std::thread> th;
+  for (int g = 0; g < ngpu; ++g) {
+    th.emplace_back([&, g] {
+      CK(cudaSetDevice(g));
+      uint8_t *h_a, *h_b, *d_a, *d_b;
+      CK(cudaHostAlloc(&h_a, n, cudaHostAllocPortable));
+      CK(cudaHostAlloc(&h_b, n, cudaHostAllocPortable));
+      memset(h_a, 1, n); memset(h_b, 2, n);
+      CK(cudaMalloc(&d_a, n)); CK(cudaMalloc(&d_b, n));
+      cudaStream_t s1, s2;
+      CK(cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking)); CK(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+      cudaEvent_t a, b, c; CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b)); CK(cudaEventCreate(&c));
+      for (int test = 0; test < 3; ++test) {
+        double best = 0;
+        for (int r = 0; r < reps + 1; ++r) {
+          CK(cudaDeviceSynchronize());
+          barrier(ngpu);
+          const auto t0 = std::chrono::steady_clock::now();
+          CK(cudaEventRecord(a, s1));
+          CK(cudaStreamWaitEvent(s2, a));
+          if (test != 1) CK(cudaMemcpyAsync(d_a, h_a, n, cudaMemcpyHostToDevice, s1));
+          if (test != 0) CK(cudaMemcpyAsync(h_b, d_b, n, cudaMemcpyDeviceToHost, s2));
+          CK(cudaEventRecord(c, s2));
+          CK(cudaStreamWaitEvent(s1, c));
+          CK(cudaEventRecord(b, s1));
+          CK(cudaEventSynchronize(b));
+          const double span = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+          float ms; CK(cudaEventElapsedTime(&ms, a, b));
+          const double bytes = test == 2 ? 2.0 * n : (double)n;
+          if (r > 0) best = std::max(best, bytes / (ms * 1e-3) / 1e9);  // r = 0 is the warm-up
+          barrier(ngpu);
+          if (g == 0 && r > 0) wall[test] = std::max(wall[test], bytes * ngpu / span / 1e9);
+        }
+        (test == 0 ? res[g].h2d : test == 1 ? res[g].d2h : res[g].bi) = best;
+      }
+      cudaFreeHost(h_a); cudaFreeHost(h_b); cudaFree(d_a); cudaFree(d_b);
+    });
+  }
+  for (auto& t : th) t.join();
+  printf("{\"mode\": \"all_gpus_concurrent\", \"gpus\": %d, \"bytes\": %zu, \"per_gpu\": [", ngpu, n);
+  double sh = 0, sd = 0, sb = 0;
+  for (int g = 0; g < ngpu; ++g) {
+    printf("%s{\"gpu\": %d, \"ce_h2d_gbs\": %.2f, \"ce_d2h_gbs\": %.2f, \"ce_bidir_gbs\": %.2f}", g ? ", " : "", g,
+           res[g].h2d, res[g].d2h, res[g].bi);
+    sh += res[g].h2d; sd += res[g].d2h; sb += res[g].bi;
+  }
+  printf("], \"sum_of_per_gpu\": {\"ce_h2d_gbs\": %.2f, \"ce_d2h_gbs\": %.2f, \"ce_bidir_gbs\": %.2f}, "
+         "\"aggregate_wall\": {\"ce_h2d_gbs\": %.2f, \"ce_d2h_gbs\": %.2f, \"ce_bidir_gbs\": %.2f}}\n",
+         sh, sd, sb, wall[0], wall[1], wall[2]);
+}
+
 int main(int argc, char** argv) {
+  if (argc > 1 && std::string(argv[1]) == "--all") {  // host_link_probe --all [ngpu] [bytes]
+    int ndev = 0;
+    CK(cudaGetDeviceCount(&ndev));
+    const int ngpu = argc > 2 ? std::min(ndev, atoi(argv[2])) : ndev;
+    const size_t bytes = argc > 3 ? strtoull(argv[3], 0, 0) : (size_t)256 << 20;
+    concurrent(std::max(1, ngpu), bytes, 5);
+    return 0;
+  }
   size_t n = (argc > 1 ? strtoull(argv[1], 0, 0) : (size_t)1 << 30);
   int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
   cudaDeviceProp prop; CK(cudaGetDeviceProperties(&prop, 0));
