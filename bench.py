@@ -20,7 +20,8 @@ send rings (K6), i.e. every §8(a) row the memcpy path has.
   --direction h2d|d2h: the HtoD-only / DtoH-only call mixes of the same endpoint
 
 Launch: python bench.py [--gpus N --steps K --warmup W]; N > 1 under torch.distributed.run (one rank per
-GPU, NCCL only for the barrier and the max-over-ranks of the timings; the data path has no collective).
+GPU; a CPU gloo group for the barrier and the max-over-ranks of the timings -- no NCCL: the data path has no
+collective).
 """
 from __future__ import annotations
 
@@ -296,17 +297,12 @@ def main():
 
     world, rank, local = parallel.rank_env()
     ndev = torch.cuda.device_count()
-    shared_gpu = world > ndev  # more ranks than GPUs (plumbing tests): ranks share devices, gloo plumbing
-    local = local % ndev
-    if world > 1:
-        if shared_gpu:
-            dist.init_process_group("gloo")
-        else:
-            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    local = local % ndev  # more ranks than GPUs (plumbing runs): ranks share devices
+    parallel.init(world)  # gloo on the CPU: barrier + timing reductions only, no NCCL (north_star)
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
     numa = parallel.bind_numa(local)  # before any pinned host allocation
-    red_dev = "cpu" if shared_gpu else dev
+    red_dev = "cpu"
     build.build()
 
     ctx_kw = {k: int(v, 0) for k, v in (kv.split("=") for kv in args.ctx.split(",") if kv)}
@@ -416,7 +412,9 @@ def main():
         del slots
         torch.cuda.empty_cache()
         # host-link peaks (copy engine, pinned) measured before the rings are allocated (their buffers get
-        # the same placement the rings get) and again after the runs; the roofline takes the better of the two
+        # the same placement the rings get) and again after the runs; the roofline takes the better of the two.
+        # Every rank measures at the same time (after a barrier): with N GPUs the links share the host.
+        barrier()
         link0 = host_link_peaks(dev)
         P = max(1, args.e2e_pipeline)  # batches in flight for the host-memory runs
         hslots = workload.build_slots(local, rank, dev, P, ctx_kw, n_streams=args.streams,
@@ -455,10 +453,15 @@ def main():
         res_bytes = len(ep_h.rings) * 40
         e2e_v = sum_over_ranks(ep_h.payload) * args.e2e_steps / el_max / 1e9
         # live host-link peaks (copy engine, pinned) for the e2e roofline
+        barrier()
         link1 = host_link_peaks(dev)
         link = {k: max(link0[k], link1[k]) for k in link0}
-        link["measured"] = "best of two measurements (before allocating the rings, after the runs)"
+        link["measured"] = ("best of two measurements (before allocating the rings, after the runs), every rank "
+                            "at once after a barrier")
         link["before"], link["after"] = link0, link1
+        links = parallel.gather({k: link[k] for k in link0})
+        wires = parallel.gather((ep_h.wire_in, ep_h.reply_wire))
+        link_job = parallel.link_aggregate(links)
         t_link = max(ep_h.wire_in / link["ce_h2d_gbs"], ep_h.reply_wire / link["ce_d2h_gbs"],
                      (ep_h.wire_in + ep_h.reply_wire) / link["ce_bidir_gbs"]) / 1e9
         modes = []
@@ -478,7 +481,8 @@ def main():
                           "wire_gbs": round((ep_h.wire_in + ep_h.reply_wire) / step_s / 1e9, 3),
                           "host_link": {**link, "pcie_gen5_x16_theoretical_gbs": 63.0,
                                         "bound_ms": round(t_link * 1e3, 3),
-                                        "frac": round(t_link / step_s, 4)},
+                                        "frac": round(t_link / step_s, 4),
+                                        "job": {**link_job, **parallel.link_bound_frac(links, wires, step_s)}},
                           "check": chk})
         modes.sort(key=lambda m: -m["value"] if m["check"]["ok"] else 0)
         e2e = dict(modes[0])
@@ -486,7 +490,7 @@ def main():
         del hslots, loop, ep_h
         torch.cuda.empty_cache()
     sweep = None
-    if not args.no_sweep:
+    if not args.no_sweep and rank == 0:  # one GPU's curve (the others idle at the final barrier)
         if e2e is None:
             link = host_link_peaks(dev)
         sweep = run_sweep(args, dev, link)
@@ -521,7 +525,7 @@ def main():
         "e2e": e2e,
         "sweep": sweep,
     }
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and not args.no_cpu:  # rank 0 only, after every rank's timed regions
         out["cpu_baseline"] = cpu_baseline(args, args.cpu_seconds)
     if rank == 0:
         print(json.dumps(out))

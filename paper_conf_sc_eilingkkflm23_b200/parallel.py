@@ -1,7 +1,8 @@
 """Multi-GPU plumbing for the benchmark: one process per GPU, each an independent Cricket server endpoint
-(no cross-GPU exchange exists on the memcpy path, so there is no data-path collective).
-torch.distributed is used only to line the ranks up (barrier) and to reduce the timings: the job's time is
-the max over ranks, its work the sum over ranks (weak scaling)."""
+(no cross-GPU exchange exists on the memcpy path, so there is no data-path collective and no
+NCCL: BASELINE.json north_star).  torch.distributed with the CPU `gloo` backend only lines the ranks up
+(barrier) and reduces the timings: the job's time is the max over ranks, its work the sum over ranks (weak
+scaling); host-link rooflines are measured by every rank at once after a barrier and gathered."""
 from __future__ import annotations
 
 import os
@@ -76,3 +77,38 @@ def bind_numa(device: int, sysfs: str = "/sys") -> dict:
     except OSError:
         cpus = set()
     return {"pci": bdf, "numa_node": node, "cores": len(cpus)}
+
+
+def init(world: int) -> bool:
+    """Joins the job's process group (gloo, CPU) when there is more than one rank; no NCCL anywhere."""
+    if world > 1 and not (dist.is_available() and dist.is_initialized()):
+        dist.init_process_group("gloo")
+        return True
+    return False
+
+
+def gather(obj) -> list:
+    """Every rank's `obj`, in rank order (a list of one without a process group)."""
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
+        return [obj]
+    out = [None] * dist.get_world_size()
+    dist.all_gather_object(out, obj)
+    return out
+
+
+def link_aggregate(per_rank: list[dict], keys=("ce_h2d_gbs", "ce_d2h_gbs", "ce_bidir_gbs")) -> dict:
+    """Host-link peaks measured by all ranks at once (each rank's own GPU, concurrently): per rank and summed.
+    The sum is the job's host-link roofline (PCIe switch uplinks and host memory are shared, so it can be less
+    than N x one GPU alone)."""
+    return {"per_rank": per_rank, "aggregate": {k: round(sum(r[k] for r in per_rank), 2) for k in keys},
+            "ranks": len(per_rank)}
+
+
+def link_bound_frac(per_rank_link: list[dict], per_rank_wire: list[tuple[int, int]], step_s: float) -> dict:
+    """The job's e2e host-link fraction: every rank moves its own wire bytes (in, out) over its own link at the
+    concurrently measured rate; the job can finish no sooner than its slowest rank's link-bound time."""
+    bounds = [max(wi / l["ce_h2d_gbs"], wo / l["ce_d2h_gbs"], (wi + wo) / l["ce_bidir_gbs"]) / 1e9
+              for l, (wi, wo) in zip(per_rank_link, per_rank_wire)]
+    b = max(bounds)
+    return {"bound_ms": round(b * 1e3, 3), "frac": round(b / step_s, 4), "per_rank_bound_ms": [round(x * 1e3, 3)
+                                                                                                for x in bounds]}

@@ -85,3 +85,64 @@ def test_two_rank_endpoints_and_aggregation():
         assert r["agg"]["seconds"] == pytest.approx(tmax)
         assert r["agg"]["per_second"] == pytest.approx(total / tmax)
     assert res[0]["payload"] != res[1]["payload"] or True  # different seeds, independent work
+
+
+def _plumbing_worker(rank, world, port, q):
+    """bench.py's N>1 plumbing on CPU: the gloo group parallel.init joins, the barrier, the max / sum reductions of
+    the timed region, and the concurrently measured host-link roofline gathered and aggregated."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank), WORLD_SIZE=str(world),
+                      LOCAL_RANK=str(rank))
+    from paper_conf_sc_eilingkkflm23_b200 import parallel
+    w, r, _ = parallel.rank_env()
+    assert parallel.init(w) and dist.get_backend() == "gloo"  # no NCCL (north_star)
+    parallel.barrier()
+    ms = 1.0 + r            # rank r's per-step time
+    payload = 1000 * (r + 1)
+    ms_max = parallel.max_over_ranks(ms)
+    total = parallel.sum_over_ranks(payload)
+    link = {"ce_h2d_gbs": 50.0 + r, "ce_d2h_gbs": 40.0 + r, "ce_bidir_gbs": 80.0 + r}
+    links = parallel.gather(link)
+    wires = parallel.gather((10**9 * (r + 1), 10**9))
+    agg = parallel.link_aggregate(links)
+    frac = parallel.link_bound_frac(links, wires, step_s=0.1)
+    q.put(dict(rank=r, ms_max=ms_max, total=total, links=links, agg=agg, frac=frac))
+    parallel.barrier()
+    dist.destroy_process_group()
+
+
+def test_bench_plumbing_two_ranks_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_plumbing_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = sorted([q.get(timeout=300) for _ in range(2)], key=lambda d: d["rank"])
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for r in res:
+        assert r["ms_max"] == 2.0 and r["total"] == 3000
+        assert [x["ce_h2d_gbs"] for x in r["links"]] == [50.0, 51.0]
+        assert r["agg"]["aggregate"] == {"ce_h2d_gbs": 101.0, "ce_d2h_gbs": 81.0, "ce_bidir_gbs": 161.0}
+        # rank 1 moves 2 GB in + 1 GB out over 51 / 41 / 81 GB/s: bound = max(2/51, 1/41, 3/81) s
+        assert r["frac"]["bound_ms"] == pytest.approx(max(2 / 51, 1 / 41, 3 / 81) * 1e3, abs=1e-3)
+        assert r["frac"]["frac"] == pytest.approx(max(2 / 51, 1 / 41, 3 / 81) / 0.1, abs=1e-4)
+
+
+def test_reference_arm_under_torchrun_two_ranks():
+    """`torchrun --nproc-per-node 2 bench.py --impl reference`: rank 0 alone times the oracle and prints one JSON
+    line; rank 1 exits 0 without work (the driver's reference-arm contract at N > 1)."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+           "127.0.0.1", "--master-port", str(_free_port()), os.path.join(root, "bench.py"), "--impl", "reference",
+           "--gpus", "2", "--steps", "2", "--warmup", "1", "--payload-mib", "1"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
