@@ -288,6 +288,7 @@ typedef struct {
   int strict;            /* 1: nonzero pad -> E_PAD, unconsumed bytes -> E_TRAILING, opaque n != size -> E_SIZE */
   uint32_t proc_h2d;     /* built-in (ptr u64, mem opaque<>, size u64) */
   uint32_t proc_d2h;     /* built-in (ptr u64, size u64) */
+  uint32_t proc_stripe;  /* built-in (ptr u64, mem opaque<>, size u64, parent u32, offset u64, total u64); 0: off */
 } or_cfg;
 
 typedef struct {
@@ -394,18 +395,29 @@ int or_parse_call(const uint8_t* L, uint64_t n, const or_cfg* cfg, const or_sche
 #undef OR_FAIL
 }
 
-/* The built-in memcpy schemas (reading R9; Cricket's RPCL is not in the paper). */
-void or_builtin_schemas(const or_cfg* cfg, or_schema* out2) {
-  memset(out2, 0, 2 * sizeof(or_schema));
-  out2[0].proc = cfg->proc_h2d;
-  out2[0].n_items = 3;
-  out2[0].items[0] = OR_K_U64;
-  out2[0].items[1] = OR_K_OPAQUE_VAR;
-  out2[0].items[2] = OR_K_U64;
-  out2[1].proc = cfg->proc_d2h;
-  out2[1].n_items = 2;
-  out2[1].items[0] = OR_K_U64;
-  out2[1].items[1] = OR_K_U64;
+/* The built-in memcpy schemas (readings R9, R22; Cricket's RPCL is not in the paper): HtoD, DtoH and
+ * the HtoD stripe (one part of a memcpy sent over one of several connections).  With
+ * proc_stripe == 0 the third entry repeats the HtoD schema (the first match wins, so it is never used). */
+void or_builtin_schemas(const or_cfg* cfg, or_schema* out3) {
+  memset(out3, 0, 3 * sizeof(or_schema));
+  out3[0].proc = cfg->proc_h2d;
+  out3[0].n_items = 3;
+  out3[0].items[0] = OR_K_U64;
+  out3[0].items[1] = OR_K_OPAQUE_VAR;
+  out3[0].items[2] = OR_K_U64;
+  out3[1].proc = cfg->proc_d2h;
+  out3[1].n_items = 2;
+  out3[1].items[0] = OR_K_U64;
+  out3[1].items[1] = OR_K_U64;
+  if (cfg->proc_stripe == 0) { out3[2] = out3[0]; return; }
+  out3[2].proc = cfg->proc_stripe;
+  out3[2].n_items = 6;
+  out3[2].items[0] = OR_K_U64;        /* ptr: the destination of the whole memcpy */
+  out3[2].items[1] = OR_K_OPAQUE_VAR; /* mem: this stripe's bytes */
+  out3[2].items[2] = OR_K_U64;        /* size */
+  out3[2].items[3] = OR_K_U32;        /* parent: the memcpy's xid */
+  out3[2].items[4] = OR_K_U64;        /* offset of this stripe within the memcpy */
+  out3[2].items[5] = OR_K_U64;        /* total bytes of the memcpy */
 }
 
 /* =====================================================================================
@@ -524,6 +536,45 @@ typedef struct {
   uint64_t reply_wire;
 } or_serve_rec;
 
+/* memcpy HtoD stripe (reading R22; SURVEY.md §8(f) NEXT-1 -- Cricket's parallel-socket memcpy,
+ * PAPER.md:170, :238, :240): a memcpy of `total` bytes to `ptr` sent as several CALLs, one per connection, each
+ * carrying bytes [offset, offset + size) and the memcpy's own xid as `parent`.  Checks of one stripe, in order:
+ * strict mem.n == size (E_SIZE); total < 2^63 and offset + m <= total (E_SIZE); [ptr + offset, + m) inside the
+ * region (E_PTR).  A stripe that passes copies its bytes and has no reply of its own. */
+static int or_stripe_check(const or_call* c, const or_cfg* cfg, uint64_t region_base, uint64_t region_bytes,
+                           uint64_t* m_out) {
+  uint64_t n = c->count[1], size = c->value[2], ptr = c->value[0], off = c->value[4], tot = c->value[5];
+  uint64_t m = (cfg->strict || n <= size) ? n : size;
+  *m_out = 0;
+  if (cfg->strict && n != size) return OR_E_SIZE;
+  if (tot >= (1ull << 63) || off > tot || m > tot - off) return OR_E_SIZE;
+  if (ptr > ~0ull - off) return OR_E_PTR;
+  ptr += off;
+  if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) return OR_E_PTR;
+  *m_out = m;
+  return OR_OK;
+}
+
+/* One parent memcpy of a serve step: it is complete when its OK stripes agree on (ptr, total), their sizes sum
+ * to total, and one of them starts at offset 0 -- the lead, the earliest such stripe in index order, whose
+ * record then carries the parent's reply REPLY(parent) | int 0 (the HtoD reply) in its ring's reply order. */
+typedef struct {
+  uint32_t parent, bad;
+  uint64_t ptr, total, landed;
+  uint32_t lead;         /* index of the lead record, or 0xffffffff */
+  uint32_t nstripes;     /* OK stripes seen */
+} or_parent;
+
+static or_parent* or_parent_of(or_parent* ps, uint32_t* np, uint32_t parent) {
+  uint32_t k;
+  for (k = 0; k < *np; ++k)
+    if (ps[k].parent == parent) return &ps[k];
+  memset(&ps[*np], 0, sizeof(or_parent));
+  ps[*np].parent = parent;
+  ps[*np].lead = 0xffffffffu;
+  return &ps[(*np)++];
+}
+
 int or_serve(uint32_t n_rings, const uint8_t* const* rings, const uint64_t* caps, const uint64_t* heads,
              const uint64_t* tails, uint64_t max_record_bytes, uint32_t max_frags_per_ring,
              uint32_t max_records_per_ring, const or_cfg* cfg, const or_schema* user_schemas, uint32_t n_user,
@@ -531,14 +582,19 @@ int or_serve(uint32_t n_rings, const uint8_t* const* rings, const uint64_t* caps
              const uint64_t* send_caps, const uint64_t* out_off, uint32_t F, int32_t* scan_status,
              uint64_t* consumed, uint64_t* reply_bytes, or_serve_rec* out_recs, uint32_t max_out,
              uint32_t* n_out) {
-  uint32_t r, i, total = 0, ns = n_user + 2;
+  uint32_t r, i, total = 0, ns = n_user + 3, pass, n_parents = 0;
   or_schema* schemas = (or_schema*)calloc(ns, sizeof(or_schema));
   or_frag* frags = (or_frag*)malloc((size_t)(max_frags_per_ring ? max_frags_per_ring : 1) * sizeof(or_frag));
   or_rec* recs = (or_rec*)malloc((size_t)(max_records_per_ring ? max_records_per_ring : 1) * sizeof(or_rec));
   uint32_t* seen_xid = (uint32_t*)malloc((size_t)(max_out ? max_out : 1) * sizeof(uint32_t));
   uint8_t* xid_readable = (uint8_t*)malloc((size_t)(max_out ? max_out : 1));
+  or_parent* parents = (or_parent*)malloc((size_t)(max_out ? max_out : 1) * sizeof(or_parent));
   or_builtin_schemas(cfg, schemas);
-  for (i = 0; i < n_user; ++i) schemas[2 + i] = user_schemas[i];
+  for (i = 0; i < n_user; ++i) schemas[3 + i] = user_schemas[i];
+  /* Pass 0 decides every record and gathers the stripes of each parent memcpy (a stripe's reply depends on
+   * stripes in other rings); pass 1 repeats the same decisions and carries them out in index order. */
+  for (pass = 0; pass < 2; ++pass) {
+  total = 0;
   for (r = 0; r < n_rings; ++r) {
     uint32_t nf = 0, nr = 0;
     uint64_t w = out_off[r];
@@ -567,7 +623,49 @@ int or_serve(uint32_t n_rings, const uint8_t* const* rings, const uint64_t* caps
       seen_xid[total] = c.xid;
       xid_readable[total] = recs[i].len >= 4;
       if (o->status == OR_OK && dup) o->status = OR_E_XID;
-      if (o->status == OR_OK && c.proc == cfg->proc_h2d) {
+      if (pass == 0) {  /* decisions only: gather the OK stripes of each parent */
+        if (o->status == OR_OK && cfg->proc_stripe && c.proc == cfg->proc_stripe) {
+          uint64_t m;
+          if (or_stripe_check(&c, cfg, region_base, region_bytes, &m) == OR_OK) {
+            or_parent* P = or_parent_of(parents, &n_parents, (uint32_t)c.value[3]);
+            if (P->nstripes++ == 0) {  /* the first OK stripe fixes the memcpy's ptr and total */
+              P->ptr = c.value[0];
+              P->total = c.value[5];
+            }
+            if (P->ptr != c.value[0] || P->total != c.value[5]) P->bad = 1;
+            P->landed += m;
+            if (c.value[4] == 0 && P->lead == 0xffffffffu) P->lead = total;
+          }
+        }
+        total++;
+        free(L);
+        continue;
+      }
+      if (o->status == OR_OK && cfg->proc_stripe && c.proc == cfg->proc_stripe) {
+        uint64_t m, b;
+        o->status = or_stripe_check(&c, cfg, region_base, region_bytes, &m);
+        if (o->status == OR_OK) {
+          const or_parent* P = or_parent_of(parents, &n_parents, (uint32_t)c.value[3]);
+          uint64_t dst = c.value[0] + c.value[4] - region_base;
+          for (b = 0; b < m; ++b) region[dst + b] = L[c.off[1] + b];
+          if (P->lead == total && !P->bad && P->landed == P->total) {  /* the parent's reply */
+            uint8_t tmp[32];
+            uint64_t ln = or_rpc_put_reply_header(tmp, 0, P->parent), wl;
+            ln = or_xdr_put_u32(tmp, ln, 0);
+            wl = or_frame_wire_size(ln, F);
+            if (send_rings) {
+              uint8_t* wire = (uint8_t*)malloc(wl);
+              or_frame_record(tmp, ln, F, wire);
+              for (b = 0; b < wl; ++b) send_rings[r][(w + b) & (send_caps[r] - 1)] = wire[b];
+              free(wire);
+            }
+            o->reply_err = 0;
+            o->reply_off = w;
+            o->reply_wire = wl;
+            w += wl;
+          }
+        }
+      } else if (o->status == OR_OK && c.proc == cfg->proc_h2d) {
         uint64_t n = c.count[1], size = c.value[2], ptr = c.value[0];
         uint64_t m = (cfg->strict || n <= size) ? n : size;
         if (cfg->strict && n != size) { o->status = OR_E_SIZE; o->reply_err = 1; }
@@ -620,7 +718,8 @@ int or_serve(uint32_t n_rings, const uint8_t* const* rings, const uint64_t* caps
     }
     reply_bytes[r] = w - out_off[r];
   }
+  }
   *n_out = total;
-  free(schemas); free(frags); free(recs); free(seen_xid); free(xid_readable);
+  free(schemas); free(frags); free(recs); free(seen_xid); free(xid_readable); free(parents);
   return OR_OK;
 }

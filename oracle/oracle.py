@@ -28,6 +28,7 @@ E_TRAILING, E_XID, E_PTR, E_CAPACITY, E_PROC = -8, -9, -10, -11, -12
 
 # schema item kinds
 K_U32, K_U64, K_OPAQUE_VAR, K_OPAQUE_FIX = 1, 2, 3, 4
+N_BUILTIN = 3  # or_builtin_schemas: HtoD, DtoH, HtoD stripe
 K_I32_VAR, K_U32_VAR, K_F32_VAR, K_I64_VAR, K_U64_VAR, K_F64_VAR = 5, 6, 7, 8, 9, 10
 K_I32_FIX, K_U32_FIX, K_F32_FIX, K_I64_FIX, K_U64_FIX, K_F64_FIX = 11, 12, 13, 14, 15, 16
 MAX_ITEMS = 8
@@ -59,7 +60,7 @@ class Schema(C.Structure):
 
 class Cfg(C.Structure):
     _fields_ = [("prog", C.c_uint32), ("vers", C.c_uint32), ("strict", C.c_int), ("proc_h2d", C.c_uint32),
-                ("proc_d2h", C.c_uint32)]
+                ("proc_d2h", C.c_uint32), ("proc_stripe", C.c_uint32)]
 
 
 class Call(C.Structure):
@@ -295,23 +296,24 @@ class Config:
     strict: bool = True
     proc_h2d: int = 1
     proc_d2h: int = 2
+    proc_stripe: int = 3  # the HtoD stripe (NEXT-1, reading R22); 0 disables it
     frag_payload: int = 65536
     user_schemas: dict = field(default_factory=dict)  # proc -> list of item codes
 
     def c(self) -> Cfg:
-        return Cfg(self.prog, self.vers, int(self.strict), self.proc_h2d, self.proc_d2h)
+        return Cfg(self.prog, self.vers, int(self.strict), self.proc_h2d, self.proc_d2h, self.proc_stripe)
 
     def schemas(self):
-        n = 2 + len(self.user_schemas)
+        n = N_BUILTIN + len(self.user_schemas)
         arr = (Schema * n)()
         cfg = self.c()
         lib().or_builtin_schemas(C.byref(cfg), arr)
         for i, (proc, items) in enumerate(self.user_schemas.items()):
             assert len(items) <= MAX_ITEMS
-            arr[2 + i].proc = proc
-            arr[2 + i].n_items = len(items)
+            arr[N_BUILTIN + i].proc = proc
+            arr[N_BUILTIN + i].n_items = len(items)
             for j, it in enumerate(items):
-                arr[2 + i].items[j] = it
+                arr[N_BUILTIN + i].items[j] = it
         return arr, n
 
 
@@ -416,7 +418,7 @@ def serve(rings, cfg: Config, region: np.ndarray, region_base: int, send_caps, o
     cc = cfg.c()
     assert region.dtype == np.uint8 and region.flags.c_contiguous
     lib().or_serve(n, ring_ptrs, caps, heads, tails, max_record_bytes, max_frags_per_ring, max_records_per_ring,
-                   C.byref(cc), C.cast(C.byref(arr, 2 * C.sizeof(Schema)), C.POINTER(Schema)), ns - 2,
+                   C.byref(cc), C.cast(C.byref(arr, N_BUILTIN * C.sizeof(Schema)), C.POINTER(Schema)), ns - N_BUILTIN,
                    _p(region) if region.size else _p(np.zeros(1, np.uint8)), region_base, region.size,
                    send_ptrs, scaps, offs, cfg.frag_payload, sst, cons, rbytes, recs, max_out, C.byref(nout))
     out = [dict(status=r.status, reply_err=r.reply_err, ring=r.ring, xid=r.xid, proc=r.proc,
