@@ -115,6 +115,10 @@ typedef struct {
   uint32_t scan_chunking;    /* 0 (default): windows of at least 2 chunks (>= 512 KiB) are scanned by the chunked
                                 multi-CTA scan (one CTA per chunk); 1: always one CTA per ring */
   uint64_t fused_front_max_window; /* default 1 MiB (one CTA scans the rings in turn) */
+  uint32_t proc_h2d_stripe;  /* built-in schema (ptr u64, mem opaque<>, size u64, parent u32, offset u64, total u64):
+                                one stripe of a memcpy sent over several connections (reading R22;
+                                default 3, 0 = no such procedure) */
+  uint32_t pad1_;
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;
@@ -315,6 +319,10 @@ uint64_t crk_call_logical_size(const crk_item_src* items, uint32_t n_items);
  *   proc_h2d: E_SIZE / E_PTR (ptr range outside [region_base, +region_bytes)) -> reply err = 1,
  *             else copy the payload to ptr and reply err = 0;
  *   proc_d2h: E_PTR -> reply err = 1 (void arm), else reply err = 0 + the `size` bytes at ptr;
+ *   proc_h2d_stripe: E_SIZE (strict n != size; offset + n > total) / E_PTR (ptr + offset range outside the
+ *             region) -> no reply; else the bytes land at ptr + offset and, when the step holds every stripe of
+ *             the memcpy (over all rings: sizes sum to total, ptr and total agree, one stripe at offset 0), the
+ *             offset-0 stripe's place in its ring gets the memcpy's reply REPLY(parent) | int 0 (reading R22);
  *   other registered procs -> OK, no reply (decode them per argument).
  * Replies of ring r are framed with cfg.frag_payload and appended to send_rings[r] from cursor
  * send_offs[r] in record order.  All HtoD destinations and DtoH sources of one call must be disjoint

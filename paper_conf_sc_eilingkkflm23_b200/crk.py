@@ -45,7 +45,8 @@ class Config(C.Structure):
                 ("scan_stride_guess", C.c_uint32), ("tile_bytes", C.c_uint32), ("max_jobs", C.c_uint32),
                 ("ctas_per_sm", C.c_uint32), ("scan_threads", C.c_uint32), ("mover_stages", C.c_uint32),
                 ("mover_run", C.c_uint32), ("mover_tail_tiles", C.c_uint32), ("mover_reserve_ctas", C.c_uint32),
-                ("fused_front_max_records", C.c_uint32), ("scan_chunking", C.c_uint32), ("fused_front_max_window", C.c_uint64)]
+                ("fused_front_max_records", C.c_uint32), ("scan_chunking", C.c_uint32), ("fused_front_max_window", C.c_uint64),
+                ("proc_h2d_stripe", C.c_uint32), ("pad1_", C.c_uint32)]
 
 
 class CRing(C.Structure):

@@ -267,6 +267,7 @@ void crk_config_init(crk_config* c) {
   c->mover_reserve_ctas = 0;
   c->fused_front_max_records = 128;
   c->fused_front_max_window = 1ull << 20;
+  c->proc_h2d_stripe = 3;
 }
 
 int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
@@ -277,7 +278,8 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   if (cfg.frag_payload == 0 || cfg.frag_payload > 0x7fffffffu || !pow2(cfg.tile_bytes) || cfg.tile_bytes < 1024 ||
       cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 64 ||
       cfg.scan_threads > 1024 || (cfg.scan_threads & 63) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
-      cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64 || cfg.scan_chunking > 1)
+      cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64 || cfg.scan_chunking > 1 ||
+      (cfg.proc_h2d_stripe && (cfg.proc_h2d_stripe == cfg.proc_h2d || cfg.proc_h2d_stripe == cfg.proc_d2h)))
     return CRK_E_ARG;
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -310,8 +312,12 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.tail = cfg.mover_tail_tiles;
   d.reserve = cfg.mover_reserve_ctas;
   d.no_chunked_scan = cfg.scan_chunking == 1 ? 1u : 0u;
+  d.proc_stripe = cfg.proc_h2d_stripe;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
+  if (cfg.proc_h2d_stripe)  // ptr, mem, size, parent, offset, total (reading R22)
+    add_builtin(c->host_schemas, cfg.proc_h2d_stripe,
+                {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64, CRK_K_U32, CRK_K_U64, CRK_K_U64});
   // scratch: one block
   Scratch& sc = c->sc;
   sc.max_jobs = cfg.max_jobs;
@@ -353,7 +359,8 @@ void crk_ctx_destroy(crk_ctx* c) {
 
 int crk_proc_schema_register(crk_ctx* c, uint32_t proc, const uint32_t* items, uint32_t n) {
   if (!c || (n && !items) || n > (uint32_t)kMaxItems) return CRK_E_ARG;
-  if (proc == c->cfg.proc_h2d || proc == c->cfg.proc_d2h) return CRK_E_ARG;
+  if (proc == c->cfg.proc_h2d || proc == c->cfg.proc_d2h || (c->cfg.proc_h2d_stripe && proc == c->cfg.proc_h2d_stripe))
+    return CRK_E_ARG;
   for (uint32_t i = 0; i < n; ++i) {
     const uint32_t k = items[i] & 0xff, fixed = items[i] >> 8;
     if (!kind_valid(k) || (kind_var(k) && fixed) || ((k == CRK_K_U32 || k == CRK_K_U64) && fixed)) return CRK_E_ARG;
@@ -409,7 +416,8 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
       4 * (size_t)R, 4 * (size_t)R, 8 * (size_t)R, 8 * (size_t)R,               // serve
       8 * (size_t)hs,
       sizeof(uint2) * (size_t)CC * kCand * kLogCap, sizeof(ChainSum) * (size_t)CC * kCand,  // chunked scan
-      sizeof(ChunkState) * (size_t)CC, sizeof(ChunkStop) * (size_t)CC, sizeof(RingPlan) * max_rings, 16};
+      sizeof(ChunkState) * (size_t)CC, sizeof(ChunkStop) * (size_t)CC, sizeof(RingPlan) * max_rings, 16,
+      sizeof(StripeEnt) * (size_t)hs, 4 * (size_t)R, 8};  // striped memcpys
   constexpr int N = sizeof(sz) / sizeof(sz[0]);
   size_t total = 0, off[N];
   for (int i = 0; i < N; ++i) { off[i] = total; total += (sz[i] + 255) & ~(size_t)255; }
@@ -450,8 +458,12 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
   ix.ms.stops = (ChunkStop*)(b + off[i++]);
   ix.ms.plan = (RingPlan*)(b + off[i++]);
   ix.ms.stats = (uint32_t*)(b + off[i++]);
+  ix.stripe = (StripeEnt*)(b + off[i++]);
+  ix.stripe_list = (uint32_t*)(b + off[i++]);
+  ix.stripe_n = (uint32_t*)(b + off[i++]);
   e = cudaMemset(x->block, 0, total);
   if (e == cudaSuccess) e = cudaMemset(ix.xid_hash, 0xff, 8 * (size_t)hs);
+  if (e == cudaSuccess) e = cudaMemset(ix.stripe, 0xff, sizeof(StripeEnt) * (size_t)hs);
   for (uint32_t r = 0; e == cudaSuccess && r < max_rings; ++r)  // no stop recorded
     e = cudaMemset(&ix.ms.plan[r].stop_key, 0xff, sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMallocHost(&x->host_res, sizeof(crk_ring_result) * max_rings);

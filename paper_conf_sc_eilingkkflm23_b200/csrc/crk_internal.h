@@ -70,6 +70,16 @@ struct MultiScanDev {
   uint32_t* stats;                  // [4] diagnostic totals: rings resolved chunked, rings that fell back
 };
 
+// One parent memcpy of a serve step's striped HtoD CALLs (reading R22).  Open addressing by parent xid over
+// a table that is all ~0 between steps (the planner resets the entries it used): key = parent xid; ptr / total
+// claimed by the first OK stripe (CAS from ~0), good cleared by a stripe that disagrees; landed_c = ~(bytes
+// landed); lead = the smallest dense id of an OK stripe at offset 0.
+struct StripeEnt {                  // 48 bytes
+  unsigned long long key, ptr, total, landed_c;
+  uint32_t lead, good;
+  unsigned long long pad_;
+};
+
 // Device-resident tables of one index (pointers into one cudaMalloc block).
 struct IndexDev {
   uint32_t max_rings, frags_per_ring, recs_per_ring, max_records;
@@ -102,6 +112,9 @@ struct IndexDev {
   uint64_t* s_reply_wire;
   unsigned long long* xid_hash;  // (xid << 32 | dense id), empty = ~0
   MultiScanDev ms;               // chunked scan scratch
+  StripeEnt* stripe;             // [hash_mask + 1] parent memcpys of the step (reading R22)
+  uint32_t* stripe_list;         // [max_records] table slots in use
+  uint32_t* stripe_n;            // [2]: slots in use, planning-pass ticket
 };
 
 // ---- mover jobs ----------------------------------------------------------------------------------
@@ -156,6 +169,7 @@ struct ConfigDev {
   uint32_t scan_threads, stages, run, tail;  // tail: per-CTA single-tile claims at the end of each queue
   uint32_t reserve;         // mover CTAs that run only when the launch found the GPU free (crk_config.mover_reserve_ctas)
   uint32_t no_chunked_scan; // crk_config.scan_chunking == 1: one CTA per ring always
+  uint32_t proc_stripe, pad2_;  // crk_config.proc_h2d_stripe (0: none)
   uint64_t max_record_bytes;
   unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };

@@ -98,6 +98,36 @@ __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint6
     sc.jobs[d] = job;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = 2 * total; sc.counters[4] = total; }
+  if (!cfg.proc_stripe) return;
+  // striped memcpys (reading R22): the last block, once every stripe has decided, gives the leads of complete
+  // parents their reply and empties the parent table for the next step
+  __shared__ uint32_t last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(ix.stripe_n + 1, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  const uint32_t n = __ldcg(ix.stripe_n);
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const StripeEnt* e = ix.stripe + ix.stripe_list[i];
+    const uint32_t d = __ldcg(&e->lead);
+    if (d != ~0u && __ldcg(&e->good) != 0 && ~__ldcg(&e->landed_c) == __ldcg(&e->total)) {
+      const uint64_t w = wire_of(28, cfg.F);
+      ix.s_reply_err[d] = 0;
+      ix.s_reply_wire[d] = w;
+      wire[d] = w;
+    }
+  }
+  __syncthreads();
+  stripe_clear(ix, n, threadIdx.x, blockDim.x);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    ix.stripe_n[0] = 0;
+    ix.stripe_n[1] = 0;
+  }
 }
 
 // pass 2: reply cursors (prefix of wire sizes within each ring) and the encode jobs

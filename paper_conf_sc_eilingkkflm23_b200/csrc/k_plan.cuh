@@ -75,8 +75,54 @@ __device__ __forceinline__ void reply_words(Piece& p, uint32_t xid, int32_t err,
   p.nbytes = with_len ? 32 : 28;
 }
 
+// ---- striped memcpys (reading R22): the parent table of a serve step ------------------------------------
+// An OK stripe of `parent` adds its bytes; the first OK stripe claims (ptr, total), a disagreeing one marks the
+// parent inconsistent; a stripe at offset 0 offers itself as the lead (smallest dense id).
+__device__ __forceinline__ void stripe_add(const IndexDev& ix, uint32_t parent, uint64_t ptr, uint64_t total,
+                                           uint64_t m, bool at0, uint32_t d) {
+  uint32_t h = (parent * 0x9E3779B1u) & ix.hash_mask;
+  for (;;) {
+    StripeEnt& e = ix.stripe[h];
+    const unsigned long long k = atomicCAS(&e.key, ~0ull, (unsigned long long)parent);
+    if (k == ~0ull) ix.stripe_list[atomicAdd(ix.stripe_n, 1u)] = h;  // a new parent: remember its slot
+    if (k == ~0ull || k == parent) {
+      const unsigned long long p0 = atomicCAS(&e.ptr, ~0ull, (unsigned long long)ptr);
+      const unsigned long long t0 = atomicCAS(&e.total, ~0ull, (unsigned long long)total);
+      if ((p0 != ~0ull && p0 != ptr) || (t0 != ~0ull && t0 != total)) atomicAnd(&e.good, 0u);
+      atomicAdd(&e.landed_c, (unsigned long long)(0ull - m));  // ~landed - m = ~(landed + m)
+      if (at0) atomicMin(&e.lead, d);
+      return;
+    }
+    h = (h + 1) & ix.hash_mask;
+  }
+}
+
+// True when stripe record d (OK, at offset 0) leads a complete parent: consistent, every byte landed.
+__device__ __forceinline__ bool stripe_leads(const IndexDev& ix, uint32_t parent, uint32_t d) {
+  uint32_t h = (parent * 0x9E3779B1u) & ix.hash_mask;
+  for (;;) {
+    const StripeEnt* e = ix.stripe + h;
+    const unsigned long long k = __ldcg(&e->key);
+    if (k == ~0ull) return false;
+    if (k == parent)
+      return __ldcg(&e->lead) == d && __ldcg(&e->good) != 0 && ~__ldcg(&e->landed_c) == __ldcg(&e->total);
+    h = (h + 1) & ix.hash_mask;
+  }
+}
+
+// Resets the parent slots a step used (entries [i0, n) of the list, stride st) to the empty state.
+__device__ __forceinline__ void stripe_clear(const IndexDev& ix, uint32_t n, uint32_t i0, uint32_t st) {
+  for (uint32_t i = i0; i < n; i += st) {
+    StripeEnt& e = ix.stripe[ix.stripe_list[i]];
+    e.key = e.ptr = e.total = e.landed_c = ~0ull;
+    e.lead = e.good = ~0u;
+  }
+}
+
 // Serve decisions for dense record d (oracle or_serve): final status, reply discriminant (-1: no reply),
-// reply logical length, and the HtoD decode job.
+// reply logical length, and the HtoD decode job.  A striped memcpy's stripe (reading R22) decides like an
+// HtoD copy to ptr + offset with no reply; whether the offset-0 stripe carries its parent's reply is known
+// only once every stripe of the step has decided (stripe_leads, after a block / grid barrier).
 __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev& cfg, uint32_t d, uint64_t region_base,
                                              uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job) {
   // every field the decision can need is loaded at once (one memory round trip), then the xid lookup
@@ -96,6 +142,22 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
     else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
     else { err = 0; job = dec_job(ix, ptr, m, o1, d, 1); }
     Ll = 28;
+  } else if (st == CRK_OK && cfg.proc_stripe && proc == cfg.proc_stripe) {
+    const uint64_t v3 = ix.p_value[b + 3], off = ix.p_value[b + 4], tot = ix.p_value[b + 5];
+    const uint64_t nb = c1, size = v2;
+    const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
+    if (cfg.strict && nb != size) st = CRK_E_SIZE;
+    else if (tot >= (1ull << 63) || off > tot || m > tot - off) st = CRK_E_SIZE;
+    else if (v0 > ~0ull - off) st = CRK_E_PTR;
+    else {
+      const uint64_t ptr = v0 + off;
+      if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) st = CRK_E_PTR;
+      else {
+        job = dec_job(ix, ptr, m, o1, d, 1);
+        stripe_add(ix, (uint32_t)v3, v0, tot, m, off == 0, d);
+        Ll = 28;  // the parent's reply, if this stripe turns out to lead a complete memcpy
+      }
+    }
   } else if (st == CRK_OK && proc == cfg.proc_d2h) {
     const uint64_t ptr = v0, size = v1;
     if (size > 0xffffffffull || ptr < region_base || size > region_bytes || ptr - region_base > region_bytes - size) {
@@ -112,10 +174,13 @@ __device__ __forceinline__ Job serve_reply_job(const IndexDev& ix, const ConfigD
   Job job{};
   if (err < 0) return job;
   const uint64_t b = (uint64_t)d * kMaxItems;
-  const bool d2h = ix.p_proc[d] == cfg.proc_d2h && err == 0;
+  const uint32_t proc = ix.p_proc[d];
+  const bool d2h = proc == cfg.proc_d2h && err == 0;
   const uint64_t n = d2h ? ix.p_value[b + 1] : 0;
+  // a striped memcpy's reply carries the parent memcpy's xid (reading R22)
+  const uint32_t xid = (cfg.proc_stripe && proc == cfg.proc_stripe) ? (uint32_t)ix.p_value[b + 3] : ix.p_xid[d];
   Piece* P = sc.pieces + 2ull * d;
-  reply_words(P[0], ix.p_xid[d], err, d2h, n);
+  reply_words(P[0], xid, err, d2h, n);
   uint32_t np = 1;
   uint64_t Ll = P[0].nbytes;
   if (d2h) {
@@ -203,8 +268,14 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
     first = prefix_s ? prefix_s[ring] : ix.rec_prefix[ring];
     end = prefix_s ? prefix_s[ring + 1] : ix.rec_prefix[ring + 1];
-    w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   }
+  if (cfg.proc_stripe) {  // every stripe of the step has decided: the leads of complete memcpys reply
+    __syncthreads();
+    if (d < total && st == CRK_OK && Ll == 28 && err < 0 && ix.p_proc[d] == cfg.proc_stripe &&
+        stripe_leads(ix, (uint32_t)ix.p_value[(uint64_t)d * kMaxItems + 3], d))
+      err = 0;
+  }
+  if (d < total) w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   uint64_t tot;
   const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets
   if (d < total && d == first) ring_first_pre[ring] = pre;
@@ -233,6 +304,12 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   if (d < total) {
     sc.scan_tmp[d] = pd;
     sc.scan_tmp[total + d] = tot_d + pe;
+  }
+  if (cfg.proc_stripe) {  // leave the parent table empty for the next step (every lead has read it)
+    const uint32_t n = __ldcg(ix.stripe_n);
+    stripe_clear(ix, n, threadIdx.x, blockDim.x);
+    __syncthreads();
+    if (d == 0 && n) *ix.stripe_n = 0;
   }
   if (d == 0) {
     sc.scan_tmp[sc.max_jobs + 1] = tot_d + tot_e;

@@ -9,7 +9,8 @@ output against the generator's values.  Writes one JSON object (stdout).
   C3   bandwidth sweep: HtoD (scan+parse+decode) and DtoH (reply encode) GB/s per size, buffers rotated
        over >= 256 MiB so repeated runs do not hit L2
   C4   256 MiB typed-array stress: decode GB/s (all items, regular and irregular framing)
-  NEXT-1  one 1 GiB memcpy striped over 16 rings (16 CALLs of 64 MiB at ptr + offset), served as one batch
+  NEXT-1  one 1 GiB memcpy striped over 16 / 4 rings (stripe CALLs, reading R22: one reply for the memcpy) vs one
+          1 GiB CALL on one ring and 16 separate 64 MiB CALLs, each served as one batch
   NEXT-2  gen.cusolver_endpoint (100 iterations of A 900x900 f64 + b HtoD, x DtoH; 1 and 4 client streams) and
           gen.histogram_endpoint (64 MiB HtoD, 256-bin result DtoH), served by crk_serve
 """
@@ -375,6 +376,31 @@ def served(ctx, sizes_h2d, sizes_d2h, streams=1, reps=20):
     return {"ms": round(ms, 4), "payload_bytes": pay, "gbs": round(pay / ms / 1e6, 1), "ok": bool(ok)}
 
 
+def striped(total, k, reps=20):
+    """NEXT-1: one memcpy of `total` bytes striped over k rings (reading R22: k stripe CALLs, the offset-0 stripe
+    carries the memcpy's reply), served as one crk_serve step; payload GB/s and the check."""
+    ctx = Ctx()
+    region = torch.zeros(total + 256, dtype=torch.uint8, device=dev)
+    base = region.data_ptr()
+    payload = torch.from_numpy(gen.random_bytes(0x51, total)).to(dev)
+    per = total // k
+    rings, sends = [], []
+    for i in range(k):
+        a, b = i * per, total if i == k - 1 else (i + 1) * per
+        ring = crk.Ring.device(next_pow2(b - a + 4 * ((b - a) // 65536 + 2) + 128))
+        w = ctx.encode_call(0x5100 + i, 3, [(crk.K_U64, base), (crk.K_OPAQUE_VAR, payload[a:b]), (crk.K_U64, b - a),
+                                            (crk.K_U32, 0x51), (crk.K_U64, a), (crk.K_U64, total)], ring, 0)
+        rings.append((ring, 0, w))
+        sends.append(crk.Ring.device(4096))
+    idx = ctx.index(k, 1 << 16, 1 << 10)
+    ms = timed(lambda _: idx.serve(rings, sends, [0] * k, base, region.numel()), reps)
+    res = idx.ring_results(k)
+    ok = all(r["status"] == 0 for r in res) and res[0]["reply_bytes"] == 32 and sum(r["reply_bytes"] for r in res) == 32
+    ok &= bool(torch.equal(region[:total], payload))
+    return {"ms": round(ms, 4), "stripes": k, "payload_bytes": total, "gbs": round(total / ms / 1e6, 1), "ok": bool(ok),
+            "scan_stats": idx.scan_stats()}
+
+
 def profile(streams, region_bytes, reps=10):
     """A gen workload profile (NEXT-2) served by crk_serve: payload GB/s and the per-ring check."""
     from paper_conf_sc_eilingkkflm23_b200 import workload
@@ -398,8 +424,10 @@ def main():
         "C3_sweep": lambda: c3(Ctx()),
         "C4_typed_regular": lambda: c4(Ctx(), False),
         "C4_typed_irregular": lambda: c4(Ctx(), True),
-        "NEXT1_striped_1GiB_16_rings": lambda: served(Ctx(), [64 * MiB] * 16, [], streams=16),
+        "NEXT1_striped_1GiB_16_rings": lambda: striped(GiB, 16),
+        "NEXT1_striped_1GiB_4_rings": lambda: striped(GiB, 4),
         "NEXT1_single_1GiB_1_ring": lambda: served(Ctx(), [GiB], [], streams=1),
+        "NEXT1_16_separate_64MiB_calls": lambda: served(Ctx(), [64 * MiB] * 16, [], streams=16),
         "NEXT2_cusolver_100_iters": lambda: profile(*gen.cusolver_endpoint(iterations=100)),
         "NEXT2_cusolver_100_iters_4_streams": lambda: profile(*gen.cusolver_endpoint(iterations=100, n_streams=4)),
         "NEXT2_histogram": lambda: profile(*gen.histogram_endpoint()),
