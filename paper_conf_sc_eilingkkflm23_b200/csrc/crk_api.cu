@@ -312,6 +312,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.tail = cfg.mover_tail_tiles;
   d.reserve = cfg.mover_reserve_ctas;
   d.no_chunked_scan = cfg.scan_chunking == 1 ? 1u : 0u;
+  c->sc.pdl = pdl_of(d) ? 1u : 0u;
   d.proc_stripe = cfg.proc_h2d_stripe;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});

@@ -82,6 +82,15 @@ __device__ __forceinline__ uint4 swap16(uint4 v, uint32_t esize) {
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
+// Programmatic dependent launch (launch_k in crk_internal.h): the first statement of every kernel of the
+// library.  griddepcontrol.wait returns once the previous kernel of the stream has completed and its memory
+// is visible (a no-op without the launch attribute); launch_dependents then lets the stream's next kernel be
+// scheduled, so its CTAs are resident and waiting when this one ends instead of paying the launch gap.
+__device__ __forceinline__ void pdl_entry() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // RFC 4506 §3: bytes of zero pad after n bytes of opaque / array data
 __device__ __forceinline__ uint64_t pad4(uint64_t n) { return (4 - (n & 3)) & 3; }
 

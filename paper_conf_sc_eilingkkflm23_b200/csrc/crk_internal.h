@@ -162,6 +162,7 @@ struct Scratch {          // ctx-owned device scratch
   uint32_t* run_job;      // [max_jobs]: the job holding each mover run's first tile (queue 0 runs, then queue 1)
   uint32_t max_jobs, max_lens, max_pieces;
   uint32_t mover_seq;     // host-side count of this context's mover launches (the launch stamp's sequence)
+  uint32_t pdl;           // launches with programmatic dependent launch (see launch_k)
 };
 
 struct ConfigDev {
@@ -266,6 +267,31 @@ cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratc
 
 // host-visible counter of our kernel launches
 void count_launch(int n = 1);
+
+// Every library kernel is launched with programmatic stream serialization (PDL): it may be scheduled while
+// the stream's previous kernel is still running and waits for it in pdl_entry() (crk_device.cuh).
+// pdl = false launches it as an ordinary stream-ordered kernel (its pdl_entry() waits for nothing).
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k_opt(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                         Args&&... args) {
+  cudaLaunchConfig_t c = {};
+  c.gridDim = grid;
+  c.blockDim = block;
+  c.dynamicSmemBytes = smem;
+  c.stream = s;
+  cudaLaunchAttribute a[1];
+  a[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  a[0].val.programmaticStreamSerializationAllowed = 1;
+  c.attrs = a;
+  c.numAttrs = pdl ? 1 : 0;
+  count_launch();
+  return cudaLaunchKernelEx(&c, kernel, static_cast<KArgs>(args)...);
+}
+// A context launches this way unless it keeps reserved mover CTAs (crk_config.mover_reserve_ctas > 0: a
+// pipelined server loop with batches in flight on several streams): there, kernels resident early would sit on
+// the SM slots the other batches' kernels need (measured: C5 step 0.347 -> 0.371 ms), while a lone call saves
+// each launch gap (C3 4 KiB HtoD call 31 -> 21 us).
+__host__ __device__ inline bool pdl_of(const ConfigDev& cfg) { return cfg.reserve == 0; }
 
 // optional CUDA-event timing of the pipeline stages (crk_profile_*)
 enum { PROF_SCAN = 0, PROF_PARSE = 1, PROF_PLAN = 2, PROF_MOVE = 3, PROF_STAGES = 4 };

@@ -29,6 +29,7 @@ struct FrontParams {
 };
 
 __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontParams P) {
+  pdl_entry();
   __shared__ ScanState S;
   __shared__ SchemaTable sch;
   __shared__ __align__(16) uint8_t heads[kFrontWarps][kHeadBuf];
@@ -107,8 +108,10 @@ cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch
   P.region_base = region_base;
   P.region_bytes = region_bytes;
   prof_mark(PROF_SCAN, true, s);
-  front_small_kernel<<<1, kFrontThreads, 0, s>>>(P);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), front_small_kernel, 1, kFrontThreads, 0, s, P);
+    if (le != cudaSuccess) return le;
+  }
   prof_mark(PROF_SCAN, false, s);
   return cudaGetLastError();
 }

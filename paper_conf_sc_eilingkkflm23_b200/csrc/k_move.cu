@@ -259,6 +259,7 @@ __device__ __forceinline__ uint32_t find_job(const uint64_t* prefix, uint32_t n_
 #define CRK_MOVER_MIN_BLOCKS 2
 #endif
 __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_kernel(MoveParams M) {
+  pdl_entry();
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t full[kMaxStages], empty[kMaxStages];
   const uint32_t kStages = M.cfg.stages;
@@ -581,6 +582,7 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
 // the tile prefix.  counters[12] = queue-0 run count, counters[13] = 1 when the map applies.
 __global__ void run_map_kernel(Scratch sc, ConfigDev cfg, uint32_t grid, uint32_t run, const uint64_t* prefix,
                                const uint32_t* n_jobs_dev, const uint64_t* total_tiles) {
+  pdl_entry();
   const uint64_t total = *total_tiles;
   const uint32_t n_jobs = *n_jobs_dev;
   const uint32_t n_split = sc.counters[4] < n_jobs ? sc.counters[4] : n_jobs;
@@ -611,6 +613,7 @@ __global__ void run_map_kernel(Scratch sc, ConfigDev cfg, uint32_t grid, uint32_
 
 // tiles per job: output range cut at tile_bytes-aligned boundaries
 __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, const uint32_t* n_jobs_dev) {
+  pdl_entry();
   const uint32_t n = *n_jobs_dev;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     sc.counters[0] = 0;  // decode-queue run cursor
@@ -632,6 +635,7 @@ __global__ void plan_count_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, co
 constexpr uint32_t kSmallJobs = 2048;
 __global__ void __launch_bounds__(256) plan_small_kernel(Scratch sc, ConfigDev cfg, uint64_t* tiles, uint64_t* total,
                                                          const uint32_t* n_jobs_dev) {
+  pdl_entry();
   __shared__ uint64_t warp_sum[8];
   const uint32_t n = *n_jobs_dev;
   if (threadIdx.x == 0) {
@@ -690,13 +694,17 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   cudaError_t e;
   if (planned) {
   } else if (max_jobs_bound <= kSmallJobs) {
-    plan_small_kernel<<<1, 256, 0, s>>>(sc, cfg, tiles, total, n_jobs_dev);
-    count_launch();
+    {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), plan_small_kernel, 1, 256, 0, s, sc, cfg, tiles, total, n_jobs_dev);
+    if (le != cudaSuccess) return le;
+  }
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   } else {
     const uint32_t cnt_blocks = (max_jobs_bound + 255) / 256;
-    plan_count_kernel<<<min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s>>>(sc, cfg, tiles, n_jobs_dev);
-    count_launch();
+    {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), plan_count_kernel, min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s, sc, cfg, tiles, n_jobs_dev);
+    if (le != cudaSuccess) return le;
+  }
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     e = launch_exclusive_scan_u64(tiles, max_jobs_bound, n_jobs_dev, total, sc, s);
     if (e != cudaSuccess) return e;
@@ -712,8 +720,10 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   }
   bool use_map = false;
   if (!planned && run > 1) {  // the run -> job map for this launch's run boundaries
-    run_map_kernel<<<(uint32_t)sms * 2, 256, 0, s>>>(sc, cfg, (uint32_t)move_ctas, run, tiles, n_jobs_dev, total);
-    count_launch();
+    {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), run_map_kernel, (uint32_t)sms * 2, 256, 0, s, sc, cfg, (uint32_t)move_ctas, run, tiles, n_jobs_dev, total);
+    if (le != cudaSuccess) return le;
+  }
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     use_map = true;
   }
@@ -745,8 +755,12 @@ cudaError_t launch_mover(const IndexDev* ix, const ConfigDev& cfg, Scratch& sc, 
   const uint32_t smem = mover_smem_bytes(1u << cfg.tile_shift, cfg.stages);
   if ((e = ensure_mover_smem(smem)) != cudaSuccess) return e;
   prof_mark(PROF_MOVE, true, s);
-  mover_kernel<<<move_ctas, kMoverThreads, smem, s>>>(M);
-  count_launch();
+  {
+    // Not early-scheduled when it keeps reserved CTAs (a pipelined server loop): CTAs resident early would sit
+    // on SM slots the next batch's front end needs, and would all pass the launch-time gate at once.
+    const cudaError_t le = launch_k_opt(cfg.reserve == 0, mover_kernel, move_ctas, kMoverThreads, smem, s, M);
+    if (le != cudaSuccess) return le;
+  }
   prof_mark(PROF_MOVE, false, s);
   return cudaGetLastError();
 }

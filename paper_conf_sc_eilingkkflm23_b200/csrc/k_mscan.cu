@@ -601,6 +601,7 @@ __device__ void resolve_ring(const IndexDev& ix, const ChunkParam& P, uint32_t r
 }
 
 __global__ void __launch_bounds__(kThreads) chunk_walk_kernel(IndexDev ix, ChunkParam P, ConfigDev cfg) {
+  pdl_entry();
   TL_BEGIN(cfg, TL_SCAN);
   extern __shared__ __align__(128) uint8_t zone[];
   __shared__ SelSmem M;
@@ -695,6 +696,7 @@ __device__ void emit_chunk(const IndexDev& ix, const ChunkParam& P, const Config
 }
 
 __global__ void __launch_bounds__(kThreads) chunk_emit_kernel(IndexDev ix, ChunkParam P, ConfigDev cfg) {
+  pdl_entry();
   TL_BEGIN(cfg, TL_SCAN);
   __shared__ ScanState S;
   __shared__ uint32_t last, fb;
@@ -820,11 +822,15 @@ cudaError_t launch_chunk_scan(const IndexDev& ix, const void* param, const Confi
   cudaError_t e = ensure_walk_smem();
   if (e != cudaSuccess) return e;
   const uint32_t n = P.chunk0[P.n_rings];
-  chunk_walk_kernel<<<n, kThreads, kZoneBytes, s>>>(ix, P, cfg);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), chunk_walk_kernel, n, kThreads, kZoneBytes, s, ix, P, cfg);
+    if (le != cudaSuccess) return le;
+  }
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  chunk_emit_kernel<<<n, kThreads, 0, s>>>(ix, P, cfg);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), chunk_emit_kernel, n, kThreads, 0, s, ix, P, cfg);
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 

@@ -7,6 +7,7 @@ namespace {
 
 __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, const SchemaTable* __restrict__ tab,
                                                                   ConfigDev cfg, uint32_t n_rings) {
+  pdl_entry();
   __shared__ SchemaTable sch;
   __shared__ uint32_t prefix[kMaxRings + 1];
   __shared__ __align__(16) uint8_t heads[kParseWarps][kHeadBuf];
@@ -40,8 +41,10 @@ cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const C
   const uint64_t bound = (uint64_t)ix.recs_per_ring * n_rings;
   const uint64_t want = (bound + kParseWarps - 1) / kParseWarps, most = (uint64_t)sms * 8;
   const uint32_t grid = (uint32_t)(want < most ? want : most);
-  parse_kernel<<<grid ? grid : 1, kParseWarps * 32, 0, s>>>(ix, schemas, cfg, n_rings);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), parse_kernel, grid ? grid : 1, kParseWarps * 32, 0, s, ix, schemas, cfg, n_rings);
+    if (le != cudaSuccess) return le;
+  }
   prof_mark(PROF_PARSE, false, s);
   return cudaGetLastError();
 }

@@ -11,6 +11,7 @@ namespace {
 __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint32_t n, const uint32_t* xids,
                                    void* const* dsts, const uint64_t* dst_bytes, int32_t* statuses, uint64_t* copied,
                                    H2DReq single, uint32_t use_single) {
+  pdl_entry();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const uint32_t xid = use_single ? single.xid : xids[i];
     const uint64_t dst = (uint64_t)(use_single ? single.dst : dsts[i]);
@@ -50,6 +51,7 @@ __global__ void resolve_h2d_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint3
 // typed / opaque argument requests (oracle or_decode_item)
 __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint32_t n, const crk_item_req* reqs,
                                      crk_item_req single, uint32_t use_single) {
+  pdl_entry();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const crk_item_req r = use_single ? single : reqs[i];
     Job job{};
@@ -82,6 +84,7 @@ __global__ void resolve_items_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uin
 
 __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint64_t region_base,
                                    uint64_t region_bytes) {
+  pdl_entry();
   const uint32_t total = *ix.total;
   uint64_t* wire = sc.scan_tmp;  // reply wire sizes -> prefix
   for (uint32_t d = blockIdx.x * blockDim.x + threadIdx.x; d < total; d += gridDim.x * blockDim.x) {
@@ -132,6 +135,7 @@ __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint6
 
 // pass 2: reply cursors (prefix of wire sizes within each ring) and the encode jobs
 __global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendRingsParam S) {
+  pdl_entry();
   const uint32_t total = *ix.total;
   const uint64_t* pre = sc.scan_tmp;
   if (blockIdx.x == 0)
@@ -151,6 +155,7 @@ __global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendR
 __global__ void __launch_bounds__(kSmallServe) serve_plan_small_kernel(IndexDev ix, ConfigDev cfg, Scratch sc,
                                                                        SendRingsParam S, uint64_t region_base,
                                                                        uint64_t region_bytes) {
+  pdl_entry();
   __shared__ uint64_t warp_sums[32];
   __shared__ uint64_t ring_first_pre[kMaxRings];
   TL_BEGIN(cfg, TL_PLAN);
@@ -159,6 +164,7 @@ __global__ void __launch_bounds__(kSmallServe) serve_plan_small_kernel(IndexDev 
 }
 
 __global__ void put_enc_jobs_kernel(Scratch sc, ConfigDev cfg, EncJobParam p, RingDesc out) {
+  pdl_entry();
   if (threadIdx.x == 0) {
     for (uint32_t j = 0; j < p.n_jobs; ++j) sc.jobs[j] = p.jobs[j];
     sc.out_rings[0] = out;
@@ -170,6 +176,7 @@ __global__ void put_enc_jobs_kernel(Scratch sc, ConfigDev cfg, EncJobParam p, Ri
 }
 
 __global__ void d2h_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uint64_t* bytes, const int32_t* errs) {
+  pdl_entry();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int32_t err = errs ? errs[i] : 0;
     const uint64_t nb = err == 0 ? bytes[i] : 0;
@@ -182,6 +189,7 @@ __global__ void d2h_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const ui
 __global__ void d2h_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const uint32_t* xids, const void* const* srcs,
                                 const uint64_t* bytes, const int32_t* errs, RingDesc out, uint64_t out_off,
                                 uint64_t* wire_offs, uint64_t* total_dev, const uint64_t* total_scan) {
+  pdl_entry();
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     sc.out_rings[0] = out;
     if (total_dev) *total_dev = *total_scan;
@@ -242,6 +250,7 @@ __device__ __forceinline__ uint64_t reply_item_logical(crk_reply_req r) {
 }
 
 __global__ void replies_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const crk_reply_req* reqs) {
+  pdl_entry();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
     sc.scan_tmp[i] = wire_of(reply_item_logical(reqs[i]), cfg.F);
   if (blockIdx.x == 0 && threadIdx.x == 0) { sc.counters[1] = n; sc.counters[4] = n; }
@@ -250,6 +259,7 @@ __global__ void replies_sizes_kernel(Scratch sc, ConfigDev cfg, uint32_t n, cons
 __global__ void replies_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const crk_reply_req* reqs, RingDesc out,
                                     uint64_t out_off, uint64_t* wire_offs, uint64_t* total_dev,
                                     const uint64_t* total_scan) {
+  pdl_entry();
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     sc.out_rings[0] = out;
     if (total_dev) *total_dev = *total_scan;
@@ -304,6 +314,7 @@ __global__ void replies_jobs_kernel(Scratch sc, ConfigDev cfg, uint32_t n, const
 }
 
 __global__ void lens_prep_kernel(Scratch sc, const uint32_t* lens32, uint32_t n) {
+  pdl_entry();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     sc.lens_pool[i] = lens32[i];
     sc.lens_pool[sc.max_lens + i] = (uint64_t)lens32[i] + 4;  // -> wire starts after the scan
@@ -322,9 +333,11 @@ cudaError_t launch_resolve_h2d(const IndexDev& ix, const ConfigDev& cfg, Scratch
                                const H2DReq* single, cudaStream_t s) {
   H2DReq one{};
   if (single) one = *single;
-  resolve_h2d_kernel<<<blocks_for(n), 256, 0, s>>>(ix, cfg, sc, n, xids, dsts, dst_bytes, statuses, copied, one,
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), resolve_h2d_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, xids, dsts, dst_bytes, statuses, copied, one,
                                                     single ? 1u : 0u);
-  count_launch();
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 
@@ -332,8 +345,10 @@ cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scrat
                                  const crk_item_req* reqs, const crk_item_req* single, cudaStream_t s) {
   crk_item_req one{};
   if (single) one = *single;
-  resolve_items_kernel<<<blocks_for(n), 256, 0, s>>>(ix, cfg, sc, n, reqs, one, single ? 1u : 0u);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), resolve_items_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, reqs, one, single ? 1u : 0u);
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 
@@ -342,8 +357,10 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
                               uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s) {
   const uint32_t bound = ix.max_records;
   prof_mark(PROF_PLAN, true, s);
-  serve_plan1_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, region_base, region_bytes);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan1_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, region_base, region_bytes);
+    if (le != cudaSuccess) return le;
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   e = launch_exclusive_scan_u64(sc.scan_tmp, bound, ix.total, nullptr, sc, s);
@@ -357,8 +374,10 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
     S.off[r] = send_offs ? send_offs[r] : 0;
   }
   S.doorbell = doorbell;
-  serve_plan2_kernel<<<blocks_for(bound), 256, 0, s>>>(ix, cfg, sc, S);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan2_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, S);
+    if (le != cudaSuccess) return le;
+  }
   prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();
 }
@@ -375,16 +394,20 @@ cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Sc
   }
   S.doorbell = doorbell;
   prof_mark(PROF_PLAN, true, s);
-  serve_plan_small_kernel<<<1, kSmallServe, 0, s>>>(ix, cfg, sc, S, region_base, region_bytes);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan_small_kernel, 1, kSmallServe, 0, s, ix, cfg, sc, S, region_base, region_bytes);
+    if (le != cudaSuccess) return le;
+  }
   prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();
 }
 
 cudaError_t launch_put_enc_jobs(Scratch& sc, const ConfigDev& cfg, const EncJobParam& p, const RingDesc& out,
                                 cudaStream_t s) {
-  put_enc_jobs_kernel<<<1, 64, 0, s>>>(sc, cfg, p, out);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), put_enc_jobs_kernel, 1, 64, 0, s, sc, cfg, p, out);
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 
@@ -392,37 +415,47 @@ cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n,
                                   const void* const* srcs, const uint64_t* bytes, const int32_t* errs,
                                   const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
                                   cudaStream_t s) {
-  d2h_sizes_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, bytes, errs);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), d2h_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, bytes, errs);
+    if (le != cudaSuccess) return le;
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
   e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
   if (e != cudaSuccess) return e;
-  d2h_jobs_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), d2h_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
                                                  tot);
-  count_launch();
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 
 cudaError_t launch_replies_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const crk_reply_req* reqs,
                                 const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
                                 cudaStream_t s) {
-  replies_sizes_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, reqs);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), replies_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs);
+    if (le != cudaSuccess) return le;
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
   e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
   if (e != cudaSuccess) return e;
-  replies_jobs_kernel<<<blocks_for(n), 256, 0, s>>>(sc, cfg, n, reqs, out, out_off, wire_offs, total, tot);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), replies_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs, out, out_off, wire_offs, total, tot);
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 
 cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n, cudaStream_t s) {
-  lens_prep_kernel<<<blocks_for(n), 256, 0, s>>>(sc, lens32_dev, n);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(sc.pdl != 0, lens_prep_kernel, blocks_for(n), 256, 0, s, sc, lens32_dev, n);
+    if (le != cudaSuccess) return le;
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   return launch_exclusive_scan_u64(sc.lens_pool + sc.max_lens, n, nullptr, nullptr, sc, s);

@@ -22,6 +22,7 @@ template <typename T>
 __global__ void __launch_bounds__(kScanBlock) scan_kernel(T* data, uint32_t n_static, const uint32_t* n_dev, T* total,
                                                           unsigned long long* state, uint32_t* block_counter,
                                                           uint32_t single) {
+  pdl_entry();
   __shared__ uint32_t s_bid;
   __shared__ uint64_t s_warp[kScanBlock / 32];
   __shared__ uint64_t s_excl;
@@ -95,16 +96,20 @@ cudaError_t launch_scan(T* data, uint32_t n, const uint32_t* n_dev, T* total, Sc
   const uint32_t per = kScanBlock * kScanIPT;
   const uint32_t blocks = n == 0 ? 1 : (n + per - 1) / per;
   if (blocks == 1) {  // one block: no look-back, no state to reset
-    scan_kernel<T><<<1, kScanBlock, 0, s>>>(data, n, n_dev, total, sc.scan_state, sc.counters + 5, 1u);
-    count_launch();
+    {
+    const cudaError_t le = launch_k_opt(sc.pdl != 0, scan_kernel<T>, 1, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 1u);
+    if (le != cudaSuccess) return le;
+  }
     return cudaGetLastError();
   }
   cudaError_t e = cudaMemsetAsync(sc.scan_state, 0, sizeof(unsigned long long) * (blocks + 1), s);
   if (e != cudaSuccess) return e;
   e = cudaMemsetAsync(sc.counters + 5, 0, sizeof(uint32_t), s);
   if (e != cudaSuccess) return e;
-  scan_kernel<T><<<blocks, kScanBlock, 0, s>>>(data, n, n_dev, total, sc.scan_state, sc.counters + 5, 0u);
-  count_launch();
+  {
+    const cudaError_t le = launch_k_opt(sc.pdl != 0, scan_kernel<T>, blocks, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 0u);
+    if (le != cudaSuccess) return le;
+  }
   return cudaGetLastError();
 }
 

@@ -9,6 +9,7 @@ namespace crk {
 namespace {
 
 __global__ void __launch_bounds__(1024) frame_scan_kernel(IndexDev ix, ScanRingsParam P, ConfigDev cfg) {
+  pdl_entry();
   TL_BEGIN(cfg, TL_SCAN);
   const uint32_t ring = blockIdx.x;
   RingDesc R = P.r[ring];
@@ -60,8 +61,10 @@ cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const
   if (!cfg.no_chunked_scan && chunk_plan(ix, p, sms, chunk_param.data())) {
     e = launch_chunk_scan(ix, chunk_param.data(), cfg, s);
   } else {
-    frame_scan_kernel<<<p.n_rings, cfg.scan_threads, 0, s>>>(ix, p, cfg);
-    count_launch();
+    {
+    const cudaError_t le = launch_k_opt(pdl_of(cfg), frame_scan_kernel, p.n_rings, cfg.scan_threads, 0, s, ix, p, cfg);
+    if (le != cudaSuccess) return le;
+  }
     e = cudaGetLastError();
   }
   prof_mark(PROF_SCAN, false, s);
