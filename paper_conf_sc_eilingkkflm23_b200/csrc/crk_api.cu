@@ -413,6 +413,7 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
       8 * (size_t)F, 8 * (size_t)F, 4 * (size_t)F,                              // frags
       8 * (size_t)R, 8 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R,               // records
       4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R,  // parsed scalars
+      4 * (size_t)R, 4 * (size_t)R, 4 * (size_t)R,                              // parsed fragment coordinates
       4 * MI, 8 * MI, 8 * MI, 8 * MI,                                           // items
       4 * (size_t)R, 4 * (size_t)R, 8 * (size_t)R, 8 * (size_t)R,               // serve
       8 * (size_t)hs,
@@ -444,6 +445,9 @@ int crk_index_create(crk_ctx* c, uint32_t max_rings, uint32_t max_frags, uint32_
   ix.p_proc = (uint32_t*)(b + off[i++]);
   ix.p_status = (int32_t*)(b + off[i++]);
   ix.p_nitems = (uint32_t*)(b + off[i++]);
+  ix.p_frag0 = (uint32_t*)(b + off[i++]);
+  ix.p_nfrags = (uint32_t*)(b + off[i++]);
+  ix.p_flen0 = (uint32_t*)(b + off[i++]);
   ix.p_kind = (uint32_t*)(b + off[i++]);
   ix.p_off = (uint64_t*)(b + off[i++]);
   ix.p_count = (uint64_t*)(b + off[i++]);

@@ -102,6 +102,9 @@ struct IndexDev {
   uint32_t* p_proc;
   int32_t* p_status;
   uint32_t* p_nitems;
+  uint32_t* p_frag0;            // the record's first fragment (absolute), fragment count, first fragment's length:
+  uint32_t* p_nfrags;           // written by the parser, so a decode job is built without the chain of
+  uint32_t* p_flen0;            // slot -> record table -> fragment table loads
   uint32_t* p_kind;
   uint64_t* p_off;
   uint64_t* p_count;

@@ -12,6 +12,7 @@ struct LogicalRecord {
   const uint64_t* lstart;
   const uint32_t* hdr;
   uint32_t nfrags;
+  uint32_t frag0;  // absolute index of the first fragment
   uint32_t hint;
   uint64_t len;
   uint64_t F0;
@@ -19,6 +20,7 @@ struct LogicalRecord {
   __device__ __forceinline__ void init(const IndexDev& ix, const RingDesc& r, uint32_t slot) {
     R = r;
     const uint32_t f0 = ix.rec_frag0[slot];
+    frag0 = f0;
     nfrags = ix.rec_nfrags[slot];
     len = ix.rec_len[slot];
     phys = ix.frag_phys + f0;

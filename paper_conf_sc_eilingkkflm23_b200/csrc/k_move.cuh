@@ -197,13 +197,12 @@ __device__ __forceinline__ uint8_t enc_wire_byte(const EncCtx& c, uint64_t w) {
 __device__ __forceinline__ void enc_bytes(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb) {
   for (uint64_t w = wa + T.tid; w < wb; w += T.nthr) c.O.base[(c.start + w) & c.O.mask] = enc_wire_byte(c, w);
 }
-__device__ void enc_segment_direct(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb, uint64_t src_at_wa,
-                                   uint32_t es) {
+// The interior 16-byte chunks of data run [wa, wb) (the aligned chunks it covers whole), from direct loads.
+__device__ void enc_segment_interior(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb, uint64_t src_at_wa,
+                                     uint32_t es) {
   const uint64_t ca = c.start + wa, cb = c.start + wb;
   const uint64_t c0 = (ca + 15) & ~15ull, c1 = cb & ~15ull;
-  if (c0 >= c1) { enc_bytes(T, c, wa, wb); return; }
-  enc_bytes(T, c, wa, wa + (c0 - ca));
-  enc_bytes(T, c, wb - (cb - c1), wb);
+  if (c0 >= c1) return;
   const uint64_t s0 = src_at_wa + (c0 - ca);
   const uint32_t sh = (uint32_t)(s0 & 15);
   const uint64_t ab = s0 - sh;
@@ -211,6 +210,41 @@ __device__ void enc_segment_direct(const Team& T, const EncCtx& c, uint64_t wa, 
   chunk_loop(T, (c1 - c0) >> 4, sh,
              [&](uint64_t i) { return swap16(ld16_stream(reinterpret_cast<const void*>(ab + 16 * i)), es); },
              [&](uint64_t i, uint4 v) { st16(O.base + ((c0 + 16 * i) & O.mask), v); });
+}
+__device__ void enc_segment_direct(const Team& T, const EncCtx& c, uint64_t wa, uint64_t wb, uint64_t src_at_wa,
+                                   uint32_t es) {
+  const uint64_t ca = c.start + wa, cb = c.start + wb;
+  const uint64_t c0 = (ca + 15) & ~15ull, c1 = cb & ~15ull;
+  if (c0 >= c1) { enc_bytes(T, c, wa, wb); return; }
+  enc_bytes(T, c, wa, wa + (c0 - ca));
+  enc_bytes(T, c, wb - (cb - c1), wb);
+  enc_segment_interior(T, c, wa, wb, src_at_wa, es);
+}
+// The output bytes of aligned chunks [g0, g1) (absolute out-ring cursors, 16-byte aligned) that lie inside
+// [xa, xb), composed chunk by chunk in registers from the exact wire map (fragment headers, REPLY / CALL words,
+// pads, data edges): one 16-byte store per chunk inside [xa, xb); byte stores only for a chunk the range cuts
+// (the first / last chunk of a job, shared with the neighbouring record).  Used for everything of an encode
+// tile outside its data runs' interior chunks, so a send ring in pinned host memory receives whole-chunk
+// writes over PCIe instead of single-byte ones (SURVEY.md §7 "PCIe efficiency").
+// A warp takes two chunks at a time: lane l computes byte l & 15 of chunk l >> 4 (all 32 in parallel), the
+// bytes are gathered into words and the words into the chunk's first lane with shuffles.
+__device__ void enc_gap_chunks(const Team& T, const EncCtx& c, uint64_t g0, uint64_t g1, uint64_t xa, uint64_t xb) {
+  const uint32_t lane = threadIdx.x & 31, j = lane & 15;
+  for (uint64_t p = g0 + 32ull * T.warp; p < g1; p += 32ull * T.nwarps) {  // warp-uniform
+    const uint64_t x0 = p + 16 * (lane >> 4), x = x0 + j;
+    const bool in = x0 < g1 && x >= xa && x < xb;
+    const bool whole = x0 < g1 && x0 >= xa && x0 + 16 <= xb;
+    const uint32_t b = in ? enc_wire_byte(c, x - c.start) : 0u;
+    uint32_t w = b | (__shfl_down_sync(0xffffffffu, b, 1) << 8) | (__shfl_down_sync(0xffffffffu, b, 2) << 16) |
+                 (__shfl_down_sync(0xffffffffu, b, 3) << 24);  // valid at j % 4 == 0
+    const uint32_t w1 = __shfl_down_sync(0xffffffffu, w, 4), w2 = __shfl_down_sync(0xffffffffu, w, 8),
+                   w3 = __shfl_down_sync(0xffffffffu, w, 12);
+    if (whole) {
+      if (j == 0) st16(c.O.base + (x0 & c.O.mask), make_uint4(w, w1, w2, w3));
+    } else if (in) {
+      c.O.base[x & c.O.mask] = (uint8_t)b;
+    }
+  }
 }
 // Walks wire range [ra, rb) of the record as runs: fragment headers, then per fragment the pieces'
 // data / literal parts.  emit(kind, wa, wb, src_at_wa, es) is called for each run in order.
@@ -247,12 +281,21 @@ __device__ __forceinline__ bool enc_runs(const EncCtx& c, uint64_t ra, uint64_t 
   }
   return true;
 }
+// Encode of wire range [ra, rb): each data run's interior chunks by 16-byte copies, everything between them
+// (headers, words, pads, data edges) by enc_gap_chunks, in wire order.
 __device__ void enc_tile_generic(const Team& T, const EncCtx& c, uint64_t ra, uint64_t rb) {
+  const uint64_t xa = c.start + ra, xb = c.start + rb;
+  uint64_t gap = xa & ~15ull;  // first chunk not yet written
   enc_runs(c, ra, rb, [&](uint32_t kind, uint64_t wa, uint64_t wb, uint64_t src, uint32_t es) {
-    if (kind == SEG_LIT) enc_bytes(T, c, wa, wb);
-    else enc_segment_direct(T, c, wa, wb, src, es);
+    if (kind == SEG_LIT) return true;
+    const uint64_t c0 = (c.start + wa + 15) & ~15ull, c1 = (c.start + wb) & ~15ull;
+    if (c0 >= c1) return true;
+    enc_gap_chunks(T, c, gap, c0, xa, xb);
+    enc_segment_interior(T, c, wa, wb, src, es);
+    gap = c1;
     return true;
   });
+  enc_gap_chunks(T, c, gap, (xb + 15) & ~15ull, xa, xb);
 }
 
 

@@ -162,6 +162,9 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
     if (strict && P.o != P.L.len) st = CRK_E_TRAILING;
   } while (0);
   ix.p_slot[d] = slot;
+  ix.p_frag0[d] = P.L.frag0;
+  ix.p_nfrags[d] = P.L.nfrags;
+  ix.p_flen0[d] = (uint32_t)P.L.F0;
   ix.p_ring[d] = ring;
   ix.p_xid[d] = xid;
   ix.p_proc[d] = proc;

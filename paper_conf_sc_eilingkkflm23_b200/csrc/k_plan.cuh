@@ -39,7 +39,14 @@ __device__ __forceinline__ uint64_t wire_of(uint64_t Ll, uint32_t F) {
 // A decode job carries its record's fragment-table coordinates (first fragment, count, ring, first
 // fragment length), so the mover's producer resolves a fresh job with one load instead of a chain of
 // record-table loads.
-__device__ __forceinline__ Job dec_job(const IndexDev& ix, uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec,
+// Its coordinates are the parser's per-record copies (p_frag0 / p_nfrags / p_flen0 / p_ring): one round trip.
+struct RecCoord {
+  uint32_t frag0, nfrags, flen0, ring;
+};
+__device__ __forceinline__ RecCoord rec_coord(const IndexDev& ix, uint32_t rec) {
+  return RecCoord{ix.p_frag0[rec], ix.p_nfrags[rec], ix.p_flen0[rec], ix.p_ring[rec]};
+}
+__device__ __forceinline__ Job dec_job(const RecCoord& rc, uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec,
                                        uint32_t es) {
   Job j{};
   j.type = nbytes ? JOB_DEC : JOB_NONE;
@@ -49,14 +56,16 @@ __device__ __forceinline__ Job dec_job(const IndexDev& ix, uint64_t dst, uint64_
   j.out_end = dst + nbytes;
   j.loff = loff;
   if (nbytes) {
-    const uint32_t slot = ix.p_slot[rec];
-    const uint32_t f0 = ix.rec_frag0[slot];
-    j.piece0 = f0;
-    j.n_pieces = ix.rec_nfrags[slot];
-    j.out_ring = ix.p_ring[rec];
-    j.F = ix.frag_hdr[f0] & 0x7fffffffu;
+    j.piece0 = rc.frag0;
+    j.n_pieces = rc.nfrags;
+    j.out_ring = rc.ring;
+    j.F = rc.flen0;
   }
   return j;
+}
+__device__ __forceinline__ Job dec_job(const IndexDev& ix, uint64_t dst, uint64_t nbytes, uint64_t loff, uint32_t rec,
+                                       uint32_t es) {
+  return dec_job(rec_coord(ix, rec), dst, nbytes, loff, rec, es);
 }
 
 // ---- serve: statuses, HtoD decode jobs and reply sizes (pass 1) --------------------------------
@@ -131,6 +140,7 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
   const uint32_t proc = ix.p_proc[d], xid = ix.p_xid[d];
   const uint64_t v0 = ix.p_value[b], v1 = ix.p_value[b + 1], v2 = ix.p_value[b + 2];
   const uint64_t c1 = ix.p_count[b + 1], o1 = ix.p_off[b + 1];
+  const RecCoord rc = rec_coord(ix, d);
   err = -1;
   Ll = 0;
   job = Job{};
@@ -140,7 +150,7 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
     const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
     if (cfg.strict && nb != size) { st = CRK_E_SIZE; err = 1; }
     else if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) { st = CRK_E_PTR; err = 1; }
-    else { err = 0; job = dec_job(ix, ptr, m, o1, d, 1); }
+    else { err = 0; job = dec_job(rc, ptr, m, o1, d, 1); }
     Ll = 28;
   } else if (st == CRK_OK && cfg.proc_stripe && proc == cfg.proc_stripe) {
     const uint64_t v3 = ix.p_value[b + 3], off = ix.p_value[b + 4], tot = ix.p_value[b + 5];
@@ -153,7 +163,7 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
       const uint64_t ptr = v0 + off;
       if (ptr < region_base || m > region_bytes || ptr - region_base > region_bytes - m) st = CRK_E_PTR;
       else {
-        job = dec_job(ix, ptr, m, o1, d, 1);
+        job = dec_job(rc, ptr, m, o1, d, 1);
         stripe_add(ix, (uint32_t)v3, v0, tot, m, off == 0, d);
         Ll = 28;  // the parent's reply, if this stripe turns out to lead a complete memcpy
       }
@@ -246,6 +256,15 @@ __device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_su
   return base + x - v;
 }
 
+#ifdef CRK_PLAN_TRACE
+// Diagnostic build only: %globaltimer at the sub-phases of plan_small_block (thread 0), per translation unit.
+__device__ unsigned long long g_plan_trace[16];
+#define PLAN_MARK(i) do { if (threadIdx.x == 0) { unsigned long long t_; \
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_)); g_plan_trace[i] = t_; } } while (0)
+#else
+#define PLAN_MARK(i) do { } while (0)
+#endif
+
 // Small batches (<= kSmallServe records): statuses, reply offsets, decode and encode jobs, their tile
 // prefix and the mover cursors, by one block of kSmallServe threads (thread d owns record d).
 // warp_sums (32) and ring_first_pre (kMaxRings) are the block's shared scratch.  Used by the
@@ -255,6 +274,7 @@ __device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_su
 __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
                                  uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
                                  uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr) {
+  PLAN_MARK(0);
   const uint32_t total = prefix_s ? prefix_s[S.n_rings] : *ix.total;
   const uint32_t d = threadIdx.x;
   for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
@@ -269,17 +289,19 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     first = prefix_s ? prefix_s[ring] : ix.rec_prefix[ring];
     end = prefix_s ? prefix_s[ring + 1] : ix.rec_prefix[ring + 1];
   }
-  if (cfg.proc_stripe) {  // every stripe of the step has decided: the leads of complete memcpys reply
-    __syncthreads();
-    if (d < total && st == CRK_OK && Ll == 28 && err < 0 && ix.p_proc[d] == cfg.proc_stripe &&
-        stripe_leads(ix, (uint32_t)ix.p_value[(uint64_t)d * kMaxItems + 3], d))
-      err = 0;
-  }
+  PLAN_MARK(1);
+  // every stripe of the step has decided: the leads of complete memcpys reply (the block-wide OR of "an OK
+  // stripe here" skips the parent table altogether in steps without stripes)
+  const bool my_stripe = cfg.proc_stripe && d < total && st == CRK_OK && Ll == 28 && err < 0;  // only OK stripes
+  const bool any_stripe = cfg.proc_stripe && __syncthreads_or(my_stripe);
+  if (my_stripe && stripe_leads(ix, (uint32_t)ix.p_value[(uint64_t)d * kMaxItems + 3], d)) err = 0;
   if (d < total) w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
+  PLAN_MARK(2);
   uint64_t tot;
   const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets
   if (d < total && d == first) ring_first_pre[ring] = pre;
   __syncthreads();
+  PLAN_MARK(3);
   Job enc{};
   if (d < total) {
     const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre - ring_first_pre[ring]);
@@ -297,6 +319,7 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     if (j.type == JOB_NONE || j.out_end <= j.out_start) return 0;
     return ((j.out_end - 1) >> cfg.tile_shift) - (j.out_start >> cfg.tile_shift) + 1;
   };
+  PLAN_MARK(4);
   const uint64_t td = d < total ? tiles_of(dec) : 0, te = d < total ? tiles_of(enc) : 0;
   uint64_t tot_d, tot_e;
   const uint64_t pd = block_excl_sum(td, warp_sums, &tot_d);
@@ -305,7 +328,8 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     sc.scan_tmp[d] = pd;
     sc.scan_tmp[total + d] = tot_d + pe;
   }
-  if (cfg.proc_stripe) {  // leave the parent table empty for the next step (every lead has read it)
+  PLAN_MARK(5);
+  if (any_stripe) {  // leave the parent table empty for the next step (every lead has read it)
     const uint32_t n = __ldcg(ix.stripe_n);
     stripe_clear(ix, n, threadIdx.x, blockDim.x);
     __syncthreads();
@@ -320,6 +344,7 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     sc.counters[1] = 2 * total;
     sc.counters[4] = total;
   }
+  PLAN_MARK(6);
 }
 
 }  // namespace

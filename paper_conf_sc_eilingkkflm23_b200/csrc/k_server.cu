@@ -230,6 +230,12 @@ extern "C" int crk_debug_server_scan_trace(unsigned long long* out, uint32_t* co
 }
 #endif
 
+#ifdef CRK_PLAN_TRACE
+extern "C" int crk_debug_server_plan_trace(unsigned long long* out16) {
+  return cudaMemcpyFromSymbol(out16, g_plan_trace, sizeof(g_plan_trace)) == cudaSuccess ? 0 : -100;
+}
+#endif
+
 cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SchemaTable* schemas,
                           crk_server_bell* bell, uint32_t n_rings, const crk_ring* rings, const crk_ring* send_rings,
                           uint64_t region_base, uint64_t region_bytes, cudaStream_t s) {

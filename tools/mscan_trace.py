@@ -18,16 +18,23 @@ L = crk.lib()
 L.crk_debug_mscan_trace.argtypes = [C.c_void_p]
 ctx = crk.Context(0)
 names = ["zone", "hop1", "score", "select", "walk", "resolve"]
-for label, mib in (("8MiB", 8), ("1GiB", 1024)):
-    n = mib * MiB
-    payload = gen.c3_payload(30)[:n]
-    Lr = O.call_header(0xC3, gen.PROG, gen.VERS, gen.PROC_H2D) + O.put_u64(0) + O.put_u32(n)
-    w = np.frombuffer(O.frame(Lr + payload.tobytes() + O.put_u64(n), 65536), np.uint8)
-    ring = crk.Ring.device(1 << 31)
-    ring.tensor()[:len(w)].copy_(torch.from_numpy(w.copy()))
-    idx = ctx.index(1, 1 << 15, 16)
+from paper_conf_sc_eilingkkflm23_b200 import workload  # noqa: E402
+for label, mib in (("8MiB", 8), ("1GiB", 1024), ("C5", 0)):
+    if label == "C5":  # the bench endpoint: 16 rings, mixed HtoD / DtoH memcpy CALLs
+        ep = workload.c5_endpoint(ctx, 0, torch.device("cuda:0"))
+        rings = ep.rings
+        idx = ctx.index(16, 1 << 20, 1 << 14)
+    else:
+        n = mib * MiB
+        payload = gen.c3_payload(30)[:n]
+        Lr = O.call_header(0xC3, gen.PROG, gen.VERS, gen.PROC_H2D) + O.put_u64(0) + O.put_u32(n)
+        w = np.frombuffer(O.frame(Lr + payload.tobytes() + O.put_u64(n), 65536), np.uint8)
+        ring = crk.Ring.device(1 << 31)
+        ring.tensor()[:len(w)].copy_(torch.from_numpy(w.copy()))
+        idx = ctx.index(1, 1 << 15, 16)
+        rings = [(ring, 0, len(w))]
     for _ in range(3):
-        idx.frame_scan([(ring, 0, len(w))])
+        idx.frame_scan(rings)
     torch.cuda.synchronize()
     buf = np.zeros((4096, 12), np.uint64)
     L.crk_debug_mscan_trace(buf.ctypes.data)
@@ -55,5 +62,5 @@ for label, mib in (("8MiB", 8), ("1GiB", 1024)):
     sums = crk.copy_to_host(ptrs[0], 64 * 4 * cap.value).view(SumT).reshape(cap.value, 4)[:len(t)]
     nc = (sums["kind"] != 0).sum(1)
     print("  candidates per chunk:", np.bincount(nc).tolist(), "kinds:", np.bincount(sums["kind"].ravel()).tolist())
-    del ring, idx
+    del rings, idx
     torch.cuda.empty_cache()
