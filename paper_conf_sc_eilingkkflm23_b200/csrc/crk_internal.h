@@ -290,6 +290,13 @@ cudaError_t launch_k_opt(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 blo
   count_launch();
   return cudaLaunchKernelEx(&c, kernel, static_cast<KArgs>(args)...);
 }
+// Launches a kernel through launch_k_opt; returns its error from the calling launcher.
+#define CRK_LAUNCH(...)                            \
+  do {                                             \
+    const cudaError_t le_ = launch_k_opt(__VA_ARGS__); \
+    if (le_ != cudaSuccess) return le_;            \
+  } while (0)
+
 // A context launches this way unless it keeps reserved mover CTAs (crk_config.mover_reserve_ctas > 0: a
 // pipelined server loop with batches in flight on several streams): there, kernels resident early would sit on
 // the SM slots the other batches' kernels need (measured: C5 step 0.347 -> 0.371 ms), while a lone call saves

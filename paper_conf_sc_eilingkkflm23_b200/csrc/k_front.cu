@@ -108,10 +108,7 @@ cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch
   P.region_base = region_base;
   P.region_bytes = region_bytes;
   prof_mark(PROF_SCAN, true, s);
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), front_small_kernel, 1, kFrontThreads, 0, s, P);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), front_small_kernel, 1, kFrontThreads, 0, s, P);
   prof_mark(PROF_SCAN, false, s);
   return cudaGetLastError();
 }

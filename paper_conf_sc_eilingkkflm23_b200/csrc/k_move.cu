@@ -687,17 +687,11 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   cudaError_t e;
   if (planned) {
   } else if (max_jobs_bound <= kSmallJobs) {
-    {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), plan_small_kernel, 1, 256, 0, s, sc, cfg, tiles, total, n_jobs_dev);
-    if (le != cudaSuccess) return le;
-  }
+    CRK_LAUNCH(pdl_of(cfg), plan_small_kernel, 1, 256, 0, s, sc, cfg, tiles, total, n_jobs_dev);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   } else {
     const uint32_t cnt_blocks = (max_jobs_bound + 255) / 256;
-    {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), plan_count_kernel, min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s, sc, cfg, tiles, n_jobs_dev);
-    if (le != cudaSuccess) return le;
-  }
+    CRK_LAUNCH(pdl_of(cfg), plan_count_kernel, min(cnt_blocks, (uint32_t)sms * 8), 256, 0, s, sc, cfg, tiles, n_jobs_dev);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     e = launch_exclusive_scan_u64(tiles, max_jobs_bound, n_jobs_dev, total, sc, s);
     if (e != cudaSuccess) return e;
@@ -713,10 +707,7 @@ cudaError_t launch_plan_and_move(const IndexDev* ix, const ConfigDev& cfg, Scrat
   }
   bool use_map = false;
   if (!planned && run > 1) {  // the run -> job map for this launch's run boundaries
-    {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), run_map_kernel, (uint32_t)sms * 2, 256, 0, s, sc, cfg, (uint32_t)move_ctas, run, tiles, n_jobs_dev, total);
-    if (le != cudaSuccess) return le;
-  }
+    CRK_LAUNCH(pdl_of(cfg), run_map_kernel, (uint32_t)sms * 2, 256, 0, s, sc, cfg, (uint32_t)move_ctas, run, tiles, n_jobs_dev, total);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     use_map = true;
   }

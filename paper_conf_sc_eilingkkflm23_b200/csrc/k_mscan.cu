@@ -822,15 +822,9 @@ cudaError_t launch_chunk_scan(const IndexDev& ix, const void* param, const Confi
   cudaError_t e = ensure_walk_smem();
   if (e != cudaSuccess) return e;
   const uint32_t n = P.chunk0[P.n_rings];
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), chunk_walk_kernel, n, kThreads, kZoneBytes, s, ix, P, cfg);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), chunk_walk_kernel, n, kThreads, kZoneBytes, s, ix, P, cfg);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), chunk_emit_kernel, n, kThreads, 0, s, ix, P, cfg);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), chunk_emit_kernel, n, kThreads, 0, s, ix, P, cfg);
   return cudaGetLastError();
 }
 

@@ -41,10 +41,7 @@ cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const C
   const uint64_t bound = (uint64_t)ix.recs_per_ring * n_rings;
   const uint64_t want = (bound + kParseWarps - 1) / kParseWarps, most = (uint64_t)sms * 8;
   const uint32_t grid = (uint32_t)(want < most ? want : most);
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), parse_kernel, grid ? grid : 1, kParseWarps * 32, 0, s, ix, schemas, cfg, n_rings);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), parse_kernel, grid ? grid : 1, kParseWarps * 32, 0, s, ix, schemas, cfg, n_rings);
   prof_mark(PROF_PARSE, false, s);
   return cudaGetLastError();
 }

@@ -333,11 +333,8 @@ cudaError_t launch_resolve_h2d(const IndexDev& ix, const ConfigDev& cfg, Scratch
                                const H2DReq* single, cudaStream_t s) {
   H2DReq one{};
   if (single) one = *single;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), resolve_h2d_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, xids, dsts, dst_bytes, statuses, copied, one,
+  CRK_LAUNCH(pdl_of(cfg), resolve_h2d_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, xids, dsts, dst_bytes, statuses, copied, one,
                                                     single ? 1u : 0u);
-    if (le != cudaSuccess) return le;
-  }
   return cudaGetLastError();
 }
 
@@ -345,10 +342,7 @@ cudaError_t launch_resolve_items(const IndexDev& ix, const ConfigDev& cfg, Scrat
                                  const crk_item_req* reqs, const crk_item_req* single, cudaStream_t s) {
   crk_item_req one{};
   if (single) one = *single;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), resolve_items_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, reqs, one, single ? 1u : 0u);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), resolve_items_kernel, blocks_for(n), 256, 0, s, ix, cfg, sc, n, reqs, one, single ? 1u : 0u);
   return cudaGetLastError();
 }
 
@@ -357,10 +351,7 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
                               uint64_t region_bytes, const uint64_t* doorbell, cudaStream_t s) {
   const uint32_t bound = ix.max_records;
   prof_mark(PROF_PLAN, true, s);
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan1_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, region_base, region_bytes);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), serve_plan1_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, region_base, region_bytes);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   e = launch_exclusive_scan_u64(sc.scan_tmp, bound, ix.total, nullptr, sc, s);
@@ -374,10 +365,7 @@ cudaError_t launch_serve_plan(const IndexDev& ix, const ConfigDev& cfg, Scratch&
     S.off[r] = send_offs ? send_offs[r] : 0;
   }
   S.doorbell = doorbell;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan2_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, S);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), serve_plan2_kernel, blocks_for(bound), 256, 0, s, ix, cfg, sc, S);
   prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();
 }
@@ -394,20 +382,14 @@ cudaError_t launch_serve_plan_small(const IndexDev& ix, const ConfigDev& cfg, Sc
   }
   S.doorbell = doorbell;
   prof_mark(PROF_PLAN, true, s);
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), serve_plan_small_kernel, 1, kSmallServe, 0, s, ix, cfg, sc, S, region_base, region_bytes);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), serve_plan_small_kernel, 1, kSmallServe, 0, s, ix, cfg, sc, S, region_base, region_bytes);
   prof_mark(PROF_PLAN, false, s);
   return cudaGetLastError();
 }
 
 cudaError_t launch_put_enc_jobs(Scratch& sc, const ConfigDev& cfg, const EncJobParam& p, const RingDesc& out,
                                 cudaStream_t s) {
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), put_enc_jobs_kernel, 1, 64, 0, s, sc, cfg, p, out);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), put_enc_jobs_kernel, 1, 64, 0, s, sc, cfg, p, out);
   return cudaGetLastError();
 }
 
@@ -415,47 +397,32 @@ cudaError_t launch_d2h_batch_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n,
                                   const void* const* srcs, const uint64_t* bytes, const int32_t* errs,
                                   const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
                                   cudaStream_t s) {
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), d2h_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, bytes, errs);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), d2h_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, bytes, errs);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
   e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
   if (e != cudaSuccess) return e;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), d2h_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
+  CRK_LAUNCH(pdl_of(cfg), d2h_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, xids, srcs, bytes, errs, out, out_off, wire_offs, total,
                                                  tot);
-    if (le != cudaSuccess) return le;
-  }
   return cudaGetLastError();
 }
 
 cudaError_t launch_replies_jobs(Scratch& sc, const ConfigDev& cfg, uint32_t n, const crk_reply_req* reqs,
                                 const RingDesc& out, uint64_t out_off, uint64_t* wire_offs, uint64_t* total,
                                 cudaStream_t s) {
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), replies_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), replies_sizes_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   uint64_t* tot = sc.scan_tmp + sc.max_jobs + 1;
   e = launch_exclusive_scan_u64(sc.scan_tmp, n, nullptr, tot, sc, s);
   if (e != cudaSuccess) return e;
-  {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), replies_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs, out, out_off, wire_offs, total, tot);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(pdl_of(cfg), replies_jobs_kernel, blocks_for(n), 256, 0, s, sc, cfg, n, reqs, out, out_off, wire_offs, total, tot);
   return cudaGetLastError();
 }
 
 cudaError_t launch_put_lens(Scratch& sc, const uint32_t* lens32_dev, uint32_t n, cudaStream_t s) {
-  {
-    const cudaError_t le = launch_k_opt(sc.pdl != 0, lens_prep_kernel, blocks_for(n), 256, 0, s, sc, lens32_dev, n);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(sc.pdl != 0, lens_prep_kernel, blocks_for(n), 256, 0, s, sc, lens32_dev, n);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   return launch_exclusive_scan_u64(sc.lens_pool + sc.max_lens, n, nullptr, nullptr, sc, s);

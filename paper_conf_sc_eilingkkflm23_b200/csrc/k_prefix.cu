@@ -96,20 +96,14 @@ cudaError_t launch_scan(T* data, uint32_t n, const uint32_t* n_dev, T* total, Sc
   const uint32_t per = kScanBlock * kScanIPT;
   const uint32_t blocks = n == 0 ? 1 : (n + per - 1) / per;
   if (blocks == 1) {  // one block: no look-back, no state to reset
-    {
-    const cudaError_t le = launch_k_opt(sc.pdl != 0, scan_kernel<T>, 1, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 1u);
-    if (le != cudaSuccess) return le;
-  }
+    CRK_LAUNCH(sc.pdl != 0, scan_kernel<T>, 1, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 1u);
     return cudaGetLastError();
   }
   cudaError_t e = cudaMemsetAsync(sc.scan_state, 0, sizeof(unsigned long long) * (blocks + 1), s);
   if (e != cudaSuccess) return e;
   e = cudaMemsetAsync(sc.counters + 5, 0, sizeof(uint32_t), s);
   if (e != cudaSuccess) return e;
-  {
-    const cudaError_t le = launch_k_opt(sc.pdl != 0, scan_kernel<T>, blocks, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 0u);
-    if (le != cudaSuccess) return le;
-  }
+  CRK_LAUNCH(sc.pdl != 0, scan_kernel<T>, blocks, kScanBlock, 0, s, data, n, n_dev, total, sc.scan_state, sc.counters + 5, 0u);
   return cudaGetLastError();
 }
 

@@ -61,10 +61,7 @@ cudaError_t launch_frame_scan(const IndexDev& ix, const ScanRingsParam& p, const
   if (!cfg.no_chunked_scan && chunk_plan(ix, p, sms, chunk_param.data())) {
     e = launch_chunk_scan(ix, chunk_param.data(), cfg, s);
   } else {
-    {
-    const cudaError_t le = launch_k_opt(pdl_of(cfg), frame_scan_kernel, p.n_rings, cfg.scan_threads, 0, s, ix, p, cfg);
-    if (le != cudaSuccess) return le;
-  }
+    CRK_LAUNCH(pdl_of(cfg), frame_scan_kernel, p.n_rings, cfg.scan_threads, 0, s, ix, p, cfg);
     e = cudaGetLastError();
   }
   prof_mark(PROF_SCAN, false, s);
