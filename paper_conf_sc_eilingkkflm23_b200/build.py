@@ -63,6 +63,8 @@ def build_trace() -> str:
 def build_variant(name: str, defines: list[str]) -> str:
     """Experiment build with extra -D defines (e.g. scan prefetch knobs) -> lib/libcrk_<name>.so."""
     out = os.path.join(PKG, "lib", f"libcrk_{name}.so")
+    if os.path.exists(out) and all(os.path.getmtime(d) <= os.path.getmtime(out) for d in deps()):
+        return out
     r = subprocess.run([NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-o", out, *sources()], capture_output=True,
                        text=True)
     if r.returncode != 0:

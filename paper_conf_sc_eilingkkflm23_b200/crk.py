@@ -656,6 +656,9 @@ class Server:
         if self.h:
             h, self.h = self.h, None
             _check(lib().crk_server_stop(h), "crk_server_stop")
+            # free the bell now, while no server runs: cudaFreeHost waits for the whole device, so freeing it
+            # later (when the object is collected) would block behind the next persistent server forever
+            self.buf.free()
 
     def __del__(self):
         try:

@@ -10,7 +10,7 @@ import torch
 
 import oracle as O
 from paper_conf_sc_eilingkkflm23_b200 import crk, gen
-from tests.gpu_util import ctx_for, d2h_call, h2d_call, ocfg
+from tests.gpu_util import ctx_for, d2h_call, h2d_call, make_ring, ocfg
 
 pytestmark = [pytest.mark.gpu, pytest.mark.timeout(300)]
 
@@ -176,3 +176,27 @@ def test_serve_steps_across_the_wrap_match_oracle(fused):
         for r in range(n_rings):
             tails[r] = want["consumed"][r] if step == 5 and r == 1 else tails[r]
             send_offs[r] += want["reply_bytes"][r]
+
+
+def test_servers_back_to_back_on_one_context():
+    """A persistent server stopped and another started on the same context and index (the binding frees each
+    bell at stop: freeing pinned memory later would wait for the next running server forever)."""
+    import gc
+    cfg = ocfg()
+    ctx = ctx_for(cfg)
+    region = torch.zeros(1 << 16, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    ring = make_ring(1 << 14)
+    payload = gen.random_bytes(9, 4096)
+    w = O.encode_call(7, gen.PROC_H2D, [(O.K_U64, base + 64), (O.K_OPAQUE_VAR, payload.tobytes()),
+                                        (O.K_U64, 4096)], cfg)
+    ring.write(0, w)
+    send = make_ring(1 << 12)
+    idx = ctx.index(1, 64, 16)
+    for rep in range(3):
+        srv = crk.Server(idx, [ring], [send], base, region.numel())
+        gc.collect()  # the previous server object goes away while this one runs
+        out = srv.step([(0, len(w))], [0], timeout_s=20)
+        assert out["results"][0]["status"] == O.OK and out["results"][0]["reply_bytes"] == 32
+        srv.stop()
+    assert region[64:64 + 4096].cpu().numpy().tobytes() == payload.tobytes()
