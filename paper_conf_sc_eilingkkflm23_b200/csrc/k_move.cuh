@@ -70,8 +70,19 @@ struct DecCtx {
   uint64_t dst, loff;
   uint32_t es;
 };
+// From the decode job's own record coordinates (dec_job: first fragment, count, ring, first fragment's length):
+// one round trip for the ring descriptor instead of the job -> record -> fragment table chain.
 __device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, const Job& j) {
-  c.L.init(ix, ix.rings[ix.p_ring[j.rec]], ix.p_slot[j.rec]);
+  LogicalRecord& L = c.L;
+  L.R = ix.rings[j.out_ring];
+  L.frag0 = j.piece0;
+  L.nfrags = j.n_pieces;
+  L.len = ~0ull;  // not needed by the decode paths (they stay inside the job's range)
+  L.phys = ix.frag_phys + j.piece0;
+  L.lstart = ix.frag_lstart + j.piece0;
+  L.hdr = ix.frag_hdr + j.piece0;
+  L.hint = 0;
+  L.F0 = j.F;
   c.dst = j.out_start;
   c.loff = j.loff;
   c.es = j.esize;
