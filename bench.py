@@ -339,8 +339,10 @@ def main():
     l0 = crk.kernel_launches()
     barrier()
     with ClockSampler(local) as clk:
+        torch.cuda.profiler.start()  # the timed region is the profiler window (ncu --profile-from-start off)
         e0, e1 = run(args.steps)
         torch.cuda.synchronize()
+        torch.cuda.profiler.stop()
     launches = crk.kernel_launches() - l0
     ms = e0.elapsed_time(e1) / args.steps
     ms_max = max_over_ranks(ms)

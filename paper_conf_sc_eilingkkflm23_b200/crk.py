@@ -14,7 +14,7 @@ import numpy as np
 import torch
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIBPATH = os.environ.get("CRK_LIB") or os.path.join(PKG, "lib", "libcrk.so")
+LIBPATH = os.environ.get("CRK_LIB") or os.path.join(PKG, "lib", "libcrk.so")  # CRK_LIB: a diagnostic / A-B build variant
 
 OK, INCOMPLETE = 0, 1
 E_ARG, E_TRUNCATED, E_FRAG, E_RPC, E_AUTH, E_PAD, E_SIZE = -1, -2, -3, -4, -5, -6, -7

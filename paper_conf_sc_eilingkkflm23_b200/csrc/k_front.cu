@@ -28,6 +28,15 @@ struct FrontParams {
   uint32_t plan;         // 0: scan + parse only (crk_rpc_frame_scan)
 };
 
+#ifdef CRK_FRONT_TRACE
+// Diagnostic build only: %globaltimer at the fused front end's phase ends (thread 0).
+__device__ unsigned long long g_front_trace[8];
+#define FRONT_MARK(i) do { if (threadIdx.x == 0) { unsigned long long t_; \
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_)); g_front_trace[i] = t_; } } while (0)
+#else
+#define FRONT_MARK(i) do { } while (0)
+#endif
+
 __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontParams P) {
   pdl_entry();
   __shared__ ScanState S;
@@ -36,6 +45,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   __shared__ uint64_t warp_sums[32];
   __shared__ uint64_t ring_first_pre[kMaxRings];
   __shared__ uint32_t prefix[kMaxRings + 1];
+  FRONT_MARK(0);
   TL_BEGIN(P.cfg, TL_FUSED);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const IndexDev& ix = P.ix;
@@ -45,6 +55,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
   __syncthreads();
+  FRONT_MARK(1);
   // ---- K1: each ring in turn by the whole CTA, then dense record numbering
   for (uint32_t r = 0; r < n_rings; ++r) {
     RingDesc R = P.rings.r[r];
@@ -59,6 +70,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   }
   if (threadIdx.x == 0) dense_numbering(ix, n_rings);
   __syncthreads();
+  FRONT_MARK(2);
   // ---- K3: one warp per record
   for (uint32_t i = threadIdx.x; i <= n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
   __syncthreads();
@@ -77,14 +89,22 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
     return;
   }
   __syncthreads();
+  FRONT_MARK(3);
   // ---- serve planning: statuses, reply offsets, jobs, their tile prefix, mover cursors
   plan_small_block(ix, P.cfg, P.sc, P.send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix);
+  FRONT_MARK(4);
   TL_END(P.cfg, TL_FUSED);
 }
 
 }  // namespace
 
 uint32_t front_small_threads() { return kFrontThreads; }
+
+#ifdef CRK_FRONT_TRACE
+extern "C" int crk_debug_front_trace(unsigned long long* out8) {
+  return cudaMemcpyFromSymbol(out8, g_front_trace, sizeof(g_front_trace)) == cudaSuccess ? 0 : -100;
+}
+#endif
 
 cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch& sc, const SchemaTable* schemas,
                                const ScanRingsParam& rings, uint32_t n_rings, const crk_ring* send_rings,

@@ -1,6 +1,10 @@
 // K3 kernel: one warp per record runs parse_record (k_parse.cuh).
 #include "k_parse.cuh"
 
+#ifndef CRK_PARSE_CTAS_PER_SM
+#define CRK_PARSE_CTAS_PER_SM 8
+#endif
+
 namespace crk {
 
 namespace {
@@ -39,7 +43,7 @@ cudaError_t launch_parse(const IndexDev& ix, const SchemaTable* schemas, const C
   prof_mark(PROF_PARSE, true, s);
   // no more CTAs than the index's record slots of these rings can occupy
   const uint64_t bound = (uint64_t)ix.recs_per_ring * n_rings;
-  const uint64_t want = (bound + kParseWarps - 1) / kParseWarps, most = (uint64_t)sms * 8;
+  const uint64_t want = (bound + kParseWarps - 1) / kParseWarps, most = (uint64_t)sms * CRK_PARSE_CTAS_PER_SM;
   const uint32_t grid = (uint32_t)(want < most ? want : most);
   CRK_LAUNCH(pdl_of(cfg), parse_kernel, grid ? grid : 1, kParseWarps * 32, 0, s, ix, schemas, cfg, n_rings);
   prof_mark(PROF_PARSE, false, s);

@@ -81,10 +81,11 @@ def main():
     a = ap.parse_args()
     tag = f"r{a.round:02d}"
     os.makedirs(PROF, exist_ok=True)
-    if os.path.exists(os.path.join(OUT, "launches.csv")):
-        json.dump(launches(os.path.join(OUT, "launches.csv")), open(os.path.join(PROF, f"{tag}_launches.json"), "w"),
-                  indent=1)
-    for name in ("mover", "scan"):
+    for lst in ("launches", "bench_launches", "smoke_launches"):
+        if os.path.exists(os.path.join(OUT, f"{lst}.csv")):
+            json.dump(launches(os.path.join(OUT, f"{lst}.csv")), open(os.path.join(PROF, f"{tag}_{lst}.json"), "w"),
+                      indent=1)
+    for name in ("mover", "scan", "walk", "emit"):
         rep = os.path.join(OUT, f"{name}.ncu-rep")
         if not os.path.exists(rep):
             continue
