@@ -539,25 +539,34 @@ __global__ void __launch_bounds__(kMoverThreads, CRK_MOVER_MIN_BLOCKS) mover_ker
         if (H.fallback) {
           enc_tile_generic(T, c, H.a - c.start, H.b - c.start);
         } else {
-          // data runs' interior chunks from the stage (or direct loads), then every other byte of the tile --
-          // fragment headers, REPLY words, pads, data edges -- composed per 16-byte chunk (enc_gap_chunks)
-          uint64_t gap = H.a & ~15ull;
+          // (composing the literal runs and data edges per 16-byte chunk instead -- enc_gap_chunks -- measured no
+          // PCIe-byte gain for host send rings and cost the pipelined step ~5%: the edges stay byte stores here)
           for (uint32_t g = 0; g < H.nseg; ++g) {
             const Seg S = H.seg[g];
             const uint32_t kind = S.flags >> 8 & 0xff, es = S.flags >> 16 & 0xff;
-            if (kind == SEG_LIT) continue;
-            const uint64_t c0 = (S.out_a + 15) & ~15ull, c1 = S.out_b & ~15ull;
-            if (c0 >= c1) continue;
-            enc_gap_chunks(T, c, gap, c0, H.a, H.b);
-            if (!(S.flags & 1)) {
-              enc_segment_interior(T, c, S.out_a - c.start, S.out_b - c.start, S.src, es);
-            } else {
-              const uint64_t s0 = S.src + (c0 - S.out_a);
-              staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, &H.R, es, false);
+            if (kind == SEG_LIT) {
+              enc_bytes(T, c, S.out_a - c.start, S.out_b - c.start);
+              continue;
             }
-            gap = c1;
+            if (!(S.flags & 1)) {
+              enc_segment_direct(T, c, S.out_a - c.start, S.out_b - c.start, S.src, es);
+              continue;
+            }
+            const uint64_t c0 = (S.out_a + 15) & ~15ull, c1 = S.out_b & ~15ull;
+            const uint64_t s0 = S.src + (c0 - S.out_a);
+            staged_chunks(T, buf + S.smem_off, (uint32_t)(s0 & 15), (c1 - c0) >> 4, c0, &H.R, es, false);
+            if (S.flags & 2) {  // edge bytes of plain data, from the widened stage window
+              const uint64_t ea = min(S.out_b, c0), eb = max(S.out_a, c1);
+              const uint32_t ne = (uint32_t)((ea - S.out_a) + (S.out_b - eb));
+              if (T.tid < ne) {
+                const uint64_t x = T.tid < ea - S.out_a ? S.out_a + T.tid : eb + (T.tid - (ea - S.out_a));
+                H.R.base[x & H.R.mask] = buf[(int64_t)S.smem_off + (int64_t)(S.src + (x - S.out_a) - (s0 & ~15ull))];
+              }
+            } else {
+              enc_bytes(T, c, S.out_a - c.start, min(S.out_b, c0) - c.start);
+              enc_bytes(T, c, max(S.out_a, c1) - c.start, S.out_b - c.start);
+            }
           }
-          enc_gap_chunks(T, c, gap, (H.b + 15) & ~15ull, H.a, H.b);
         }
       }
       mbar_arrive(&empty[s]);  // every consumer thread releases the stage after its last read of it

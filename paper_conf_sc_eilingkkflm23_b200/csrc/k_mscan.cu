@@ -74,8 +74,11 @@ __device__ __forceinline__ void mtrace(uint32_t ph) {
 #define MTRACE(ph) do { } while (0)
 #endif
 
+constexpr uint32_t kInlineChunks = 32;  // rings of at most this many chunks are emitted by their resolving CTA
+
 struct ChunkParam {
   uint32_t n_rings;
+  uint32_t need_emit;              // some ring has more than kInlineChunks chunks: chunk_emit_kernel runs
   uint32_t chunk0[kMaxRings + 1];  // exclusive prefix of the rings' chunk counts
   uint64_t S[kMaxRings];           // chunk size per ring
   RingDesc r[kMaxRings];
@@ -600,6 +603,48 @@ __device__ void resolve_ring(const IndexDev& ix, const ChunkParam& P, uint32_t r
   }
 }
 
+// Emission of chunk g's true chain by one warp (defined below).
+__device__ void emit_chunk(const IndexDev& ix, const ChunkParam& P, const ConfigDev& cfg, uint32_t r, uint32_t i,
+                           uint32_t g, const RingDesc& R, uint32_t lane);
+
+// Ring r's result from its chunks' emission (the first failing hop, else the end of the chain); resets the
+// ring's plan for the next launch.  One thread.
+__device__ void finalize_ring(const IndexDev& ix, uint32_t r, bool fb) {
+  RingPlan* pl = ix.ms.plan + r;
+  if (!fb) {
+    const unsigned long long key = __ldcg(&pl->stop_key);
+    crk_ring_result rr;
+    if (key != ~0ull) {
+      const ChunkStop* cs = ix.ms.stops + (key & 0xffffffull);
+      rr.status = __ldcg(&cs->status);
+      rr.n_records = __ldcg(&cs->nr);
+      rr.n_frags = __ldcg(&cs->kept);
+      rr.consumed = __ldcg(&cs->consumed);
+    } else {
+      rr.status = __ldcg(&pl->end.status);
+      rr.n_records = __ldcg(&pl->end.n_records);
+      rr.n_frags = __ldcg(&pl->end.n_frags);
+      rr.consumed = __ldcg(&pl->end.consumed);
+    }
+    rr.rec_base = 0;
+    rr.reply_bytes = 0;
+    ix.res[r] = rr;
+  }
+  pl->ticket_b = 0;
+  pl->stop_key = ~0ull;
+  pl->fallback = 0;
+}
+
+// Ring r is final: the last ring of the launch numbers the records densely across rings.  One thread.
+__device__ void ring_done(const IndexDev& ix, uint32_t n_rings) {
+  __threadfence();
+  if (atomicAdd(ix.ticket, 1u) == n_rings - 1) {
+    __threadfence();
+    dense_numbering(ix, n_rings);
+    *ix.ticket = 0;
+  }
+}
+
 __global__ void __launch_bounds__(kThreads) chunk_walk_kernel(IndexDev ix, ChunkParam P, ConfigDev cfg) {
   pdl_entry();
   TL_BEGIN(cfg, TL_SCAN);
@@ -615,6 +660,7 @@ __global__ void __launch_bounds__(kThreads) chunk_walk_kernel(IndexDev ix, Chunk
   const RingDesc R = P.r[r];
   if (K == 1) {  // a short window: the one-CTA scan
     scan_ring_cta(ix, R, false, r, cfg, S);
+    if (threadIdx.x == 0) ring_done(ix, P.n_rings);
     TL_END(cfg, TL_SCAN);
     return;
   }
@@ -655,6 +701,21 @@ __global__ void __launch_bounds__(kThreads) chunk_walk_kernel(IndexDev ix, Chunk
   if (last) {
     __threadfence();
     resolve_ring(ix, P, r, K, R, RS, zone);
+    if (K <= kInlineChunks) {  // a ring of few chunks is emitted here: its warps take the chunks in turn
+      __syncthreads();
+      const bool fb = __ldcg(&ix.ms.plan[r].fallback) != 0;
+      if (fb) {
+        scan_ring_cta(ix, R, false, r, cfg, S);  // no candidate fitted: the one-CTA scan of the whole window
+      } else {
+        for (uint32_t c = warp; c < K; c += blockDim.x >> 5) emit_chunk(ix, P, cfg, r, c, P.chunk0[r] + c, R, lane);
+        __syncthreads();
+      }
+      if (threadIdx.x == 0) {
+        __threadfence();
+        finalize_ring(ix, r, fb);
+        ring_done(ix, P.n_rings);
+      }
+    }
   }
   MTRACE(6);
   TL_END(cfg, TL_SCAN);
@@ -695,6 +756,7 @@ __device__ void emit_chunk(const IndexDev& ix, const ChunkParam& P, const Config
   }
 }
 
+// Rings of more than kInlineChunks chunks: one CTA per chunk emits it; the ring's last CTA finalizes it.
 __global__ void __launch_bounds__(kThreads) chunk_emit_kernel(IndexDev ix, ChunkParam P, ConfigDev cfg) {
   pdl_entry();
   TL_BEGIN(cfg, TL_SCAN);
@@ -702,53 +764,27 @@ __global__ void __launch_bounds__(kThreads) chunk_emit_kernel(IndexDev ix, Chunk
   __shared__ uint32_t last, fb;
   uint32_t r, i, K;
   locate(P, blockIdx.x, r, i, K);
-  const RingDesc R = P.r[r];
-  if (K > 1) {
-    RingPlan* pl = ix.ms.plan + r;
-    if (threadIdx.x == 0) fb = __ldcg(&pl->fallback);
-    __syncthreads();
-    if (fb) {
-      if (i == 0) scan_ring_cta(ix, R, false, r, cfg, S);  // the one-CTA scan of the whole window
-    } else if (threadIdx.x < 32) {
-      emit_chunk(ix, P, cfg, r, i, blockIdx.x, R, threadIdx.x);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      last = atomicAdd(&pl->ticket_b, 1u) == K - 1;
-      if (last) {
-        __threadfence();
-        if (!fb) {
-          const unsigned long long key = __ldcg(&pl->stop_key);
-          crk_ring_result rr;
-          if (key != ~0ull) {
-            const ChunkStop* cs = ix.ms.stops + (key & 0xffffffull);
-            rr.status = __ldcg(&cs->status);
-            rr.n_records = __ldcg(&cs->nr);
-            rr.n_frags = __ldcg(&cs->kept);
-            rr.consumed = __ldcg(&cs->consumed);
-          } else {
-            rr.status = __ldcg(&pl->end.status);
-            rr.n_records = __ldcg(&pl->end.n_records);
-            rr.n_frags = __ldcg(&pl->end.n_frags);
-            rr.consumed = __ldcg(&pl->end.consumed);
-          }
-          rr.rec_base = 0;
-          rr.reply_bytes = 0;
-          ix.res[r] = rr;
-        }
-        pl->ticket_b = 0;
-        pl->stop_key = ~0ull;
-        pl->fallback = 0;
-      }
-    }
+  if (K <= kInlineChunks) {  // one-CTA rings and rings emitted by their resolver are final already
+    TL_END(cfg, TL_SCAN);
+    return;
   }
-  if (threadIdx.x == 0) {  // the last CTA numbers the records densely across rings
+  const RingDesc R = P.r[r];
+  RingPlan* pl = ix.ms.plan + r;
+  if (threadIdx.x == 0) fb = __ldcg(&pl->fallback);
+  __syncthreads();
+  if (fb) {
+    if (i == 0) scan_ring_cta(ix, R, false, r, cfg, S);  // the one-CTA scan of the whole window
+  } else if (threadIdx.x < 32) {
+    emit_chunk(ix, P, cfg, r, i, blockIdx.x, R, threadIdx.x);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
     __threadfence();
-    if (atomicAdd(ix.ticket, 1u) == gridDim.x - 1) {
+    last = atomicAdd(&pl->ticket_b, 1u) == K - 1;
+    if (last) {
       __threadfence();
-      dense_numbering(ix, P.n_rings);
-      *ix.ticket = 0;
+      finalize_ring(ix, r, fb != 0);
+      ring_done(ix, P.n_rings);
     }
   }
   TL_END(cfg, TL_SCAN);
@@ -803,6 +839,8 @@ bool chunk_plan(const IndexDev& ix, const ScanRingsParam& p, int sms, void* out_
       if (!multi) return false;
       P.chunk0[p.n_rings] = acc;
       P.n_rings = p.n_rings;
+      P.need_emit = 0;
+      for (uint32_t r = 0; r < p.n_rings; ++r) P.need_emit |= P.chunk0[r + 1] - P.chunk0[r] > kInlineChunks;
       for (uint32_t r = 0; r < p.n_rings; ++r) P.r[r] = p.r[r];
       return true;
     }
@@ -824,7 +862,7 @@ cudaError_t launch_chunk_scan(const IndexDev& ix, const void* param, const Confi
   const uint32_t n = P.chunk0[P.n_rings];
   CRK_LAUNCH(pdl_of(cfg), chunk_walk_kernel, n, kThreads, kZoneBytes, s, ix, P, cfg);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  CRK_LAUNCH(pdl_of(cfg), chunk_emit_kernel, n, kThreads, 0, s, ix, P, cfg);
+  if (P.need_emit) CRK_LAUNCH(pdl_of(cfg), chunk_emit_kernel, n, kThreads, 0, s, ix, P, cfg);
   return cudaGetLastError();
 }
 
