@@ -118,7 +118,8 @@ typedef struct {
   uint32_t proc_h2d_stripe;  /* built-in schema (ptr u64, mem opaque<>, size u64, parent u32, offset u64, total u64):
                                 one stripe of a memcpy sent over several connections (reading R22;
                                 default 3, 0 = no such procedure) */
-  uint32_t pad1_;
+  uint32_t mover_max_ctas;    /* cap on the mover's grid (0 = every CTA slot the occupancy allows); a small grid
+                                leaves HBM to concurrent copy-engine traffic in a host-ring server loop */
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;

@@ -294,6 +294,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   CK(cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device));
   int occ = cfg.ctas_per_sm ? (int)cfg.ctas_per_sm : mover_occupancy(cfg.tile_bytes, cfg.mover_stages);
   c->move_ctas = c->sms * (occ > 0 ? occ : 1);
+  if (cfg.mover_max_ctas && (uint32_t)c->move_ctas > cfg.mover_max_ctas) c->move_ctas = (int)cfg.mover_max_ctas;
   if (2ull * cfg.mover_reserve_ctas >= (uint64_t)c->move_ctas) { delete c; return CRK_E_ARG; }
   ConfigDev& d = c->cd;
   d.F = cfg.frag_payload;

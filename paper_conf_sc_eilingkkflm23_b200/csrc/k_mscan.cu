@@ -836,7 +836,7 @@ bool chunk_plan(const IndexDev& ix, const ScanRingsParam& p, int sms, void* out_
       multi |= K > 1;
     }
     if (fits && acc <= ix.ms.chunk_cap) {
-      if (!multi) return false;
+      if (!multi || S > (1ull << 31)) return false;  // logs keep cursors as 32-bit offsets into the chunk
       P.chunk0[p.n_rings] = acc;
       P.n_rings = p.n_rings;
       P.need_emit = 0;
