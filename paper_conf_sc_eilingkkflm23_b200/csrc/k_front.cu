@@ -56,7 +56,8 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
   __syncthreads();
   FRONT_MARK(1);
-  // ---- K1: each ring in turn by the whole CTA, then dense record numbering
+  // ---- K1: each ring in turn by the whole CTA, then dense record numbering (prefix[] in shared memory)
+  if (threadIdx.x == 0) prefix[0] = 0;
   for (uint32_t r = 0; r < n_rings; ++r) {
     RingDesc R = P.rings.r[r];
     bool bad = false;
@@ -67,13 +68,12 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
       if (bad) R.tail = R.head;
     }
     scan_ring_cta(ix, R, bad, r, P.cfg, S);
+    if (threadIdx.x == 0) prefix[r + 1] = prefix[r] + S.nr;
   }
-  if (threadIdx.x == 0) dense_numbering(ix, n_rings);
+  if (threadIdx.x == 0) dense_numbering_cta(ix, n_rings, prefix);
   __syncthreads();
   FRONT_MARK(2);
   // ---- K3: one warp per record
-  for (uint32_t i = threadIdx.x; i <= n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
-  __syncthreads();
   const uint32_t total = prefix[n_rings];
   for (uint32_t d = warp; d < total; d += kFrontWarps) {
     uint32_t lo = 0, hi = n_rings;  // ring of dense record d
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
       const uint32_t mid = (lo + hi) >> 1;
       if (prefix[mid] <= d) lo = mid; else hi = mid;
     }
-    parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane);
+    parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane, total == 1);
     __syncwarp();
   }
   if (!P.plan) {

@@ -30,7 +30,7 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
       uint32_t mid = (lo + hi) >> 1;
       if (prefix[mid] <= d) lo = mid; else hi = mid;
     }
-    parse_record(ix, sch, cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane);
+    parse_record(ix, sch, cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane, total == 1);
     __syncwarp();  // the head buffer is free for the warp's next record
   }
   TL_END(cfg, TL_PARSE);

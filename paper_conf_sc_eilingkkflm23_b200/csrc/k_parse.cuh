@@ -43,7 +43,9 @@ struct Parser {
   __device__ int get_u32(uint32_t& v) {
     if (o + 4 > L.len) return CRK_E_TRUNCATED;
     const uint8_t* b = o + 4 <= nhead ? head + o : o >= tail_lo ? tail + (o - tail_lo) : nullptr;
-    if (b)
+    if (b && !(reinterpret_cast<uintptr_t>(b) & 3))  // one shared-memory word, byte-swapped (big-endian)
+      v = __byte_perm(*reinterpret_cast<const uint32_t*>(b), 0, 0x0123);
+    else if (b)
       v = ((uint32_t)b[0] << 24) | ((uint32_t)b[1] << 16) | ((uint32_t)b[2] << 8) | b[3];
     else
       v = L.be32(o);
@@ -72,8 +74,10 @@ struct Parser {
 // Parse of dense record d (ring `ring`, index slot `slot`) by one warp: lane 0 runs the checks in the
 // oracle's order and writes the parsed-call tables and the xid table; head_buf is the warp's kHeadBuf-byte
 // shared buffer for the record head.  Used by K3 (one warp per record) and by the persistent server.
+// `sole`: d is the step's only record, so its xid goes into the (cleared) table with a plain store instead
+// of a compare-and-swap whose result the warp would wait for.
 __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const ConfigDev& cfg, uint32_t d,
-                             uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane) {
+                             uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane, bool sole = false) {
   Parser P;
   P.L.init(ix, ix.rings[ring], slot);
   P.o = 0;
@@ -85,9 +89,10 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
   P.nhead = nh < kHead ? (uint32_t)nh : kHead;
   const uint32_t kl = P.L.nfrags - 1;
   const uint64_t ls_last = P.L.lstart[kl], ph_last = P.L.phys[kl];
+  // the tail window starts at most kTail bytes before the end, inside the last fragment and past the head
   const uint64_t want = P.L.len > kTail ? P.L.len - kTail : 0;
-  const uint64_t tlo = want > P.nhead ? want : P.nhead;
-  P.tail_lo = (P.L.len > P.nhead && ls_last <= tlo) ? tlo : P.L.len;
+  const uint64_t tlo = max(max(want, (uint64_t)P.nhead), ls_last);
+  P.tail_lo = P.L.len > tlo ? tlo : P.L.len;
   const uint32_t ntail = (uint32_t)(P.L.len - P.tail_lo);
   P.head = head_buf;
   P.tail = head_buf + kHead;
@@ -173,6 +178,10 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
   if (P.L.len >= 4) {  // xid readable: insert, the smallest dense id wins (reading R11)
     const unsigned long long key = ((unsigned long long)xid << 32) | d;
     uint32_t h = (xid * 0x9E3779B1u) & ix.hash_mask;
+    if (sole) {
+      ix.xid_hash[h] = key;
+      return;
+    }
     for (;;) {
       unsigned long long old = atomicCAS(ix.xid_hash + h, ~0ull, key);
       if (old == ~0ull) break;

@@ -92,7 +92,7 @@ __global__ void serve_plan1_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, uint6
     int32_t err;
     uint64_t Ll;
     Job job;
-    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, job);
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, job, total == 1);
     ix.s_status[d] = st;
     ix.s_reply_err[d] = err;
     const uint64_t w = err >= 0 ? wire_of(Ll, cfg.F) : 0;

@@ -132,8 +132,10 @@ __device__ __forceinline__ void stripe_clear(const IndexDev& ix, uint32_t n, uin
 // reply logical length, and the HtoD decode job.  A striped memcpy's stripe (reading R22) decides like an
 // HtoD copy to ptr + offset with no reply; whether the offset-0 stripe carries its parent's reply is known
 // only once every stripe of the step has decided (stripe_leads, after a block / grid barrier).
+// `sole`: d is the step's only record, so it owns its xid without a lookup.
 __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev& cfg, uint32_t d, uint64_t region_base,
-                                             uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job) {
+                                             uint64_t region_bytes, int& st, int32_t& err, uint64_t& Ll, Job& job,
+                                             bool sole = false) {
   // every field the decision can need is loaded at once (one memory round trip), then the xid lookup
   const uint64_t b = (uint64_t)d * kMaxItems;
   st = ix.p_status[d];
@@ -144,7 +146,7 @@ __device__ __forceinline__ void serve_decide(const IndexDev& ix, const ConfigDev
   err = -1;
   Ll = 0;
   job = Job{};
-  if (st == CRK_OK && xid_lookup(ix, xid) != d) st = CRK_E_XID;
+  if (st == CRK_OK && !sole && xid_lookup(ix, xid) != d) st = CRK_E_XID;
   if (st == CRK_OK && proc == cfg.proc_h2d) {
     const uint64_t ptr = v0, nb = c1, size = v2;
     const uint64_t m = (cfg.strict || nb <= size) ? nb : size;
@@ -284,6 +286,28 @@ __device__ __forceinline__ uint64_t block_excl_sum(uint64_t v, uint64_t* warp_su
   return a[0];
 }
 
+// The same exclusive sums over one warp (no block barrier): tot[] = the warp totals.
+template <int NV>
+__device__ __forceinline__ void warp_excl_sums(uint64_t (&v)[NV], uint64_t (&tot)[NV]) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t x[NV];
+#pragma unroll
+  for (int k = 0; k < NV; ++k) x[k] = v[k];
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      const uint64_t y = __shfl_up_sync(0xffffffffu, x[k], o);
+      if (lane >= (uint32_t)o) x[k] += y;
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    tot[k] = __shfl_sync(0xffffffffu, x[k], 31);
+    v[k] = x[k] - v[k];
+  }
+}
+
 #ifdef CRK_PLAN_TRACE
 // Diagnostic build only: %globaltimer at the sub-phases of plan_small_block (thread 0), per translation unit.
 __device__ unsigned long long g_plan_trace[16];
@@ -298,14 +322,15 @@ __device__ unsigned long long g_plan_trace[16];
 // warp_sums (32) and ring_first_pre (kMaxRings) are the block's shared scratch.  Used by the
 // single-block planning kernel, the fused front end and the persistent server; the latter two pass the
 // dense record prefix they already hold in shared memory (prefix_s, n_rings + 1 entries), which saves the
-// dependent loads of the record total and of each record's ring bounds.
-__device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
-                                 uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
-                                 uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr) {
+// dependent loads of the record total and of each record's ring bounds.  kOneWarp: a step of at most 32
+// records is planned by warp 0 alone, its sums by shuffles, with no block barrier.
+template <bool kOneWarp>
+__device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
+                                uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
+                                uint64_t* ring_first_pre, const uint32_t* prefix_s, uint32_t total) {
   PLAN_MARK(0);
-  const uint32_t total = prefix_s ? prefix_s[S.n_rings] : *ix.total;
-  const uint32_t d = threadIdx.x;
-  for (uint32_t r = threadIdx.x; r < S.n_rings; r += blockDim.x) sc.out_rings[r] = S.r[r];
+  const uint32_t d = threadIdx.x, nthreads = kOneWarp ? 32u : blockDim.x;
+  for (uint32_t r = threadIdx.x; r < S.n_rings; r += nthreads) sc.out_rings[r] = S.r[r];
   int st = CRK_OK;
   int32_t err = -1;
   uint64_t Ll = 0, w = 0;
@@ -313,7 +338,7 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   uint32_t ring = 0, first = 0, end = 0;
   if (d < total) {
     ring = ix.p_ring[d];
-    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec);
+    serve_decide(ix, cfg, d, region_base, region_bytes, st, err, Ll, dec, total == 1);
     first = prefix_s ? prefix_s[ring] : ix.rec_prefix[ring];
     end = prefix_s ? prefix_s[ring + 1] : ix.rec_prefix[ring + 1];
   }
@@ -321,14 +346,24 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   // every stripe of the step has decided: the leads of complete memcpys reply (the block-wide OR of "an OK
   // stripe here" skips the parent table altogether in steps without stripes)
   const bool my_stripe = cfg.proc_stripe && d < total && st == CRK_OK && Ll == 28 && err < 0;  // only OK stripes
-  const bool any_stripe = cfg.proc_stripe && __syncthreads_or(my_stripe);
+  if (kOneWarp) __syncwarp();  // orders the warp's parent-table atomics before the leads read the table
+  const bool any_stripe =
+      cfg.proc_stripe && (kOneWarp ? __any_sync(0xffffffffu, my_stripe) : __syncthreads_or(my_stripe));
   if (my_stripe && stripe_leads(ix, (uint32_t)ix.p_value[(uint64_t)d * kMaxItems + 3], d)) err = 0;
   if (d < total) w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   PLAN_MARK(2);
-  uint64_t tot;
-  const uint64_t pre = block_excl_sum(w, warp_sums, &tot);  // reply sizes -> offsets
+  uint64_t tot, pre;
+  if (kOneWarp) {  // reply sizes -> offsets
+    uint64_t a[1] = {w}, t[1];
+    warp_excl_sums<1>(a, t);
+    pre = a[0];
+    tot = t[0];
+  } else {
+    pre = block_excl_sum(w, warp_sums, &tot);
+  }
+  (void)tot;
   if (d < total && d == first) ring_first_pre[ring] = pre;
-  __syncthreads();
+  if (kOneWarp) __syncwarp(); else __syncthreads();
   PLAN_MARK(3);
   Job enc{};
   if (d < total) {
@@ -350,7 +385,8 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   PLAN_MARK(4);
   __shared__ uint64_t ws2[64];
   uint64_t tv[2] = {d < total ? tiles_of(dec) : 0, d < total ? tiles_of(enc) : 0}, tt[2];
-  block_excl_sums<2>(tv, ws2, tt);  // decode and encode tile counts in one pass
+  if (kOneWarp) warp_excl_sums<2>(tv, tt);
+  else block_excl_sums<2>(tv, ws2, tt);  // decode and encode tile counts in one pass
   const uint64_t pd = tv[0], pe = tv[1], tot_d = tt[0], tot_e = tt[1];
   if (d < total) {
     sc.scan_tmp[d] = pd;
@@ -359,8 +395,8 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
   PLAN_MARK(5);
   if (any_stripe) {  // leave the parent table empty for the next step (every lead has read it)
     const uint32_t n = __ldcg(ix.stripe_n);
-    stripe_clear(ix, n, threadIdx.x, blockDim.x);
-    __syncthreads();
+    stripe_clear(ix, n, threadIdx.x, nthreads);
+    if (kOneWarp) __syncwarp(); else __syncthreads();
     if (d == 0 && n) *ix.stripe_n = 0;
   }
   if (d == 0) {
@@ -373,6 +409,18 @@ __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const
     sc.counters[4] = total;
   }
   PLAN_MARK(6);
+}
+
+__device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
+                                 uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
+                                 uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr) {
+  const uint32_t total = prefix_s ? prefix_s[S.n_rings] : *ix.total;
+  if (total <= 32) {
+    if (threadIdx.x < 32)
+      plan_small_impl<true>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total);
+  } else {
+    plan_small_impl<false>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total);
+  }
 }
 
 }  // namespace

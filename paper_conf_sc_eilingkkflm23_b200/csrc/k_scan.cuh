@@ -675,5 +675,17 @@ __device__ __forceinline__ void dense_numbering(const IndexDev& ix, uint32_t n_r
   *ix.total = acc;
 }
 
+// The same numbering when one CTA scanned every ring: after ring r's scan_ring_cta, thread 0 sets
+// prefix[r + 1] = prefix[r] + S.nr (shared memory), so no result is read back; thread 0 then writes the
+// tables with stores only.
+__device__ __forceinline__ void dense_numbering_cta(const IndexDev& ix, uint32_t n_rings, const uint32_t* prefix) {
+  for (uint32_t r = 0; r < n_rings; ++r) {
+    ix.rec_prefix[r] = prefix[r];
+    ix.res[r].rec_base = prefix[r];
+  }
+  ix.rec_prefix[n_rings] = prefix[n_rings];
+  *ix.total = prefix[n_rings];
+}
+
 }  // namespace
 }  // namespace crk

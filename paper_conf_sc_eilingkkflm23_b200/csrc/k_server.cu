@@ -21,6 +21,7 @@ namespace {
 
 constexpr uint32_t kServerThreads = kSmallServe;  // plan_small_block: thread d owns record d
 constexpr uint32_t kServerWarps = kServerThreads / 32;
+static_assert(kMaxRings <= kServerThreads, "thread r < n_rings holds ring r's result");
 
 struct ServerParams {
   IndexDev ix;
@@ -130,6 +131,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     // ---- K1: each ring in turn by the whole CTA
     SCAN_TRACE(threadIdx.x == 0, 5, 0);
+    if (threadIdx.x == 0) prefix[0] = 0;
     for (uint32_t r = 0; r < P.n_rings; ++r) {
       RingDesc R = P.rings[r];
       R.head = win_head[r];
@@ -140,8 +142,9 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
         if (threadIdx.x == 0) bad_s = 1;
       }
       scan_ring_cta(ix, R, bad, r, P.cfg, S);
+      if (threadIdx.x == 0) prefix[r + 1] = prefix[r] + S.nr;
     }
-    if (threadIdx.x == 0) dense_numbering(ix, P.n_rings);
+    if (threadIdx.x == 0) dense_numbering_cta(ix, P.n_rings, prefix);
     phase_sync();
     TL_END(P.cfg, 1);
     if (threadIdx.x == 0) B->t_phase_ns[1] = gtimer();
@@ -153,14 +156,13 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
       const bool bad = R.tail < R.head || R.tail - R.head > R.mask + 1;
       if (bad) R.tail = R.head;
       scan_ring_cta(ix, R, bad, r, P.cfg, S);
+      if (threadIdx.x == 0) prefix[r + 1] = prefix[r] + S.nr;
     }
-    if (threadIdx.x == 0) dense_numbering(ix, P.n_rings);
+    if (threadIdx.x == 0) dense_numbering_cta(ix, P.n_rings, prefix);
     phase_sync();
     TL_END(P.cfg, 7);
 #endif
-    // ---- K3: one warp per record
-    for (uint32_t i = threadIdx.x; i <= P.n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
-    __syncthreads();
+    // ---- K3: one warp per record (prefix[] is the scan's dense numbering, in shared memory)
     const uint32_t total = prefix[P.n_rings];
     for (uint32_t d = warp; d < total; d += kServerWarps) {
       uint32_t lo = 0, hi = P.n_rings;  // ring of dense record d
@@ -168,7 +170,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
         const uint32_t mid = (lo + hi) >> 1;
         if (prefix[mid] <= d) lo = mid; else hi = mid;
       }
-      parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane);
+      parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane, total == 1);
       __syncwarp();
     }
     phase_sync();
@@ -182,13 +184,18 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     // ---- movers: every job cut into 8 KiB output tiles, tiles dealt to the warps round-robin
     const uint32_t n_jobs = 2 * total;
     const Team TW{lane, 32, 0, 1};
+    // plan's tile total (cfg tiles) and the step's final ring results, loaded with the jobs in the same
+    // round trip (the results are published after the move)
+    const uint64_t plan_tiles = P.sc.scan_tmp[P.sc.max_jobs + 1];
+    crk_ring_result my_res;
+    if (threadIdx.x < P.n_rings) my_res = ix.res[threadIdx.x];
     {  // the first kJobCache jobs in one round trip (every warp walks every job's descriptor)
       const uint32_t nc = n_jobs < kJobCache ? n_jobs : kJobCache;
       for (uint32_t i = threadIdx.x; i < nc * (uint32_t)(sizeof(Job) / 4); i += blockDim.x)
         reinterpret_cast<uint32_t*>(jobs_s)[i] = reinterpret_cast<const uint32_t*>(P.sc.jobs)[i];
       __syncthreads();
     }
-    const uint32_t sh = P.sc.scan_tmp[P.sc.max_jobs + 1] <= 4 ? 11u : 13u;  // plan's tile total (cfg tiles)
+    const uint32_t sh = plan_tiles <= 4 ? 11u : 13u;
     uint64_t first = 0;  // global number of the job's first tile
     for (uint32_t j = 0; j < n_jobs; ++j) {
       const Job J = j < kJobCache ? jobs_s[j] : P.sc.jobs[j];
@@ -201,7 +208,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     TL_END(P.cfg, 4);
     if (threadIdx.x == 0) B->t_phase_ns[4] = gtimer();
     // ---- publish: results into the bell, then done_seq
-    for (uint32_t r = threadIdx.x; r < P.n_rings; r += blockDim.x) B->res[r] = ix.res[r];
+    if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
     __syncthreads();
     if (threadIdx.x == 0) {
       B->status = bad_s ? CRK_E_ARG : CRK_OK;
