@@ -112,6 +112,18 @@ __device__ __forceinline__ unsigned long long tl_now() {
 #define TL_END(cfg, st) do { } while (0)
 #endif
 
+// Diagnostic step trace (-DCRK_STEP_TRACE builds; tools/server_step_trace.py): %globaltimer at numbered points
+// of one small step, taken once `dep` (a value the point waits for) is available.  One array per translation
+// unit (the persistent server's is exported).
+#ifdef CRK_STEP_TRACE
+__device__ unsigned long long g_step_trace[32];
+#define STEP_MARK(cond, i, dep) do { if (cond) { unsigned long long t_; \
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_) : "r"((uint32_t)(dep)) : "memory"); \
+  g_step_trace[i] = t_; } } while (0)
+#else
+#define STEP_MARK(cond, i, dep) do { } while (0)
+#endif
+
 // Block-wide min of a u32 (all threads must call).  smem: >= 32 words.
 __device__ __forceinline__ uint32_t block_min_u32(uint32_t v, uint32_t* smem) {
 #pragma unroll

@@ -30,25 +30,34 @@ constexpr uint32_t kHead = 64;  // record head prefetched by the warp (CALL head
 constexpr uint32_t kTail = 64;  // record tail prefetched with it (the arguments after a bulk opaque<>)
 constexpr uint32_t kHeadBuf = kHead + kTail;  // per-warp shared buffer
 
+// The checks run on all 32 lanes in lockstep (every value they branch on is warp-uniform): lane k holds word k
+// of the warp's head / tail buffer (hw), and a 4-byte-aligned read of either comes by shuffle from its lane,
+// so the dependent chain per word is a shuffle instead of a generic shared-memory load.
 struct Parser {
   LogicalRecord L;
-  uint64_t o;
+  uint64_t o;           // always a multiple of 4 (every XDR item is)
   const uint8_t* head;  // first `nhead` logical bytes, already in shared memory
   uint32_t nhead;
   const uint8_t* tail;  // logical bytes [tail_lo, L.len), already in shared memory (tail_lo == L.len: none)
   uint64_t tail_lo;
+  uint32_t hw;          // this lane's word of head (lanes 0-15) / tail (lanes 16-31), as stored
   __device__ __forceinline__ uint8_t byte(uint64_t at) {
     return at < nhead ? head[at] : (at >= tail_lo && at < L.len) ? tail[at - tail_lo] : L.byte(at);
   }
   __device__ int get_u32(uint32_t& v) {
     if (o + 4 > L.len) return CRK_E_TRUNCATED;
-    const uint8_t* b = o + 4 <= nhead ? head + o : o >= tail_lo ? tail + (o - tail_lo) : nullptr;
-    if (b && !(reinterpret_cast<uintptr_t>(b) & 3))  // one shared-memory word, byte-swapped (big-endian)
-      v = __byte_perm(*reinterpret_cast<const uint32_t*>(b), 0, 0x0123);
-    else if (b)
+    int src = -1;
+    if (o + 4 <= nhead) src = (int)(o >> 2);
+    else if (o >= tail_lo && !((o - tail_lo) & 3)) src = (int)(kHead / 4 + ((o - tail_lo) >> 2));
+    const uint32_t w = __shfl_sync(0xffffffffu, hw, src < 0 ? 0 : src);
+    if (src >= 0) {
+      v = __byte_perm(w, 0, 0x0123);  // big-endian
+    } else if (o >= tail_lo) {
+      const uint8_t* b = tail + (o - tail_lo);
       v = ((uint32_t)b[0] << 24) | ((uint32_t)b[1] << 16) | ((uint32_t)b[2] << 8) | b[3];
-    else
+    } else {
       v = L.be32(o);
+    }
     o += 4;
     return CRK_OK;
   }
@@ -71,16 +80,19 @@ struct Parser {
   }
 };
 
-// Parse of dense record d (ring `ring`, index slot `slot`) by one warp: lane 0 runs the checks in the
-// oracle's order and writes the parsed-call tables and the xid table; head_buf is the warp's kHeadBuf-byte
-// shared buffer for the record head.  Used by K3 (one warp per record) and by the persistent server.
+// Parse of dense record d (ring `ring`, index slot `slot`) by one warp: the lanes run the checks in the
+// oracle's order in lockstep (Parser), lane k keeps item k's fields, and the record's fields and the xid table
+// entry are written at the end; head_buf is the warp's kHeadBuf-byte shared buffer for the record head.
+// Used by K3 (one warp per record), the fused front end and the persistent server (warp-uniform calls).
 // `sole`: d is the step's only record, so its xid goes into the (cleared) table with a plain store instead
 // of a compare-and-swap whose result the warp would wait for.
 __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const ConfigDev& cfg, uint32_t d,
                              uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane, bool sole = false) {
+  STEP_MARK(lane == 0 && d == 0, 8, 0);
   Parser P;
   P.L.init(ix, ix.rings[ring], slot);
   P.o = 0;
+  STEP_MARK(lane == 0 && d == 0, 9, P.L.len ^ P.L.nfrags ^ P.L.frag0 ^ P.L.R.mask);
   // the warp prefetches, in one round trip, the record head from its first fragment and the record tail
   // from its last fragment (when the tail lies inside it): a memcpy CALL's header, pointer, opaque length
   // and, after the bulk data, its pad and size argument
@@ -94,6 +106,7 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
   const uint64_t tlo = max(max(want, (uint64_t)P.nhead), ls_last);
   P.tail_lo = P.L.len > tlo ? tlo : P.L.len;
   const uint32_t ntail = (uint32_t)(P.L.len - P.tail_lo);
+  STEP_MARK(lane == 0 && d == 0, 10, ntail ^ ph_last ^ P.L.phys[0]);
   P.head = head_buf;
   P.tail = head_buf + kHead;
   uint8_t b[4];
@@ -106,66 +119,100 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
   head_buf[kHead + lane] = b[2];
   head_buf[kHead + lane + 32] = b[3];
   __syncwarp();
-  if (lane != 0) return;
+  P.hw = reinterpret_cast<const uint32_t*>(head_buf)[lane];
+  STEP_MARK(lane == 0 && d == 0, 11, P.hw);
   const bool strict = cfg.strict != 0;
   uint32_t xid = 0, proc = 0, v, nitems = 0;
   int st = CRK_OK;
-  const Schema* sc = nullptr;
-  uint64_t* off = ix.p_off + (uint64_t)d * kMaxItems;
-  uint64_t* cnt = ix.p_count + (uint64_t)d * kMaxItems;
-  uint64_t* val = ix.p_value + (uint64_t)d * kMaxItems;
-  uint32_t* kinds = ix.p_kind + (uint64_t)d * kMaxItems;
+  uint32_t my_kind = 0;  // lane k: item k's fields
+  uint64_t my_off = 0, my_cnt = 0, my_val = 0;
+  // The fixed-layout head (RFC 5531 §9 call_body with zero-length cred and verf bodies, the AUTH_NONE case):
+  // its ten words sit in lanes 0-9, so the four header checks run on four lanes at once.  When they all
+  // pass and both auth lengths are 0 the sequential checks would reach offset 40 with these values; any
+  // other head takes the sequential path from offset 0 (same checks, same first failure).
+  const uint32_t wv = __byte_perm(P.hw, 0, 0x0123);
+  const uint32_t expect = lane == 1 ? 0u : lane == 2 ? 2u : lane == 3 ? cfg.prog : cfg.vers;
+  const bool fixed_ok = P.nhead >= 40 &&
+                        !__ballot_sync(0xffffffffu, lane >= 1 && lane <= 4 && wv != expect) &&
+                        __shfl_sync(0xffffffffu, wv, 7) == 0 && __shfl_sync(0xffffffffu, wv, 9) == 0;
   do {
-    if ((st = P.get_u32(xid))) break;
-    if ((st = P.get_u32(v))) break;
-    if (v != 0) { st = CRK_E_RPC; break; }          // msg_type CALL
-    if ((st = P.get_u32(v))) break;
-    if (v != 2) { st = CRK_E_RPC; break; }          // rpcvers 2
-    if ((st = P.get_u32(v))) break;
-    if (v != cfg.prog) { st = CRK_E_RPC; break; }
-    if ((st = P.get_u32(v))) break;
-    if (v != cfg.vers) { st = CRK_E_RPC; break; }
-    if ((st = P.get_u32(proc))) break;
-    for (uint32_t i = 0; i < sch.n; ++i)
-      if (sch.s[i].proc == proc) { sc = &sch.s[i]; break; }
-    if (!sc) { st = CRK_E_PROC; break; }
-    if ((st = P.get_auth(strict))) break;           // cred
-    if ((st = P.get_auth(strict))) break;           // verf
-    nitems = sc->n_items;
-    for (uint32_t it = 0; it < sc->n_items && st == CRK_OK; ++it) {
-      const uint32_t kind = sc->items[it] & 0xff, fixed = sc->items[it] >> 8, es = elem_size(kind);
-      kinds[it] = kind;
-      cnt[it] = 0;
-      val[it] = 0;
+    if (fixed_ok) {
+      xid = __shfl_sync(0xffffffffu, wv, 0);
+      proc = __shfl_sync(0xffffffffu, wv, 5);
+      P.o = 40;
+    } else {
+      if ((st = P.get_u32(xid))) break;
+      if ((st = P.get_u32(v))) break;
+      if (v != 0) { st = CRK_E_RPC; break; }          // msg_type CALL
+      if ((st = P.get_u32(v))) break;
+      if (v != 2) { st = CRK_E_RPC; break; }          // rpcvers 2
+      if ((st = P.get_u32(v))) break;
+      if (v != cfg.prog) { st = CRK_E_RPC; break; }
+      if ((st = P.get_u32(v))) break;
+      if (v != cfg.vers) { st = CRK_E_RPC; break; }
+      if ((st = P.get_u32(proc))) break;
+    }
+    // the first schema entry of the procedure (two entries per lane cover kMaxProcs <= 64)
+    static_assert(kMaxProcs <= 64, "two schema entries per lane");
+    const uint32_t hit_lo = __ballot_sync(0xffffffffu, lane < sch.n && sch.s[lane].proc == proc);
+    const uint32_t hit_hi = __ballot_sync(0xffffffffu, lane + 32 < sch.n && sch.s[lane + 32].proc == proc);
+    if (!hit_lo && !hit_hi) { st = CRK_E_PROC; break; }
+    const Schema& sc = sch.s[hit_lo ? __ffs(hit_lo) - 1 : 32 + __ffs(hit_hi) - 1];
+    if (!fixed_ok) {
+      if ((st = P.get_auth(strict))) break;           // cred
+      if ((st = P.get_auth(strict))) break;           // verf
+    }
+    nitems = sc.n_items;
+    const uint32_t my_item = lane < nitems ? sc.items[lane] : 0;
+    for (uint32_t it = 0; it < nitems && st == CRK_OK; ++it) {
+      const uint32_t code = __shfl_sync(0xffffffffu, my_item, it);
+      const uint32_t kind = code & 0xff, fixed = code >> 8, es = elem_size(kind);
+      uint64_t o_it = 0, c_it = 0, v_it = 0;
       if (kind == CRK_K_U32) {
-        if ((st = P.get_u32(v))) break;
-        off[it] = P.o - 4;
-        val[it] = v;
+        st = P.get_u32(v);
+        o_it = P.o - 4;
+        v_it = v;
       } else if (kind == CRK_K_U64) {
-        uint32_t hi32, lo32;                          // RFC 4506 §4.5: most significant word first
-        if ((st = P.get_u32(hi32))) break;
-        if ((st = P.get_u32(lo32))) break;
-        off[it] = P.o - 8;
-        val[it] = ((uint64_t)hi32 << 32) | lo32;
+        uint32_t hi32 = 0, lo32 = 0;                  // RFC 4506 §4.5: most significant word first
+        if (!(st = P.get_u32(hi32))) st = P.get_u32(lo32);
+        o_it = P.o - 8;
+        v_it = ((uint64_t)hi32 << 32) | lo32;
       } else {
-        uint64_t c;
+        uint64_t c = fixed;
         if (kind_is_var(kind)) {
-          if ((st = P.get_u32(v))) break;
+          st = P.get_u32(v);
           c = v;
-        } else {
-          c = fixed;
         }
-        const uint64_t bytes = c * es, pn = pad4(bytes);
-        if (P.o + bytes + pn > P.L.len) { st = CRK_E_TRUNCATED; break; }
-        if (strict && !P.pad_is_zero(P.o + bytes, pn)) { st = CRK_E_PAD; break; }
-        off[it] = P.o;
-        cnt[it] = c;
-        P.o += bytes + pn;
+        if (st == CRK_OK) {
+          const uint64_t bytes = c * es, pn = pad4(bytes);
+          if (P.o + bytes + pn > P.L.len) st = CRK_E_TRUNCATED;
+          else if (strict && !P.pad_is_zero(P.o + bytes, pn)) st = CRK_E_PAD;
+          else {
+            o_it = P.o;
+            c_it = c;
+            P.o += bytes + pn;
+          }
+        }
+      }
+      if (lane == it) {
+        my_kind = kind;
+        my_off = o_it;
+        my_cnt = c_it;
+        my_val = v_it;
       }
     }
     if (st != CRK_OK) break;
     if (strict && P.o != P.L.len) st = CRK_E_TRAILING;
   } while (0);
+  STEP_MARK(lane == 0 && d == 0, 12, st ^ nitems);
+  if (lane < nitems) {  // the items parsed before any failure; the tables are read only for OK / E_TRAILING
+    const uint64_t k = (uint64_t)d * kMaxItems + lane;
+    ix.p_kind[k] = my_kind;
+    ix.p_off[k] = my_off;
+    ix.p_count[k] = my_cnt;
+    ix.p_value[k] = my_val;
+  }
+  if (lane != 0) return;
   ix.p_slot[d] = slot;
   ix.p_frag0[d] = P.L.frag0;
   ix.p_nfrags[d] = P.L.nfrags;

@@ -128,7 +128,9 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
     phase_sync();
     TL_END(P.cfg, 0);
+    crk_ring_result my_res;  // thread r < n_rings: ring r's result, published after the move
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
+    STEP_MARK(threadIdx.x == 0, 0, 0);
     // ---- K1: each ring in turn by the whole CTA
     SCAN_TRACE(threadIdx.x == 0, 5, 0);
     if (threadIdx.x == 0) prefix[0] = 0;
@@ -187,7 +189,6 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     // plan's tile total (cfg tiles) and the step's final ring results, loaded with the jobs in the same
     // round trip (the results are published after the move)
     const uint64_t plan_tiles = P.sc.scan_tmp[P.sc.max_jobs + 1];
-    crk_ring_result my_res;
     if (threadIdx.x < P.n_rings) my_res = ix.res[threadIdx.x];
     {  // the first kJobCache jobs in one round trip (every warp walks every job's descriptor)
       const uint32_t nc = n_jobs < kJobCache ? n_jobs : kJobCache;
@@ -196,6 +197,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
       __syncthreads();
     }
     const uint32_t sh = plan_tiles <= 4 ? 11u : 13u;
+    STEP_MARK(threadIdx.x == 0, 16, sh ^ jobs_s[0].type);
     uint64_t first = 0;  // global number of the job's first tile
     for (uint32_t j = 0; j < n_jobs; ++j) {
       const Job J = j < kJobCache ? jobs_s[j] : P.sc.jobs[j];
@@ -204,17 +206,22 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
         move_tile(TW, P, J, t, sh);
       first += nt;
     }
+    STEP_MARK(lane == 0 && warp < 4, 27 + warp, 0);  // each of the first warps' last tile done
+    STEP_MARK(threadIdx.x == 0, 17, 0);
     phase_sync();
+    STEP_MARK(threadIdx.x == 0, 18, 0);
     TL_END(P.cfg, 4);
     if (threadIdx.x == 0) B->t_phase_ns[4] = gtimer();
     // ---- publish: results into the bell, then done_seq
     if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
     __syncthreads();
+    STEP_MARK(threadIdx.x == 0, 19, 0);
     if (threadIdx.x == 0) {
       B->status = bad_s ? CRK_E_ARG : CRK_OK;
       B->t_end_ns = gtimer();
       __threadfence_system();
       st_release_sys(&B->done_seq, seen);
+      STEP_MARK(true, 20, 0);
     }
     TL_END(P.cfg, 5);
   }
@@ -234,6 +241,12 @@ extern "C" int crk_debug_server_scan_trace(unsigned long long* out, uint32_t* co
     if (cudaMemcpyToSymbol(g_scan_trace_n, zero, sizeof(zero)) != cudaSuccess) return -100;
   }
   return 0;
+}
+#endif
+
+#ifdef CRK_STEP_TRACE
+extern "C" int crk_debug_server_step_trace(unsigned long long* out32) {
+  return cudaMemcpyFromSymbol(out32, g_step_trace, sizeof(g_step_trace)) == cudaSuccess ? 0 : -100;
 }
 #endif
 
