@@ -120,6 +120,10 @@ typedef struct {
                                 default 3, 0 = no such procedure) */
   uint32_t mover_max_ctas;    /* cap on the mover's grid (0 = every CTA slot the occupancy allows); a small grid
                                 leaves HBM to concurrent copy-engine traffic in a host-ring server loop */
+  uint32_t fused_front_max_frags; /* a small index (fused_front_max_records) whose rings hold at most this many
+                                     fragments in all also takes the fused single-CTA front end for windows past
+                                     fused_front_max_window: the index bounds the CTA's header walk (default
+                                     4096, e.g. one 256 MiB memcpy CALL in 64 KiB fragments; 0 = off) */
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;

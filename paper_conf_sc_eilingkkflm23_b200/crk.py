@@ -46,7 +46,8 @@ class Config(C.Structure):
                 ("ctas_per_sm", C.c_uint32), ("scan_threads", C.c_uint32), ("mover_stages", C.c_uint32),
                 ("mover_run", C.c_uint32), ("mover_tail_tiles", C.c_uint32), ("mover_reserve_ctas", C.c_uint32),
                 ("fused_front_max_records", C.c_uint32), ("scan_chunking", C.c_uint32), ("fused_front_max_window", C.c_uint64),
-                ("proc_h2d_stripe", C.c_uint32), ("mover_max_ctas", C.c_uint32)]
+                ("proc_h2d_stripe", C.c_uint32), ("mover_max_ctas", C.c_uint32),
+                ("fused_front_max_frags", C.c_uint32)]
 
 
 class CRing(C.Structure):

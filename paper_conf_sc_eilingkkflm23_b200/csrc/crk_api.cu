@@ -139,14 +139,18 @@ int scan_param(crk_index* idx, uint32_t n_rings, const crk_ring* rings, const ui
 
 // A small index (crk_config.fused_front_max_records) over one ring or a small window: one fused launch.
 // A window long enough for the chunked multi-CTA scan (k_mscan.cu) goes to the separate kernels even on one
-// ring: the single CTA of the fused front end would walk its whole header chain alone.
+// ring: the single CTA of the fused front end would walk its whole header chain alone -- unless the index
+// holds at most fused_front_max_frags fragments, which bounds that walk (the scan stops at the index's
+// capacity): then one launch beats the chunked scan's fixed cost (e.g. one 64 MiB memcpy CALL, 1,025 headers).
 bool fused_front(const crk_ctx* c, const crk_index* x, uint32_t n_rings, const uint64_t* heads, const uint64_t* tails,
                  const uint64_t* doorbell) {
   uint64_t window = 0;
   for (uint32_t r = 0; !doorbell && heads && tails && r < n_rings; ++r) window += tails[r] - heads[r];
-  const bool chunkable = !doorbell && c->cfg.scan_chunking == 0 && window > c->cfg.fused_front_max_window;
+  const bool capped = (uint64_t)x->ix.frags_per_ring * n_rings <= c->cfg.fused_front_max_frags;
+  const bool long_window = window > c->cfg.fused_front_max_window && !capped;
+  const bool chunkable = !doorbell && c->cfg.scan_chunking == 0 && long_window;
   return x->ix.max_records <= c->cfg.fused_front_max_records && x->ix.max_records <= front_small_threads() &&
-         !chunkable && (n_rings == 1 || (!doorbell && window <= c->cfg.fused_front_max_window));
+         !chunkable && (n_rings == 1 || (!doorbell && !long_window));
 }
 
 int run_scan(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_ring* rings, const uint64_t* heads,
@@ -267,6 +271,7 @@ void crk_config_init(crk_config* c) {
   c->mover_reserve_ctas = 0;
   c->fused_front_max_records = 128;
   c->fused_front_max_window = 1ull << 20;
+  c->fused_front_max_frags = 4096;
   c->proc_h2d_stripe = 3;
 }
 

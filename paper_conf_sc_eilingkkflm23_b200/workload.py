@@ -357,7 +357,7 @@ class LinkSweep:
             sl.dev_big = crk.Ring.device(self.big, device)
             sl.dev_small = crk.Ring.device(4096, device)
             sl.region = torch.zeros(max_n + 256, dtype=torch.uint8, device=device)
-            sl.idx = ctx.index(1, (max_n >> 15) + 64, 16)
+            sl.idx = None  # sized per call by prepare / prepare_c2
             sl.stream, sl.in_s, sl.out_s = (torch.cuda.Stream(device) for _ in range(3))
             sl.ev_in, sl.ev_served, sl.ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
             self.slots.append(sl)
@@ -372,6 +372,9 @@ class LinkSweep:
         self.n, self.direction = n, direction
         for i, sl in enumerate(self.slots):
             base = sl.region.data_ptr()
+            # an index sized for the call, as a server sizes its buffers for its calls: a small one (up to
+            # crk_config.fused_front_max_frags fragments) lets crk_serve take the fused single-CTA front end
+            sl.idx = sl.ctx.index(1, n // F + 64, 16)
             if direction == "h2d":
                 stage = self._sub(sl.dev_big, self.big)
                 w = sl.ctx.encode_call(0x5E0000 + i, gen.PROC_H2D, [(crk.K_U64, base), (crk.K_OPAQUE_VAR, payload),
@@ -400,6 +403,7 @@ class LinkSweep:
         half = self.big // 2
         for i, sl in enumerate(self.slots):
             base = sl.region.data_ptr()
+            sl.idx = sl.ctx.index(1, (1 << 21) // F + 64, 16)
             offA, offB, offC = 0, 409_600, 409_600 + 819_200
             sl.region[offC:offC + Cm.numel()].copy_(Cm)
             rx_dev, tx_dev = sl.dev_big.sub(0, 1 << 21), sl.dev_big.sub(half, 1 << 20)

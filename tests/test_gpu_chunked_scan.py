@@ -241,3 +241,26 @@ def test_serve_through_chunked_scan_matches_oracle():
         n = want["reply_bytes"][r]
         assert T["rings"][r]["reply_bytes"] == n and T["rings"][r]["consumed"] == want["consumed"][r]
         assert sends[r].read(offs[r], n) == bytes(want["send"][r][offs[r]:offs[r] + n])
+
+
+@pytest.mark.parametrize("case", ["one_call_24MiB", "irregular_capped", "capacity_stop"])
+def test_capped_small_index_takes_the_fused_front_end(case):
+    """A small index (<= fused_front_max_records records, <= fused_front_max_frags fragments in all) scans a
+    window past fused_front_max_window in the fused single-CTA front end -- its capacity bounds the header
+    walk -- and still equals or_frame_scan / or_parse_call; the same window over a larger index is chunked."""
+    cfg = ocfg()
+    if case == "one_call_24MiB":  # one C3-shaped memcpy CALL: 385 headers
+        d = gen.random_bytes(77, 24 * MiB)
+        wires, fpr, rpr = [O.encode_call(*h2d_call(0xC3, d), cfg)], 400, 4
+    elif case == "irregular_capped":  # C4-ii framing, fragments uniform in [1, 64 KiB]: every hop a new length
+        wires, fpr, rpr = irregular(31, 40 * MiB, cfg), 2048, 128
+    else:  # more records than the index holds: the one CTA stops at the record capacity
+        wires, fpr, rpr = c5_like(32, 8 * MiB, cfg, hi=256 * 1024), 2048, 16
+    s, st, w = run_scan(wires, head=12345, cap=1 << 26, fpr=fpr, rpr=rpr)
+    assert w > (1 << 20) and st == {"chunked": 0, "fallback": 0}, st  # past the window limit, yet fused
+    if case == "one_call_24MiB":
+        assert s.status == O.OK and len(s.recs) == 1
+    if case == "capacity_stop":
+        assert s.status == O.INCOMPLETE and len(s.recs) == rpr
+    s2, st2, _ = run_scan(wires, head=12345, cap=1 << 26, fpr=fpr, rpr=rpr, fused_front_max_frags=0)
+    assert st2["chunked"] + st2["fallback"] == 1 and s2.status == s.status and len(s2.recs) == len(s.recs)
