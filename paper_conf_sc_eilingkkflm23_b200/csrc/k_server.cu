@@ -219,7 +219,8 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) {
       B->status = bad_s ? CRK_E_ARG : CRK_OK;
       B->t_end_ns = gtimer();
-      __threadfence_system();
+      // a system-scope release: the step's writes (every thread's, ordered before it by the barrier; the
+      // PTX memory model's causality order is cumulative) are visible to whoever acquires done_seq
       st_release_sys(&B->done_seq, seen);
       STEP_MARK(true, 20, 0);
     }
