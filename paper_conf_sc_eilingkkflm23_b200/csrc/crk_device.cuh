@@ -82,6 +82,21 @@ __device__ __forceinline__ uint4 swap16(uint4 v, uint32_t esize) {
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
+// CTA barriers that tolerate a warp arriving diverged (barrier.sync without .aligned; __syncthreads is the
+// .aligned form, undefined when a warp's lanes reach it separately).  The single-CTA step code (scan, parse,
+// planning, the CTA movers) crosses phase boundaries right after lane-dependent loops (xid probes, per-lane
+// fragment walks, work done by warp 0 alone), where the warp need not have reconverged.
+__device__ __forceinline__ void cta_barrier() { asm volatile("barrier.sync 0;" ::: "memory"); }
+__device__ __forceinline__ bool cta_barrier_or(bool p) {
+  uint32_t r;
+  asm volatile(
+      "{\n .reg .pred q, o;\n setp.ne.u32 q, %1, 0;\n barrier.red.or.pred o, 0, q;\n selp.u32 %0, 1, 0, o;\n}\n"
+      : "=r"(r)
+      : "r"((uint32_t)p)
+      : "memory");
+  return r != 0;
+}
+
 // Programmatic dependent launch (launch_k in crk_internal.h): the first statement of every kernel of the
 // library.  griddepcontrol.wait returns once the previous kernel of the stream has completed and its memory
 // is visible (a no-op without the launch attribute); launch_dependents then lets the stream's next kernel be

@@ -54,7 +54,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
-  __syncthreads();
+  cta_barrier();
   FRONT_MARK(1);
   // ---- K1: each ring in turn by the whole CTA, then dense record numbering (prefix[] in shared memory)
   if (threadIdx.x == 0) prefix[0] = 0;
@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
     if (threadIdx.x == 0) prefix[r + 1] = prefix[r] + S.nr;
   }
   if (threadIdx.x == 0) dense_numbering_cta(ix, n_rings, prefix);
-  __syncthreads();
+  cta_barrier();
   FRONT_MARK(2);
   // ---- K3: one warp per record
   const uint32_t total = prefix[n_rings];
@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
     TL_END(P.cfg, TL_FUSED);
     return;
   }
-  __syncthreads();
+  cta_barrier();
   FRONT_MARK(3);
   // ---- serve planning: statuses, reply offsets, jobs, their tile prefix, mover cursors
   plan_small_block(ix, P.cfg, P.sc, P.send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix);

@@ -255,11 +255,11 @@ __device__ __forceinline__ void block_excl_sums(uint64_t (&v)[NV], uint64_t* war
       if (lane >= (uint32_t)o) x[k] += y;
     }
   }
-  __syncthreads();
+  cta_barrier();
   if (lane == 31)
 #pragma unroll
     for (int k = 0; k < NV; ++k) warp_sums[32 * k + w] = x[k];
-  __syncthreads();
+  cta_barrier();
   if (w == 0) {  // inclusive prefix of the warp totals, in place
 #pragma unroll
     for (int k = 0; k < NV; ++k) {
@@ -272,7 +272,7 @@ __device__ __forceinline__ void block_excl_sums(uint64_t (&v)[NV], uint64_t* war
       if (lane < nw) warp_sums[32 * k + lane] = y;
     }
   }
-  __syncthreads();
+  cta_barrier();
 #pragma unroll
   for (int k = 0; k < NV; ++k) {
     tot[k] = warp_sums[32 * k + nw - 1];
@@ -348,7 +348,7 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
   const bool my_stripe = cfg.proc_stripe && d < total && st == CRK_OK && Ll == 28 && err < 0;  // only OK stripes
   if (kOneWarp) __syncwarp();  // orders the warp's parent-table atomics before the leads read the table
   const bool any_stripe =
-      cfg.proc_stripe && (kOneWarp ? __any_sync(0xffffffffu, my_stripe) : __syncthreads_or(my_stripe));
+      cfg.proc_stripe && (kOneWarp ? __any_sync(0xffffffffu, my_stripe) : cta_barrier_or(my_stripe));
   if (my_stripe && stripe_leads(ix, (uint32_t)ix.p_value[(uint64_t)d * kMaxItems + 3], d)) err = 0;
   if (d < total) w = err >= 0 ? wire_of(Ll, cfg.F) : 0;
   PLAN_MARK(2);
@@ -363,7 +363,7 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
   }
   (void)tot;
   if (d < total && d == first) ring_first_pre[ring] = pre;
-  if (kOneWarp) __syncwarp(); else __syncthreads();
+  if (kOneWarp) __syncwarp(); else cta_barrier();
   PLAN_MARK(3);
   Job enc{};
   if (d < total) {
@@ -396,7 +396,7 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
   if (any_stripe) {  // leave the parent table empty for the next step (every lead has read it)
     const uint32_t n = __ldcg(ix.stripe_n);
     stripe_clear(ix, n, threadIdx.x, nthreads);
-    if (kOneWarp) __syncwarp(); else __syncthreads();
+    if (kOneWarp) __syncwarp(); else cta_barrier();
     if (d == 0 && n) *ix.stripe_n = 0;
   }
   if (d == 0) {

@@ -434,11 +434,11 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     S.consumed = R.head;
     S.kept_frags = 0;
   }
-  __syncthreads();
+  cta_barrier();
   const Env E{ix, R, cfg.max_record_bytes, fbase, rbase, FC, RC};
   for (;;) {
     const bool done = S.done, wide_mode = S.wide;
-    __syncthreads();  // everyone has read the mode before warp 0 / the round changes S
+    cta_barrier();  // everyone has read the mode before warp 0 / the round changes S
     if (done) break;
     if (!wide_mode) {
       // warp rounds / chase passes in warp 0 until a stop or a long regular run; the others wait
@@ -466,7 +466,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
           }
         }
       }
-      __syncthreads();
+      cta_barrier();
       continue;
     }
     const uint64_t p = S.p, r0 = S.r0, sum = S.sum;
@@ -506,7 +506,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     const uint32_t own = __ffs(__ballot_sync(0xffffffffu, first_bad == wm)) - 1;
     const uint32_t oh = __shfl_sync(0xffffffffu, bh, own), ov = __shfl_sync(0xffffffffu, bv, own);
     if (lane == 0) { S.gmin[warp] = wm; S.gh[warp] = oh; S.gv[warp] = ov; }
-    __syncthreads();
+    cta_barrier();
     uint32_t ts0 = TT, ts1 = TT, ws0 = 0, ws1 = 0;
     for (uint32_t w = 0; w < nw; ++w) {
       const uint32_t g = S.gmin[w];
@@ -575,7 +575,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
       const uint32_t fown = __ffs(__ballot_sync(0xffffffffu, first_fail == fm)) - 1;
       const uint32_t fc = __shfl_sync(0xffffffffu, my_code, fown);
       if (lane == 0) { S.fmin[warp] = fm; S.fcode[warp] = fc; }
-      __syncthreads();
+      cta_barrier();
       for (uint32_t w = 0; w < nw; ++w)
         if (S.fmin[w] < tf) { tf = S.fmin[w]; code_f = S.fcode[w]; }
     }
@@ -648,7 +648,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
         }
       }
     }
-    __syncthreads();
+    cta_barrier();
   }
   SCAN_TRACE(threadIdx.x == 0, 0, 0);  // end marker
   if (threadIdx.x == 0) {
@@ -659,7 +659,7 @@ __device__ void scan_ring_cta(const IndexDev& ix, const RingDesc& R, bool bad_wi
     rr.consumed = S.consumed;
     rr.reply_bytes = 0;
   }
-  __syncthreads();
+  cta_barrier();
 }
 
 // Dense record numbering = exclusive prefix of the rings' record counts (one thread).

@@ -50,10 +50,10 @@ __device__ __forceinline__ uint64_t gtimer() {
 }
 // Phase boundary: the block's global writes and atomics of the previous phase are visible to the block.
 __device__ __forceinline__ void phase_sync() {
-  __syncthreads();
+  cta_barrier();
 #ifdef CRK_SERVER_PHASE_FENCE  // diagnostic: a device-wide fence per phase as well
   if (threadIdx.x == 0) __threadfence();
-  __syncthreads();
+  cta_barrier();
 #endif
 }
 
@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
       const uint32_t nc = n_jobs < kJobCache ? n_jobs : kJobCache;
       for (uint32_t i = threadIdx.x; i < nc * (uint32_t)(sizeof(Job) / 4); i += blockDim.x)
         reinterpret_cast<uint32_t*>(jobs_s)[i] = reinterpret_cast<const uint32_t*>(P.sc.jobs)[i];
-      __syncthreads();
+      cta_barrier();
     }
     const uint32_t sh = plan_tiles <= 4 ? 11u : 13u;
     STEP_MARK(threadIdx.x == 0, 16, sh ^ jobs_s[0].type);
@@ -214,7 +214,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) B->t_phase_ns[4] = gtimer();
     // ---- publish: results into the bell, then done_seq
     if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
-    __syncthreads();
+    cta_barrier();
     STEP_MARK(threadIdx.x == 0, 19, 0);
     if (threadIdx.x == 0) {
       B->status = bad_s ? CRK_E_ARG : CRK_OK;
