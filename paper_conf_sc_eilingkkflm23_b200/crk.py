@@ -517,9 +517,12 @@ class Index:
         _check(lib().crk_index_ring_results_async(self.h, out.n, out.buf.ptr, _stream(stream)),
                "crk_index_ring_results_async")
 
-    def tables(self, n_rings: int | None = None) -> dict:
-        """Host copies of the index tables after synchronising the device (tests / inspection)."""
-        torch.cuda.synchronize()
+    def tables(self, n_rings: int | None = None, sync: bool = True) -> dict:
+        """Host copies of the index tables after synchronising the device (tests / inspection).  sync=False
+        skips the device-wide synchronisation (a persistent server owning the index is still running; its
+        tables are complete once its doorbell shows the step done)."""
+        if sync:
+            torch.cuda.synchronize()
         n_rings = self.n_rings if n_rings is None else n_rings
         v = self.v
         res = self.ring_results(n_rings)

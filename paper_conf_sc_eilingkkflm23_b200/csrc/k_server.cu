@@ -187,7 +187,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     const uint32_t n_jobs = 2 * total;
     const Team TW{lane, 32, 0, 1};
     // plan's tile total (cfg tiles) and the step's final ring results, loaded with the jobs in the same
-    // round trip (the results are published after the move)
+    // round trip
     const uint64_t plan_tiles = P.sc.scan_tmp[P.sc.max_jobs + 1];
     if (threadIdx.x < P.n_rings) my_res = ix.res[threadIdx.x];
     {  // the first kJobCache jobs in one round trip (every warp walks every job's descriptor)
@@ -196,6 +196,10 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
         reinterpret_cast<uint32_t*>(jobs_s)[i] = reinterpret_cast<const uint32_t*>(P.sc.jobs)[i];
       cta_barrier();
     }
+    // the results go to the bell now (host-memory writes in flight during the move; the release after the
+    // move orders them before done_seq)
+    if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
+    if (threadIdx.x == 0) B->status = bad_s ? CRK_E_ARG : CRK_OK;
     const uint32_t sh = plan_tiles <= 4 ? 11u : 13u;
     STEP_MARK(threadIdx.x == 0, 16, sh ^ jobs_s[0].type);
     uint64_t first = 0;  // global number of the job's first tile
@@ -212,12 +216,10 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     STEP_MARK(threadIdx.x == 0, 18, 0);
     TL_END(P.cfg, 4);
     if (threadIdx.x == 0) B->t_phase_ns[4] = gtimer();
-    // ---- publish: results into the bell, then done_seq
-    if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
+    // ---- publish: done_seq (the results were written before the move)
     cta_barrier();
     STEP_MARK(threadIdx.x == 0, 19, 0);
     if (threadIdx.x == 0) {
-      B->status = bad_s ? CRK_E_ARG : CRK_OK;
       B->t_end_ns = gtimer();
       // a system-scope release: the step's writes (every thread's, ordered before it by the barrier; the
       // PTX memory model's causality order is cumulative) are visible to whoever acquires done_seq
