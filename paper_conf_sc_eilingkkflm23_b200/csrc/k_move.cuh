@@ -72,9 +72,9 @@ struct DecCtx {
 };
 // From the decode job's own record coordinates (dec_job: first fragment, count, ring, first fragment's length):
 // one round trip for the ring descriptor instead of the job -> record -> fragment table chain.
-__device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, const Job& j) {
+__device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, const Job& j, const RingDesc& R) {
   LogicalRecord& L = c.L;
-  L.R = ix.rings[j.out_ring];
+  L.R = R;
   L.frag0 = j.piece0;
   L.nfrags = j.n_pieces;
   L.len = ~0ull;  // not needed by the decode paths (they stay inside the job's range)
@@ -86,6 +86,9 @@ __device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, cons
   c.dst = j.out_start;
   c.loff = j.loff;
   c.es = j.esize;
+}
+__device__ __forceinline__ void dec_ctx_init(DecCtx& c, const IndexDev& ix, const Job& j) {
+  dec_ctx_init(c, ix, j, ix.rings[j.out_ring]);
 }
 // exact source of destination byte x (element e, byte j) = logical byte loff + e*es + (es-1-j)
 __device__ __forceinline__ uint8_t dec_exact_byte(DecCtx& c, uint64_t x) {

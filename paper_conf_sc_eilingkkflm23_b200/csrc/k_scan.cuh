@@ -27,6 +27,7 @@ constexpr uint32_t kWJ = 2;                // candidate headers per lane and war
 constexpr uint32_t kWTT = 16 * kWJ;        // candidates per group and warp round (16 lanes per group)
 constexpr uint32_t kChase = 4096;          // max headers per chase pass (irregular framing)
 constexpr uint32_t kFull = 0xffffffffu;
+constexpr uint64_t kChaseFirst = 16384;     // windows up to this many bytes start with a chase pass
 
 #ifdef CRK_SCAN_TRACE
 // Diagnostic build only (build.py build_trace -> lib/libcrk_trace.so): per ring, one entry per round /
@@ -283,7 +284,9 @@ __device__ void chase(const Env& E, Walk& W, uint32_t lane) {
 // two rounds that accepted at most 2 headers each, a chase pass takes over.
 __device__ bool warp_rounds(const Env& E, Walk& W, uint32_t lane) {
   const uint32_t grp = lane >> 4, u = lane & 15;
-  uint32_t miss = 0;
+  // a short window (a few small calls) starts with a chase pass: one load per header and no speculation round
+  // (whose candidates past a one-record window are all misses); the rounds take over at a regular run
+  uint32_t miss = E.R.tail - W.p <= kChaseFirst ? 2u : 0u;
   for (;;) {
     if (miss >= 2) {
       chase(E, W, lane);

@@ -71,11 +71,11 @@ __device__ __forceinline__ void move_tile(const Team& T, const ServerParams& P, 
   const uint64_t a = max(J.out_start, (A + t) << sh), b = min(J.out_end, (A + t + 1) << sh);
   if (J.type == JOB_DEC) {
     DecCtx c;
-    dec_ctx_init(c, P.ix, J);
+    dec_ctx_init(c, P.ix, J, P.rings[J.out_ring]);  // (base and mask: the decode reads no cursor from it)
     dec_tile_generic(T, c, a, b, 0);
   } else if (J.type == JOB_ENC) {
     EncCtx c;
-    enc_ctx_init(c, P.sc, J, P.sc.out_rings[J.out_ring], P.sc.pieces + J.piece0);
+    enc_ctx_init(c, P.sc, J, P.send[J.out_ring], P.sc.pieces + J.piece0);
     enc_tile_generic(T, c, a - J.out_start, b - J.out_start);
   }
 }
