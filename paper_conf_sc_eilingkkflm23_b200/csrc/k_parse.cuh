@@ -87,7 +87,8 @@ struct Parser {
 // `sole`: d is the step's only record, so its xid goes into the (cleared) table with a plain store instead
 // of a compare-and-swap whose result the warp would wait for.
 __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const ConfigDev& cfg, uint32_t d,
-                             uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane, bool sole = false) {
+                             uint32_t ring, uint32_t slot, uint8_t* head_buf, uint32_t lane, bool sole = false,
+                             uint64_t prefetch_max = 0) {
   STEP_MARK(lane == 0 && d == 0, 8, 0);
   Parser P;
   P.L.init(ix, ix.rings[ring], slot);
@@ -107,6 +108,19 @@ __device__ void parse_record(const IndexDev& ix, const SchemaTable& sch, const C
   P.tail_lo = P.L.len > tlo ? tlo : P.L.len;
   const uint32_t ntail = (uint32_t)(P.L.len - P.tail_lo);
   STEP_MARK(lane == 0 && d == 0, 10, ntail ^ ph_last ^ P.L.phys[0]);
+  // prefetch_max (the persistent server, device-memory rings): a record of at most that many bytes has its first
+  // fragment pulled into L2 now (a hint: no registers, nothing waits), so the move that follows the planning
+  // reads the payload from L2 instead of HBM
+  if (prefetch_max && lane == 0 && P.L.len <= prefetch_max) {
+    uint64_t c = P.L.phys[0] & ~15ull;
+    const uint64_t e = (P.L.phys[0] + n0 + 15) & ~15ull;
+    while (c < e) {
+      const uint64_t o = c & P.L.R.mask, room = P.L.R.mask + 1 - o, left = e - c;
+      const uint32_t n = (uint32_t)(room < left ? room : left);
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(P.L.R.base + o), "r"(n) : "memory");
+      c += n;
+    }
+  }
   P.head = head_buf;
   P.tail = head_buf + kHead;
   uint8_t b[4];

@@ -324,10 +324,21 @@ __device__ unsigned long long g_plan_trace[16];
 // dense record prefix they already hold in shared memory (prefix_s, n_rings + 1 entries), which saves the
 // dependent loads of the record total and of each record's ring bounds.  kOneWarp: a step of at most 32
 // records is planned by warp 0 alone, its sums by shuffles, with no block barrier.
+// Optional shared-memory copies of the plan for a caller that moves the step itself (the persistent server):
+// the jobs (when 2 * total <= cap), the tile total and each ring's reply bytes, so its move phase needs no
+// load of what the plan just wrote.  reply_bytes must hold 0 for every ring beforehand.
+struct PlanOut {
+  Job* jobs;
+  uint32_t cap;
+  uint64_t* tiles;
+  uint64_t* reply_bytes;
+};
+
 template <bool kOneWarp>
 __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
                                 uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
-                                uint64_t* ring_first_pre, const uint32_t* prefix_s, uint32_t total) {
+                                uint64_t* ring_first_pre, const uint32_t* prefix_s, uint32_t total,
+                                const PlanOut* out) {
   PLAN_MARK(0);
   const uint32_t d = threadIdx.x, nthreads = kOneWarp ? 32u : blockDim.x;
   for (uint32_t r = threadIdx.x; r < S.n_rings; r += nthreads) sc.out_rings[r] = S.r[r];
@@ -376,6 +387,13 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
     sc.jobs[d] = dec;
     sc.jobs[total + d] = enc;
     if (d + 1 == end) ix.res[ring].reply_bytes = pre + w - ring_first_pre[ring];
+    if (out) {
+      if (2 * total <= out->cap) {
+        out->jobs[d] = dec;
+        out->jobs[total + d] = enc;
+      }
+      if (d + 1 == end) out->reply_bytes[ring] = pre + w - ring_first_pre[ring];
+    }
   }
   // mover plan: tiles per job (decode jobs [0, total), encode jobs [total, 2 total)) and their prefix
   auto tiles_of = [&](const Job& j) -> uint64_t {
@@ -400,6 +418,7 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
     if (d == 0 && n) *ix.stripe_n = 0;
   }
   if (d == 0) {
+    if (out) *out->tiles = tot_d + tot_e;
     sc.scan_tmp[sc.max_jobs + 1] = tot_d + tot_e;
     sc.counters[0] = 0;
     sc.counters[2] = 0;
@@ -413,13 +432,16 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
 
 __device__ void plan_small_block(const IndexDev& ix, const ConfigDev& cfg, const Scratch& sc, const SendRingsParam& S,
                                  uint64_t region_base, uint64_t region_bytes, uint64_t* warp_sums,
-                                 uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr) {
+                                 uint64_t* ring_first_pre, const uint32_t* prefix_s = nullptr,
+                                 const PlanOut* out = nullptr) {
   const uint32_t total = prefix_s ? prefix_s[S.n_rings] : *ix.total;
   if (total <= 32) {
     if (threadIdx.x < 32)
-      plan_small_impl<true>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total);
+      plan_small_impl<true>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total,
+                            out);
   } else {
-    plan_small_impl<false>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total);
+    plan_small_impl<false>(ix, cfg, sc, S, region_base, region_bytes, warp_sums, ring_first_pre, prefix_s, total,
+                           out);
   }
 }
 

@@ -33,6 +33,7 @@ struct ServerParams {
   RingDesc rings[kMaxRings];   // base / mask; cursors come from the bell
   RingDesc send[kMaxRings];
   uint64_t region_base, region_bytes;
+  uint64_t dev_rings;          // bit r: receive ring r is device memory (its small records are prefetched to L2)
 };
 
 __device__ __forceinline__ uint64_t ld_acquire_sys(const volatile uint64_t* p) {
@@ -61,6 +62,7 @@ __device__ __forceinline__ void phase_sync() {
 // (generic paths of k_move.cuh).
 // tiles dealt to the warps round-robin: 2 KiB (one chunk-loop pass per warp) when the step moves at most
 // ~4 mover tiles' worth of bytes, else 8 KiB
+constexpr uint64_t kPrefetchMax = 64 * 1024;  // records up to this size have their payload prefetched to L2
 constexpr uint32_t kJobCache = 32;   // jobs staged in shared memory at the start of the move phase
 __device__ __forceinline__ uint64_t job_tiles(const Job& J, uint32_t sh) {
   if (J.type == JOB_NONE || J.out_end <= J.out_start) return 0;
@@ -91,6 +93,8 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
   __shared__ uint64_t win_head[kMaxRings], win_tail[kMaxRings];
   __shared__ uint64_t seq_s;
   __shared__ Job jobs_s[kJobCache];
+  __shared__ uint64_t tiles_s, reply_s[kMaxRings];
+  __shared__ crk_ring_result res_s[kMaxRings];
   __shared__ uint32_t stop_s, bad_s;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   crk_server_bell* B = P.bell;
@@ -128,7 +132,6 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
     phase_sync();
     TL_END(P.cfg, 0);
-    crk_ring_result my_res;  // thread r < n_rings: ring r's result, published after the move
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     STEP_MARK(threadIdx.x == 0, 0, 0);
     // ---- K1: each ring in turn by the whole CTA
@@ -164,6 +167,13 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     phase_sync();
     TL_END(P.cfg, 7);
 #endif
+    // the rings' scan results (final but for reply_bytes, which the plan hands over in shared memory): copied to
+    // shared memory now by the last warp (the first parses record 0), overlapping the parse
+    if (warp == kServerWarps - 1)
+      for (uint32_t r = lane; r < P.n_rings; r += 32) {
+        res_s[r] = ix.res[r];
+        reply_s[r] = 0;
+      }
     // ---- K3: one warp per record (prefix[] is the scan's dense numbering, in shared memory)
     const uint32_t total = prefix[P.n_rings];
     for (uint32_t d = warp; d < total; d += kServerWarps) {
@@ -172,33 +182,36 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
         const uint32_t mid = (lo + hi) >> 1;
         if (prefix[mid] <= d) lo = mid; else hi = mid;
       }
-      parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane, total == 1);
+      parse_record(ix, sch, P.cfg, d, lo, lo * ix.recs_per_ring + (d - prefix[lo]), heads[warp], lane, total == 1,
+                   (P.dev_rings >> lo) & 1 ? kPrefetchMax : 0);
       __syncwarp();
     }
     phase_sync();
     TL_END(P.cfg, 2);
     if (threadIdx.x == 0) B->t_phase_ns[2] = gtimer();
     // ---- serve planning (statuses, reply offsets, jobs)
-    plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix);
+    const PlanOut out{jobs_s, kJobCache, &tiles_s, reply_s};
+    plan_small_block(ix, P.cfg, P.sc, send, P.region_base, P.region_bytes, warp_sums, ring_first_pre, prefix, &out);
     phase_sync();
     TL_END(P.cfg, 3);
     if (threadIdx.x == 0) B->t_phase_ns[3] = gtimer();
     // ---- movers: every job cut into 8 KiB output tiles, tiles dealt to the warps round-robin
     const uint32_t n_jobs = 2 * total;
     const Team TW{lane, 32, 0, 1};
-    // plan's tile total (cfg tiles) and the step's final ring results, loaded with the jobs in the same
-    // round trip
-    const uint64_t plan_tiles = P.sc.scan_tmp[P.sc.max_jobs + 1];
-    if (threadIdx.x < P.n_rings) my_res = ix.res[threadIdx.x];
-    {  // the first kJobCache jobs in one round trip (every warp walks every job's descriptor)
-      const uint32_t nc = n_jobs < kJobCache ? n_jobs : kJobCache;
-      for (uint32_t i = threadIdx.x; i < nc * (uint32_t)(sizeof(Job) / 4); i += blockDim.x)
+    // the plan's tile total and (up to kJobCache) jobs are in shared memory; more jobs are read from the scratch
+    const uint64_t plan_tiles = tiles_s;
+    if (n_jobs > kJobCache) {  // the first kJobCache jobs in one round trip (every warp walks every descriptor)
+      for (uint32_t i = threadIdx.x; i < kJobCache * (uint32_t)(sizeof(Job) / 4); i += blockDim.x)
         reinterpret_cast<uint32_t*>(jobs_s)[i] = reinterpret_cast<const uint32_t*>(P.sc.jobs)[i];
       cta_barrier();
     }
     // the results go to the bell now (host-memory writes in flight during the move; the release after the
     // move orders them before done_seq)
-    if (threadIdx.x < P.n_rings) B->res[threadIdx.x] = my_res;
+    if (threadIdx.x < P.n_rings) {
+      crk_ring_result my_res = res_s[threadIdx.x];
+      my_res.reply_bytes = reply_s[threadIdx.x];
+      B->res[threadIdx.x] = my_res;
+    }
     if (threadIdx.x == 0) B->status = bad_s ? CRK_E_ARG : CRK_OK;
     const uint32_t sh = plan_tiles <= 4 ? 11u : 13u;
     STEP_MARK(threadIdx.x == 0, 16, sh ^ jobs_s[0].type);
@@ -271,6 +284,11 @@ cudaError_t launch_server(const IndexDev& ix, const ConfigDev& cfg, const Scratc
   P.bell = bell;
   P.n_rings = n_rings;
   for (uint32_t r = 0; r < n_rings; ++r) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, rings[r].base) == cudaSuccess && a.type == cudaMemoryTypeDevice)
+      P.dev_rings |= 1ull << r;
+    else
+      (void)cudaGetLastError();
     P.rings[r].base = rings[r].base;
     P.rings[r].mask = rings[r].cap - 1;
     P.send[r].base = send_rings[r].base;
