@@ -393,6 +393,14 @@ int crk_server_start(crk_ctx* ctx, crk_index* idx, uint32_t n_rings, const crk_r
                      const crk_ring* send_rings, uint64_t region_base, uint64_t region_bytes, crk_server_bell* bell,
                      crk_stream_t stream, crk_server** out);
 int crk_server_stop(crk_server* server);
+/* One step through a running server whose bell is host memory (the protocol above, done in C so no
+ * interpreter sits in the round trip): writes head/tail/send_off of the server's n_rings rings, bumps seq and
+ * spins until done_seq == seq or timeout_ns elapses.  Returns the bell's status (CRK_OK, or CRK_E_ARG for an
+ * invalid window); the per-ring results and device stamps are in the bell.  CRK_E_ARG also for a device-memory
+ * bell or null arrays; CRK_E_CUDA when the step did not finish in time (the kernel failed or the timeout is too
+ * short: the server is then in an unknown state -- stop it). */
+int crk_server_step(crk_server* server, const uint64_t* heads, const uint64_t* tails, const uint64_t* send_offs,
+                    uint64_t timeout_ns);
 
 /* ---------------------------------------------------------------- memory utilities
  * Pinned, mapped, portable host memory for rings (cudaHostAlloc; with UVA the returned pointer is

@@ -132,6 +132,7 @@ def lib():
             "crk_server_start": (C.c_int, [vp, vp, u32, C.POINTER(CRing), C.POINTER(CRing), u64, u64, vp, vp,
                                            C.POINTER(vp)]),
             "crk_server_stop": (C.c_int, [vp]),
+            "crk_server_step": (C.c_int, [vp, C.POINTER(u64), C.POINTER(u64), C.POINTER(u64), u64]),
             "crk_graph_destroy": (None, [vp]),
             "crk_host_alloc": (C.c_int, [u64, C.POINTER(vp)]),
             "crk_host_free": (None, [vp]),
@@ -638,18 +639,15 @@ class Server:
         index.n_rings = self.n
 
     def step(self, windows, send_offs, timeout_s: float = 30.0) -> dict:
-        import time
+        """crk_server_step: the cursors written, seq bumped and done_seq awaited in C."""
         b = self.bell
-        for r, (head, tail) in enumerate(windows):
-            b.head[r] = head
-            b.tail[r] = tail
-            b.send_off[r] = send_offs[r]
-        seq = b.seq + 1
-        b.seq = seq
-        t0 = time.perf_counter()
-        while b.done_seq != seq:
-            if time.perf_counter() - t0 > timeout_s:
-                raise CrkError(E_CUDA, "crk_server step timed out")
+        arr = u64 * self.n
+        heads = arr(*[h for h, _ in windows])
+        tails = arr(*[t for _, t in windows])
+        offs = arr(*send_offs[:self.n])
+        st = lib().crk_server_step(self.h, heads, tails, offs, int(timeout_s * 1e9))
+        if st == E_CUDA:
+            raise CrkError(E_CUDA, "crk_server step timed out")
         res = [dict(status=x.status, n_records=x.n_records, n_frags=x.n_frags, rec_base=x.rec_base,
                     consumed=x.consumed, reply_bytes=x.reply_bytes) for x in b.res[:self.n]]
         ph = [b.t_phase_ns[i] - b.t_begin_ns for i in range(5)]

@@ -3,6 +3,7 @@
 // k_move.
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -911,6 +912,7 @@ struct crk_server {
   cudaStream_t stream;
   crk_server_bell* bell;
   bool host_bell;  // mapped host memory: the CPU writes it directly
+  uint32_t n_rings;
 };
 
 namespace {
@@ -956,6 +958,7 @@ int crk_server_start(crk_ctx* c, crk_index* x, uint32_t n_rings, const crk_ring*
   S->stream = (cudaStream_t)stream;
   S->bell = bell;
   S->host_bell = a.type == cudaMemoryTypeHost;
+  S->n_rings = n_rings;
   const cudaError_t e = launch_server(x->ix, c->cd, c->sc, c->d_schemas, bell, n_rings, rings, send_rings,
                                       region_base, region_bytes, S->stream);
   if (e != cudaSuccess) { delete S; return cuda_fail(e); }
@@ -971,6 +974,29 @@ int crk_server_stop(crk_server* S) {
   delete S;
   if (st != CRK_OK) return st;
   return e == cudaSuccess ? CRK_OK : cuda_fail(e);
+}
+
+int crk_server_step(crk_server* S, const uint64_t* heads, const uint64_t* tails, const uint64_t* send_offs,
+                    uint64_t timeout_ns) {
+  if (!S || !S->host_bell || !heads || !tails || !send_offs) return CRK_E_ARG;
+  crk_server_bell* B = S->bell;
+  for (uint32_t r = 0; r < S->n_rings; ++r) {
+    B->head[r] = heads[r];
+    B->tail[r] = tails[r];
+    B->send_off[r] = send_offs[r];
+  }
+  const uint64_t seq = B->seq + 1;
+  std::atomic_thread_fence(std::memory_order_release);  // the cursors before seq (x86: stores are ordered)
+  B->seq = seq;
+  const auto t0 = std::chrono::steady_clock::now();
+  for (uint32_t spin = 0; B->done_seq != seq; ++spin) {
+    if ((spin & 1023) == 0 &&
+        (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count() >
+            timeout_ns)
+      return CRK_E_CUDA;
+  }
+  std::atomic_thread_fence(std::memory_order_acquire);  // results after done_seq
+  return B->status;
 }
 
 int crk_host_alloc(uint64_t bytes, void** out) {

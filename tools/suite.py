@@ -199,6 +199,16 @@ def server_latency(ctx, reps=2000):
             dv.append(out["device_ns"])
             ph.append(list(out["phase_end_ns"].values()))
         ok = out["results"][0]["status"] == 0 and out["results"][0]["reply_bytes"] == 32
+        # the same step timed around the C call alone (crk_server_step: cursors, seq, spin on done_seq)
+        import ctypes as C
+        u64a = C.c_uint64 * 1
+        hs, ts, so = u64a(0), u64a(w), u64a(0)
+        crt = []
+        for i in range(reps):
+            t0 = time.perf_counter_ns()
+            st = crk.lib().crk_server_step(srv.h, hs, ts, so, 10 ** 9)
+            crt.append(time.perf_counter_ns() - t0)
+            ok &= st == 0
     finally:
         srv.stop()
     ok &= bool(torch.equal(region[4096:8192], data))  # device allocations wait for a running server
@@ -213,7 +223,9 @@ def server_latency(ctx, reps=2000):
     finally:
         srv2.stop()
     ok2 &= bool(torch.equal(region[:a.numel()], a))
-    return {"one_record_roundtrip_us_median": round(float(np.median(rt)) / 1e3, 2),
+    return {"one_record_c_roundtrip_us_median": round(float(np.median(crt)) / 1e3, 2),
+            "one_record_c_roundtrip_us_p99": round(float(np.percentile(crt, 99)) / 1e3, 2),
+            "one_record_roundtrip_us_median": round(float(np.median(rt)) / 1e3, 2),
             "one_record_device_us_median": round(float(np.median(dv)) / 1e3, 2),
             "one_record_roundtrip_us_p99": round(float(np.percentile(rt, 99)) / 1e3, 2), "ok": bool(ok),
             "one_record_phase_end_us_median": dict(zip(("setup", "scan", "parse", "plan", "move"),
