@@ -62,6 +62,11 @@ __device__ __forceinline__ void phase_sync() {
 // (generic paths of k_move.cuh).
 // tiles dealt to the warps round-robin: 2 KiB (one chunk-loop pass per warp) when the step moves at most
 // ~4 mover tiles' worth of bytes, else 8 KiB
+#ifndef CRK_SERVER_POLLERS
+#define CRK_SERVER_POLLERS 1
+#endif
+constexpr uint32_t kPollers = CRK_SERVER_POLLERS;  // warps whose lane 0 polls the doorbell (A/B on one B200: 4 staggered
+                                                   // pollers 18.1 us round trip per 4 KiB call vs 16.0 for one)
 constexpr uint64_t kPrefetchMax = 64 * 1024;  // records up to this size have their payload prefetched to L2
 constexpr uint32_t kJobCache = 32;   // jobs staged in shared memory at the start of the move phase
 __device__ __forceinline__ uint64_t job_tiles(const Job& J, uint32_t sh) {
@@ -100,18 +105,22 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
   crk_server_bell* B = P.bell;
   const IndexDev& ix = P.ix;
   uint64_t seen = B->done_seq;
+  if (threadIdx.x == 0) seq_s = seen;
+  cta_barrier();
   for (;;) {
-    // ---- wait for a new step
-    if (threadIdx.x == 0) {
+    // ---- wait for a new step: lane 0 of kPollers warps polls the doorbell (one read in flight each; more than
+    // one poller measured slower: their reads contend on the link)
+    if (lane == 0 && warp < kPollers) {
       uint64_t s;
-      while ((s = ld_acquire_sys(&B->seq)) == seen) __nanosleep(64);
-      seq_s = s;
-      stop_s = B->stop != 0;
+      while ((s = ld_acquire_sys(&B->seq)) == seen && *(volatile uint64_t*)&seq_s == seen) __nanosleep(64 + 96 * warp);
+      if (s != seen) seq_s = s;  // every poller that saw it stores the same value
+    }
+    phase_sync();
+    // the stop flag is read with the step's cursors (one round trip) and checked after the setup barrier
+    if (threadIdx.x == 0) {
       bad_s = 0;
       B->t_begin_ns = gtimer();
     }
-    phase_sync();
-    if (stop_s) break;
     TL_END(P.cfg, 6);
     seen = seq_s;
     // ---- step setup: schemas (re-read: registrations may follow the start), send cursors, xid table
@@ -119,6 +128,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
       reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
     // the step's cursors: one read of the bell per value, all in flight at once (a host bell is read
     // over PCIe; every later use is from shared memory)
+    if (threadIdx.x == blockDim.x - 1) stop_s = *(volatile uint64_t*)&B->stop != 0;
     for (uint32_t r = threadIdx.x; r < P.n_rings; r += blockDim.x) {
       send.r[r] = P.send[r];
       send.off[r] = *(volatile uint64_t*)&B->send_off[r];
@@ -131,6 +141,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     }
     for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
     phase_sync();
+    if (stop_s) break;
     TL_END(P.cfg, 0);
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     STEP_MARK(threadIdx.x == 0, 0, 0);

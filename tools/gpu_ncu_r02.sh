@@ -6,6 +6,7 @@
 #   walk.ncu-rep / emit.ncu-rep   --set full of the chunked scan's two kernels on the C5 endpoint
 #   scan.ncu-rep          --set full of the one-CTA scan (scan_chunking=1) on the C5 endpoint
 #   host_step_metrics.csv PCIe / DRAM counters of a zero-copy (host ring) server step
+#   front.ncu-rep         --set full of the fused single-CTA front end in smoke() (cold: ncu flushes the caches)
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 NCU=/usr/local/cuda/bin/ncu
@@ -18,5 +19,6 @@ $NCU --profile-from-start off --set full --import-source on --clock-control none
 $NCU --profile-from-start off --set full --import-source on --clock-control none -k regex:chunk_walk -c 1 -o gpurun_out/walk -f $PS --steps 1 > gpurun_out/ncu_walk.log 2>&1
 $NCU --profile-from-start off --set full --import-source on --clock-control none -k regex:chunk_emit -c 1 -o gpurun_out/emit -f $PS --steps 1 > gpurun_out/ncu_emit.log 2>&1
 $NCU --profile-from-start off --set full --import-source on --clock-control none -k regex:frame_scan -c 1 -o gpurun_out/scan -f $PS --steps 1 --ctx scan_chunking=1 > gpurun_out/ncu_scan.log 2>&1
+$NCU --set full --import-source on --clock-control none -k regex:front_small -c 1 -o gpurun_out/front -f python __graft_entry__.py smoke > gpurun_out/ncu_front.log 2>&1
 bash tools/gpu_ncu_host.sh
 echo done > gpurun_out/ncu_r02_done.txt

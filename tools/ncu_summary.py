@@ -85,7 +85,7 @@ def main():
         if os.path.exists(os.path.join(OUT, f"{lst}.csv")):
             json.dump(launches(os.path.join(OUT, f"{lst}.csv")), open(os.path.join(PROF, f"{tag}_{lst}.json"), "w"),
                       indent=1)
-    for name in ("mover", "scan", "walk", "emit"):
+    for name in ("mover", "scan", "walk", "emit", "front"):
         rep = os.path.join(OUT, f"{name}.ncu-rep")
         if not os.path.exists(rep):
             continue
