@@ -16,9 +16,11 @@ __global__ void __launch_bounds__(kParseWarps * 32) parse_kernel(IndexDev ix, co
   __shared__ uint32_t prefix[kMaxRings + 1];
   __shared__ __align__(16) uint8_t heads[kParseWarps][kHeadBuf];
   TL_BEGIN(cfg, TL_PARSE);
+  // the grid is sized by the index's capacity: CTAs past the step's record count leave before loading anything
+  const uint32_t total = *ix.total;
+  if (blockIdx.x * kParseWarps >= total) return;
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(tab)[i];
-  const uint32_t total = *ix.total;
   for (uint32_t i = threadIdx.x; i <= n_rings; i += blockDim.x) prefix[i] = ix.rec_prefix[i];
   __syncthreads();
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
