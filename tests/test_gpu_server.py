@@ -10,7 +10,7 @@ import torch
 
 import oracle as O
 from paper_conf_sc_eilingkkflm23_b200 import crk, gen
-from tests.gpu_util import ctx_for, d2h_call, h2d_call, make_ring, ocfg
+from tests.gpu_util import compare_parse, compare_scan, ctx_for, d2h_call, h2d_call, make_ring, ocfg
 
 pytestmark = [pytest.mark.gpu, pytest.mark.timeout(300)]
 
@@ -200,3 +200,74 @@ def test_servers_back_to_back_on_one_context():
         assert out["results"][0]["status"] == O.OK and out["results"][0]["reply_bytes"] == 32
         srv.stop()
     assert region[64:64 + 4096].cpu().numpy().tobytes() == payload.tobytes()
+
+
+@pytest.mark.parametrize("host,strict,F", [(False, True, 100), (False, False, 4096), (True, True, 1024)])
+def test_server_lean_steps_match_oracle(host, strict, F):
+    """Steps of well-formed single-fragment memcpy CALLs only -- the persistent server's lean path (one warp over a
+    shared-memory copy of the windows) -- against the oracle: ring results, reply bytes (framed with F, here smaller
+    than most replies), destination bytes, and the index tables the general phases would have written (fragment /
+    record tables vs or_frame_scan, parsed CALLs vs or_parse_call, serve decisions vs or_serve)."""
+    cfg = ocfg(strict=strict, F=F)
+    ctx = ctx_for(cfg)
+    n_rings, cap, scap = 3, 1 << 16, 1 << 18
+    region_bytes = 1 << 20
+    region = torch.zeros(region_bytes, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    g = gen.rng(0x1EA + F + 2 * strict + host)
+    host_region = gen.random_bytes(0x1EA1, region_bytes).copy()
+    region.copy_(torch.from_numpy(host_region))
+    rings = [crk.Ring.host(cap) if host else crk.Ring.device(cap) for _ in range(n_rings)]
+    sends = [crk.Ring.host(scap) if host else crk.Ring.device(scap) for _ in range(n_rings)]
+    idx = ctx.index(n_rings, 3 * 64, 3 * 32)
+    torch.cuda.synchronize()
+    srv = crk.Server(idx, rings, sends, base, region_bytes)
+    lean = 0
+    try:
+        tails = [cap - 3000 + 37 * r for r in range(n_rings)]  # windows cross the wrap
+        send_offs = [scap - 2000 + 4 * r for r in range(n_rings)]
+        for step in range(12):
+            heads = list(tails)
+            for r in range(n_rings):
+                wire = b""
+                for i in range(int(g.integers(0, 5))):
+                    xid = (step << 16) | (r << 8) | i
+                    if g.integers(0, 2):  # HtoD to a private slot of the lower half, any alignment
+                        data = gen.random_bytes((step * 7 + r * 3 + i) & 0xFFFF, int(g.integers(0, 2500)))
+                        c = h2d_call(xid, data, base + (r * 4 + i) * 4096 + int(g.integers(0, 64)))
+                    else:  # DtoH from the upper half
+                        size = int(g.integers(0, 5000))
+                        c = d2h_call(xid, base + region_bytes // 2 + int(g.integers(0, region_bytes // 2 - size)), size)
+                    wire += O.encode_call(*c, cfg, F=1 << 16)  # one fragment per CALL
+                rings[r].write(tails[r], wire)
+                tails[r] += len(wire)
+            before = [ring_bytes(rg) for rg in rings]
+            out = srv.step(list(zip(heads, tails)), send_offs)
+            want = O.serve([(b, h, t) for b, h, t in zip(before, heads, tails)], cfg, host_region, base,
+                           [scap] * n_rings, send_offs, max_frags_per_ring=64, max_records_per_ring=32)
+            assert out["status"] == O.OK
+            ph = list(out["phase_end_ns"].values())
+            lean += ph[1] == ph[2] == ph[3] == ph[4]  # the lean path stamps its phases at once
+            for r in range(n_rings):
+                res = out["results"][r]
+                assert res["status"] == want["scan_status"][r] == O.OK, (step, r, res)
+                assert res["consumed"] == want["consumed"][r] == tails[r], (step, r)
+                assert res["reply_bytes"] == want["reply_bytes"][r], (step, r)
+                n = want["reply_bytes"][r]
+                exp = bytes(np.roll(want["send"][r], -(send_offs[r] % scap))[:n])
+                assert sends[r].read(send_offs[r], n) == exp, (step, r)
+            assert np.array_equal(region.cpu().numpy(), host_region), step
+            T = idx.tables(n_rings, sync=False)
+            for r in range(n_rings):
+                s = compare_scan(T, r, before[r], heads[r], tails[r], 64, 32)
+                compare_parse(T, r, before[r], s, cfg)
+            P = T["parsed"]
+            assert [x["status"] for x in want["records"]] == list(P["serve_status"]), step
+            assert [x["reply_err"] for x in want["records"]] == list(P["serve_reply_err"]), step
+            assert [x["reply_wire"] for x in want["records"]] == list(P["serve_reply_wire"]), step
+            assert [x["reply_off"] for x in want["records"]] == list(P["serve_reply_off"]), step
+            for r in range(n_rings):
+                send_offs[r] += want["reply_bytes"][r]
+    finally:
+        srv.stop()
+    assert lean >= 6, lean  # most steps took the lean path
