@@ -6,6 +6,12 @@
 // functions are the launched kernels' own (scan_ring_cta, parse_record, plan_small_block), so the index
 // tables, statuses and jobs are identical; the phases hand data to each other inside the CTA, ordered by
 // block barriers.
+//
+// A step of well-formed single-fragment memcpy CALLs takes the lean path (k_lean.cuh): one warp over a shared-
+// memory copy of the windows, the CTA moving the payloads and replies itself, an empty plan left for the mover.
+#include <mutex>
+
+#include "k_lean.cuh"
 #include "k_parse.cuh"
 #include "k_plan.cuh"
 #include "k_scan.cuh"
@@ -39,6 +45,9 @@ __device__ unsigned long long g_front_trace[8];
 
 __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontParams P) {
   pdl_entry();
+  extern __shared__ __align__(16) uint8_t lean_sh[];  // kLeanWin: the windows of a lean step
+  __shared__ LeanState lean_s;
+  __shared__ uint64_t win_head[kLeanRings], win_tail[kLeanRings], send_off[kLeanRings];
   __shared__ ScanState S;
   __shared__ SchemaTable sch;
   __shared__ __align__(16) uint8_t heads[kFrontWarps][kHeadBuf];
@@ -54,8 +63,25 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
+  // a serve step over at most kLeanRings rings: its cursors (doorbell or parameters) for the lean path
+  const bool try_lean = P.plan && n_rings <= kLeanRings;
+  if (try_lean && threadIdx.x < n_rings) {
+    const uint32_t r = threadIdx.x;
+    win_head[r] = P.rings.doorbell ? P.rings.doorbell[r] : P.rings.r[r].head;
+    win_tail[r] = P.rings.doorbell ? P.rings.doorbell[n_rings + r] : P.rings.r[r].tail;
+    send_off[r] = P.send.doorbell ? P.send.doorbell[2 * n_rings + r] : P.send.off[r];
+  }
   cta_barrier();
   FRONT_MARK(1);
+  if (try_lean) {
+    const LeanMover mv{P.sc.scan_tmp + P.sc.max_jobs + 1, P.sc.counters};
+    if (lean_step(ix, P.cfg, sch, n_rings, [&](uint32_t r) { return P.rings.r[r]; },
+                  [&](uint32_t r) { return P.send.r[r]; }, win_head, win_tail, send_off, P.region_base,
+                  P.region_bytes, lean_sh, lean_s, nullptr, &mv)) {
+      TL_END(P.cfg, TL_FUSED);
+      return;
+    }
+  }
   // ---- K1: each ring in turn by the whole CTA, then dense record numbering (prefix[] in shared memory)
   if (threadIdx.x == 0) prefix[0] = 0;
   for (uint32_t r = 0; r < n_rings; ++r) {
@@ -128,7 +154,21 @@ cudaError_t launch_front_small(const IndexDev& ix, const ConfigDev& cfg, Scratch
   P.region_base = region_base;
   P.region_bytes = region_bytes;
   prof_mark(PROF_SCAN, true, s);
-  CRK_LAUNCH(pdl_of(cfg), front_small_kernel, 1, kFrontThreads, 0, s, P);
+  {  // the lean path's dynamic shared memory: a per-device opt-in, raised once
+    static std::mutex mu;
+    static bool set[kMaxDevices] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!set[dev]) {
+      e = cudaFuncSetAttribute(front_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kLeanWin);
+      if (e != cudaSuccess) return e;
+      set[dev] = true;
+    }
+  }
+  CRK_LAUNCH(pdl_of(cfg), front_small_kernel, 1, kFrontThreads, kLeanWin, s, P);
   prof_mark(PROF_SCAN, false, s);
   return cudaGetLastError();
 }
