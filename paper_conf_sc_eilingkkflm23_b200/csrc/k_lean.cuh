@@ -8,7 +8,8 @@ namespace {
 
 // ---- lean steps ----------------------------------------------------------------------------------------------
 // The common small step -- a few well-formed memcpy CALLs (RFC 5531 §9 call with AUTH_NONE credential and
-// verifier, one record-marking fragment each, the built-in HtoD / DtoH schemas), every one of them served OK --
+// verifier, the built-in HtoD / DtoH schemas, record-marking fragments of any length whose first one holds the
+// fixed-layout head), every one of them served OK --
 // done by one warp over a shared-memory copy of the windows, with no table round trips between the phases:
 // lane 0 walks the header chains, lane k checks record k and makes its serve decision, a warp scan gives the reply
 // offsets; then the whole CTA writes the index tables (exactly what the general phases write for such a step),
@@ -24,16 +25,23 @@ constexpr uint32_t kLeanWin = 64 * 1024;   // shadow bytes (the server's dynamic
 constexpr uint32_t kLeanRecs = 32;          // records: one per lane of warp 0
 constexpr uint32_t kLeanRings = 8;
 constexpr uint64_t kLeanD2H = 64 * 1024;    // DtoH reply data the CTA encodes itself
+constexpr uint32_t kLeanFrags = 128;        // record-marking fragments of the step
 
 struct LeanRec {
   uint64_t cur, ptr, n, off, c, size;  // header cursor; HtoD dst / DtoH src; bytes copied / DtoH size; reply cursor;
                                        // HtoD opaque count and size argument
-  uint32_t len, ring, slot, xid, d2h, Ll, w, so_, sm_, pad_;
+  uint32_t len, ring, slot, xid, d2h, Ll, w, so_, sm_;  // len: the record's logical length
+  uint32_t f0, nf, fslot;  // its fragments: first in the step's list, count, ring-local number of the first
+};
+struct LeanFrag {
+  uint64_t cur;            // header cursor
+  uint32_t len, lstart;    // data bytes, logical offset of the first one
 };
 struct LeanState {
   LeanRec rec[kLeanRecs];
+  LeanFrag frag[kLeanFrags];
   uint32_t prefix[kLeanRings + 1];
-  uint32_t soff[kLeanRings], smask[kLeanRings];
+  uint32_t soff[kLeanRings], smask[kLeanRings], fcount[kLeanRings];
   uint64_t reply_bytes[kLeanRings];
   uint32_t ok;
 };
@@ -49,6 +57,24 @@ __device__ __noinline__ uint32_t shadow_be32(const uint8_t* sh, uint32_t so, uin
   uint32_t v = 0;                                                                  // 256-byte aligned, >= 256 B)
 #pragma unroll 1
   for (uint32_t k = 0; k < 4; ++k) v = (v << 8) | sh[so + ((c + k) & sm)];
+  return v;
+}
+
+// Logical byte o of a lean record (RFC 5531 §11: the concatenation of its fragments' data).
+__device__ __noinline__ uint32_t lean_byte(const uint8_t* sh, const LeanState& L, const LeanRec& q, uint64_t o) {
+#pragma unroll 1
+  for (uint32_t k = q.f0; k < q.f0 + q.nf; ++k) {
+    const LeanFrag& f = L.frag[k];
+    if (o < (uint64_t)f.lstart + f.len) return sh[q.so_ + ((f.cur + 4 + o - f.lstart) & q.sm_)];
+  }
+  return 0;
+}
+// Big-endian word at logical offset o of a lean record.
+__device__ __forceinline__ uint32_t lean_be32(const uint8_t* sh, const LeanState& L, const LeanRec& q, uint64_t o) {
+  if (q.nf == 1) return shadow_be32(sh, q.so_, q.sm_, q.cur + 4 + o);
+  uint32_t v = 0;
+#pragma unroll 1
+  for (uint32_t k = 0; k < 4; ++k) v = (v << 8) | lean_byte(sh, L, q, o + k);
   return v;
 }
 
@@ -103,26 +129,44 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
   // ---- warp 0: the chains, the records' checks and serve decisions, the reply offsets
   if (warp == 0) {
     uint32_t ok = 1, nrec = 0;
-    if (lane == 0) {  // RFC 5531 §11 chains: every header a whole record (last bit), each record inside the window
+    if (lane == 0) {  // RFC 5531 §11 chains: whole records (up to a last fragment) inside the window, in capacity
+      uint32_t nfr = 0;
 #pragma unroll 1
-      for (uint32_t r = 0; r < n; ++r) {
+      for (uint32_t r = 0; r < n && ok; ++r) {
         L.prefix[r] = nrec;
         uint64_t p = head[r];
-        uint32_t nr = 0;
+        uint32_t nr = 0, nf = 0;
 #pragma unroll 1
         while (ok && p < tail[r]) {
-          const uint32_t h = p + 4 <= tail[r] ? shadow_be32(sh, L.soff[r], L.smask[r], p) : 0u, len = h & 0x7fffffffu;
-          if (!(h >> 31) || len < 40 || p + 4 + len > tail[r] || len > cfg.max_record_bytes || nrec >= kLeanRecs ||
-              nr >= ix.recs_per_ring || nr >= ix.frags_per_ring) { ok = 0; break; }
-          LeanRec& q = L.rec[nrec++];
+          if (nrec >= kLeanRecs || nr >= ix.recs_per_ring) { ok = 0; break; }
+          LeanRec& q = L.rec[nrec];
           q.cur = p;
-          q.len = len;
           q.ring = r;
-          q.slot = nr++;
+          q.slot = nr;
           q.so_ = L.soff[r];
           q.sm_ = L.smask[r];
-          p += 4 + len;
+          q.f0 = nfr;
+          q.fslot = nf;
+          uint64_t sum = 0;
+          bool last = false;
+#pragma unroll 1
+          while (!last) {
+            const uint32_t h = p + 4 <= tail[r] ? shadow_be32(sh, q.so_, q.sm_, p) : 0u, flen = h & 0x7fffffffu;
+            last = h >> 31;
+            if (p + 4 > tail[r] || p + 4 + flen > tail[r] || sum + flen > cfg.max_record_bytes ||
+                nf >= ix.frags_per_ring || nfr >= kLeanFrags) { ok = 0; break; }
+            L.frag[nfr++] = LeanFrag{p, flen, (uint32_t)sum};
+            ++nf;
+            sum += flen;
+            p += 4 + flen;
+          }
+          if (!ok) break;
+          q.len = (uint32_t)sum;
+          q.nf = nfr - q.f0;
+          ++nrec;
+          ++nr;
         }
+        L.fcount[r] = nf;
       }
       L.prefix[n] = nrec;
       STEP_MARK(true, 22, nrec);
@@ -137,8 +181,9 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       LeanRec& q = L.rec[lane];
       ring = q.ring;
       const uint64_t b0 = q.cur + 4;  // logical offset 0
-      uint32_t wv[14];                // the fixed-layout head (and the DtoH arguments)
-      const uint32_t o0 = (uint32_t)(b0 & q.sm_);
+      uint32_t wv[14];                // the fixed-layout head (and the DtoH arguments): in the first fragment
+      const uint32_t o0 = (uint32_t)(b0 & q.sm_), flen0 = L.frag[q.f0].len;
+      if (flen0 < 52) good = false;
       if (!(o0 & 3) && o0 + 56 <= q.sm_ + 1) {  // aligned and not across the shadow's wrap: 14 independent loads
         const uint32_t* wp = reinterpret_cast<const uint32_t*>(sh + q.so_ + o0);
 #pragma unroll
@@ -149,7 +194,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       }
       xid = wv[0];
       // RFC 5531 §9: CALL, rpcvers 2, the program and version, zero-length credential and verifier bodies
-      good = wv[1] == 0 && wv[2] == 2 && wv[3] == cfg.prog && wv[4] == cfg.vers && wv[7] == 0 && wv[9] == 0;
+      good = good && wv[1] == 0 && wv[2] == 2 && wv[3] == cfg.prog && wv[4] == cfg.vers && wv[7] == 0 && wv[9] == 0;
       const uint32_t proc = wv[5];
       uint32_t e = 0;  // the procedure's first schema entry must be the built-in memcpy layout
 #pragma unroll 1
@@ -166,9 +211,8 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
         const uint64_t c = wv[12], pn = pad4(c), o2 = 52 + c + pn;
         good = o2 + 8 == q.len;
 #pragma unroll 1
-        for (uint64_t i = 0; good && cfg.strict && i < pn; ++i) good = sh[q.so_ + ((b0 + 52 + c + i) & q.sm_)] == 0;
-        const uint64_t size = good ? ((uint64_t)shadow_be32(sh, q.so_, q.sm_, b0 + o2) << 32) |
-                                         shadow_be32(sh, q.so_, q.sm_, b0 + o2 + 4) : 0;
+        for (uint64_t i = 0; good && cfg.strict && i < pn; ++i) good = lean_byte(sh, L, q, 52 + c + i) == 0;
+        const uint64_t size = good ? ((uint64_t)lean_be32(sh, L, q, o2) << 32) | lean_be32(sh, L, q, o2 + 4) : 0;
         good = good && !(cfg.strict && c != size);              // E_SIZE (reading R9)
         q.c = c;
         q.size = size;
@@ -177,7 +221,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
         q.Ll = 28;
       } else if (d2h) {
         q.n = ((uint64_t)wv[12] << 32) | wv[13];
-        good = q.len == 56 && q.n <= 0xffffffffull && region_ok(region_base, region_bytes, q.ptr, q.n);  // E_PTR (reading R21)
+        good = q.len == 56 && flen0 >= 56 && q.n <= 0xffffffffull && region_ok(region_base, region_bytes, q.ptr, q.n);  // E_PTR (reading R21)
         d2h_bytes = q.n;
         q.Ll = (uint32_t)(32 + q.n + pad4(q.n));
       }
@@ -225,7 +269,8 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     ix.rings[tid] = R;
     crk_ring_result rr;
     rr.status = CRK_OK;
-    rr.n_records = rr.n_frags = L.prefix[tid + 1] - L.prefix[tid];
+    rr.n_records = L.prefix[tid + 1] - L.prefix[tid];
+    rr.n_frags = L.fcount[tid];
     rr.rec_base = L.prefix[tid];
     rr.consumed = tail[tid];
     rr.reply_bytes = L.reply_bytes[tid];
@@ -245,14 +290,18 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
   }
   if (tid < N) {
     const LeanRec& q = L.rec[tid];
-    const uint32_t d = tid, fs = q.ring * FC + q.slot, rs = q.ring * RC + q.slot;
-    ix.frag_phys[fs] = q.cur + 4;
-    ix.frag_lstart[fs] = 0;
-    ix.frag_hdr[fs] = q.len | 0x80000000u;
+    const uint32_t d = tid, fs = q.ring * FC + q.fslot, rs = q.ring * RC + q.slot;
+#pragma unroll 1
+    for (uint32_t j = 0; j < q.nf; ++j) {
+      const LeanFrag& f = L.frag[q.f0 + j];
+      ix.frag_phys[fs + j] = f.cur + 4;
+      ix.frag_lstart[fs + j] = f.lstart;
+      ix.frag_hdr[fs + j] = f.len | (j + 1 == q.nf ? 0x80000000u : 0u);
+    }
     ix.rec_begin[rs] = q.cur;
     ix.rec_len[rs] = q.len;
     ix.rec_frag0[rs] = fs;
-    ix.rec_nfrags[rs] = 1;
+    ix.rec_nfrags[rs] = q.nf;
     ix.p_slot[d] = rs;
     ix.p_ring[d] = q.ring;
     ix.p_xid[d] = q.xid;
@@ -260,8 +309,8 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     ix.p_status[d] = CRK_OK;
     ix.p_nitems[d] = q.d2h ? 2 : 3;
     ix.p_frag0[d] = fs;
-    ix.p_nfrags[d] = 1;
-    ix.p_flen0[d] = q.len;
+    ix.p_nfrags[d] = q.nf;
+    ix.p_flen0[d] = L.frag[q.f0].len;
     // items: u64 ptr @40; then DtoH: u64 size @48; HtoD: opaque<> @52 (count c), u64 size after its pad
     const uint64_t b = (uint64_t)d * kMaxItems, o2 = 52 + q.c + pad4(q.c), size = q.d2h ? q.n : q.size;
     ix.p_kind[b] = CRK_K_U64;
@@ -296,10 +345,15 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
 #pragma unroll 1
   for (uint32_t d = 0; d < N; ++d) {
     const LeanRec& q = L.rec[d];
-    if (!q.d2h) {
-      uint8_t* dst = reinterpret_cast<uint8_t*>(q.ptr);
+    if (!q.d2h) {  // logical [52, 52 + n) of the record, fragment by fragment
+      uint8_t* dst = reinterpret_cast<uint8_t*>(q.ptr) - 52;
 #pragma unroll 1
-      for (uint64_t i = tid; i < q.n; i += blockDim.x) dst[i] = sh[q.so_ + ((q.cur + 56 + i) & q.sm_)];
+      for (uint32_t j = 0; j < q.nf; ++j) {
+        const LeanFrag& f = L.frag[q.f0 + j];
+        const uint64_t a = max((uint64_t)f.lstart, (uint64_t)52), b = min((uint64_t)f.lstart + f.len, 52 + q.n);
+#pragma unroll 1
+        for (uint64_t o = a + tid; o < b; o += blockDim.x) dst[o] = sh[q.so_ + ((f.cur + 4 + o - f.lstart) & q.sm_)];
+      }
     }
     const RingDesc O = send_of(q.ring);
     const uint8_t* src = reinterpret_cast<const uint8_t*>(q.ptr);

@@ -211,8 +211,8 @@ def _mover_jobs(ctx) -> int:
                                                 ("server", True, True, 1024), ("serve", False, True, 100),
                                                 ("serve", True, False, 1024)])
 def test_lean_steps_match_oracle(mode, host, strict, F):
-    """Steps of well-formed single-fragment memcpy CALLs only -- the lean path (one warp over a shared-memory copy
-    of the windows) of the persistent server and of crk_serve's fused front end -- against the oracle: ring
+    """Steps of well-formed memcpy CALLs only (single- and multi-fragment) -- the lean path (one warp over a shared-
+    memory copy of the windows) of the persistent server and of crk_serve's fused front end -- against the oracle: ring
     results, reply bytes (framed with F, here smaller than most replies), destination bytes, and the index tables
     the general phases would have written (fragment / record tables vs or_frame_scan, parsed CALLs vs
     or_parse_call, serve decisions vs or_serve)."""
@@ -246,7 +246,8 @@ def test_lean_steps_match_oracle(mode, host, strict, F):
                     else:  # DtoH from the upper half
                         size = int(g.integers(0, 5000))
                         c = d2h_call(xid, base + region_bytes // 2 + int(g.integers(0, region_bytes // 2 - size)), size)
-                    wire += O.encode_call(*c, cfg, F=1 << 16)  # one fragment per CALL
+                    # one fragment per CALL, or several (the first one always holds the fixed-layout head)
+                    wire += O.encode_call(*c, cfg, F=int(g.choice([1 << 16, 1000, 256])))
                 rings[r].write(tails[r], wire)
                 tails[r] += len(wire)
             before = [ring_bytes(rg) for rg in rings]
