@@ -59,9 +59,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const IndexDev& ix = P.ix;
   const uint32_t n_rings = P.rings.n_rings;
-  // ---- setup: schemas, an empty xid table
-  for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
-    reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
+  // ---- setup: an empty xid table (the schemas are loaded below, for the general phases only)
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
   // a serve step over at most kLeanRings rings: its cursors (doorbell or parameters) for the lean path
   const bool try_lean = P.plan && n_rings <= kLeanRings;
@@ -75,13 +73,16 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   FRONT_MARK(1);
   if (try_lean) {
     const LeanMover mv{P.sc.scan_tmp + P.sc.max_jobs + 1, P.sc.counters};
-    if (lean_step(ix, P.cfg, sch, n_rings, [&](uint32_t r) { return P.rings.r[r]; },
+    if (lean_step(ix, P.cfg, n_rings, [&](uint32_t r) { return P.rings.r[r]; },
                   [&](uint32_t r) { return P.send.r[r]; }, win_head, win_tail, send_off, P.region_base,
                   P.region_bytes, lean_sh, lean_s, nullptr, &mv)) {
       TL_END(P.cfg, TL_FUSED);
       return;
     }
   }
+  for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
+    reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];
+  cta_barrier();
   // ---- K1: each ring in turn by the whole CTA, then dense record numbering (prefix[] in shared memory)
   if (threadIdx.x == 0) prefix[0] = 0;
   for (uint32_t r = 0; r < n_rings; ++r) {

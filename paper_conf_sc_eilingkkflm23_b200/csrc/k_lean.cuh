@@ -91,7 +91,7 @@ struct LeanMover {
   uint32_t* counters;
 };
 template <class RingOf, class SendOf>
-__device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& cfg, const SchemaTable& sch, uint32_t n,
+__device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& cfg, uint32_t n,
                                           RingOf ring_of, SendOf send_of, const uint64_t* head, const uint64_t* tail,
                                           const uint64_t* soff_bell, uint64_t region_base, uint64_t region_bytes,
                                           uint8_t* sh, LeanState& L, crk_server_bell* B, const LeanMover* mover) {
@@ -195,15 +195,9 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       xid = wv[0];
       // RFC 5531 §9: CALL, rpcvers 2, the program and version, zero-length credential and verifier bodies
       good = good && wv[1] == 0 && wv[2] == 2 && wv[3] == cfg.prog && wv[4] == cfg.vers && wv[7] == 0 && wv[9] == 0;
+      // the built-in memcpy procedures (their schemas cannot be re-registered: crk_proc_schema_register)
       const uint32_t proc = wv[5];
-      uint32_t e = 0;  // the procedure's first schema entry must be the built-in memcpy layout
-#pragma unroll 1
-      while (e < sch.n && sch.s[e].proc != proc) ++e;
-      const Schema* s = e < sch.n ? &sch.s[e] : nullptr;
-      const bool h2d = good && s && proc == cfg.proc_h2d && s->n_items == 3 && s->items[0] == CRK_K_U64 &&
-                       s->items[1] == CRK_K_OPAQUE_VAR && s->items[2] == CRK_K_U64;
-      const bool d2h = good && s && proc == cfg.proc_d2h && s->n_items == 2 && s->items[0] == CRK_K_U64 &&
-                       s->items[1] == CRK_K_U64;
+      const bool h2d = good && proc == cfg.proc_h2d, d2h = good && proc == cfg.proc_d2h;
       q.ptr = ((uint64_t)wv[10] << 32) | wv[11];
       q.d2h = d2h;
       good = h2d || d2h;

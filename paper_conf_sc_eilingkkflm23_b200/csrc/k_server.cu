@@ -149,7 +149,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     STEP_MARK(threadIdx.x == 0, 0, 0);
     // ---- a lean step (well-formed memcpy CALLs only), else the general phases
-    if (lean_step(ix, P.cfg, sch, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
+    if (lean_step(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
                   [&](uint32_t r) { return P.send[r]; }, win_head, win_tail, send.off, P.region_base, P.region_bytes,
                   lean_sh, lean_s, B, nullptr)) {
       if (threadIdx.x == 0) {
