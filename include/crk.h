@@ -124,6 +124,13 @@ typedef struct {
                                      fragments in all also takes the fused single-CTA front end for windows past
                                      fused_front_max_window: the index bounds the CTA's header walk (default
                                      4096, e.g. one 256 MiB memcpy CALL in 64 KiB fragments; 0 = off) */
+  uint32_t lean_steps;       /* 1 (default): a persistent-server or fused crk_serve step of well-formed memcpy CALLs
+                                (AUTH_NONE, built-in HtoD / DtoH procedures, distinct xids, all served OK, <= 32
+                                records / 64 KiB of windows and of DtoH replies) is served by one warp over a
+                                shared-memory copy of the windows (DESIGN.md §1 item 22; identical results); any
+                                other step runs the general phases.  0: always the general phases */
+  uint32_t lean_backoff;     /* steps that skip the lean attempt after a step it could not take (default 16;
+                                0: try every step) */
 } crk_config;
 
 typedef struct crk_ctx crk_ctx;

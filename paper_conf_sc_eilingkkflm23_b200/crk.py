@@ -47,7 +47,7 @@ class Config(C.Structure):
                 ("mover_run", C.c_uint32), ("mover_tail_tiles", C.c_uint32), ("mover_reserve_ctas", C.c_uint32),
                 ("fused_front_max_records", C.c_uint32), ("scan_chunking", C.c_uint32), ("fused_front_max_window", C.c_uint64),
                 ("proc_h2d_stripe", C.c_uint32), ("mover_max_ctas", C.c_uint32),
-                ("fused_front_max_frags", C.c_uint32)]
+                ("fused_front_max_frags", C.c_uint32), ("lean_steps", C.c_uint32), ("lean_backoff", C.c_uint32)]
 
 
 class CRing(C.Structure):

@@ -274,6 +274,8 @@ void crk_config_init(crk_config* c) {
   c->fused_front_max_window = 1ull << 20;
   c->fused_front_max_frags = 4096;
   c->proc_h2d_stripe = 3;
+  c->lean_steps = 1;
+  c->lean_backoff = 16;
 }
 
 int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
@@ -285,6 +287,7 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
       cfg.tile_bytes > (1u << 20) || cfg.max_jobs == 0 || cfg.proc_h2d == cfg.proc_d2h || cfg.scan_threads < 64 ||
       cfg.scan_threads > 1024 || (cfg.scan_threads & 63) || cfg.mover_stages < 2 || cfg.mover_stages > 8 ||
       cfg.mover_run < 1 || cfg.mover_run > 64 || cfg.mover_tail_tiles > 64 || cfg.scan_chunking > 1 ||
+      cfg.lean_steps > 1 ||
       (cfg.proc_h2d_stripe && (cfg.proc_h2d_stripe == cfg.proc_h2d || cfg.proc_h2d_stripe == cfg.proc_d2h)))
     return CRK_E_ARG;
   int ndev = 0;
@@ -321,6 +324,8 @@ int crk_ctx_create(int device, const crk_config* cfg_in, crk_ctx** out) {
   d.no_chunked_scan = cfg.scan_chunking == 1 ? 1u : 0u;
   c->sc.pdl = pdl_of(d) ? 1u : 0u;
   d.proc_stripe = cfg.proc_h2d_stripe;
+  d.lean = cfg.lean_steps;
+  d.lean_backoff = cfg.lean_backoff;
   add_builtin(c->host_schemas, cfg.proc_h2d, {CRK_K_U64, CRK_K_OPAQUE_VAR, CRK_K_U64});
   add_builtin(c->host_schemas, cfg.proc_d2h, {CRK_K_U64, CRK_K_U64});
   if (cfg.proc_h2d_stripe)  // ptr, mem, size, parent, offset, total (reading R22)

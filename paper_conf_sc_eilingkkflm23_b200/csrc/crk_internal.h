@@ -155,6 +155,7 @@ struct Scratch {          // ctx-owned device scratch
   Job* jobs;              // [max_jobs]
   Piece* pieces;          // [2 * max_jobs]
   uint32_t* counters;     // [16]: 0/2 mover decode/encode run cursors, 3/6 their single-tile tail cursors, 1 n_jobs,
+                          // 15 the fused front end's lean back-off (steps left before the lean path is tried again),
                           // 4 queue split, 5 K2 block counter, 8/9 mover launch stamp (sequence, start time),
                           // 12 queue-0 runs in run_job, 13 run_job valid for the next mover launch
   uint64_t* lens_pool;    // explicit framing: [2 * max_lens] (lens, then wire starts)
@@ -173,7 +174,10 @@ struct ConfigDev {
   uint32_t scan_threads, stages, run, tail;  // tail: per-CTA single-tile claims at the end of each queue
   uint32_t reserve;         // mover CTAs that run only when the launch found the GPU free (crk_config.mover_reserve_ctas)
   uint32_t no_chunked_scan; // crk_config.scan_chunking == 1: one CTA per ring always
-  uint32_t proc_stripe, pad2_;  // crk_config.proc_h2d_stripe (0: none)
+  uint32_t proc_stripe;     // crk_config.proc_h2d_stripe (0: none)
+  uint32_t lean;            // crk_config.lean_steps
+  uint32_t lean_backoff;    // crk_config.lean_backoff
+  uint32_t pad3_;
   uint64_t max_record_bytes;
   unsigned long long* tl;  // diagnostic timeline build only (-DCRK_TIMELINE): [stage][min start, max end]
 };

@@ -62,7 +62,10 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   // ---- setup: an empty xid table (the schemas are loaded below, for the general phases only)
   for (uint64_t h = threadIdx.x; h <= ix.hash_mask; h += blockDim.x) ix.xid_hash[h] = ~0ull;
   // a serve step over at most kLeanRings rings: its cursors (doorbell or parameters) for the lean path
-  const bool try_lean = P.plan && n_rings <= kLeanRings;
+  // (the context's lean back-off, scratch counter 15: steps left before the lean path is tried again)
+  __shared__ uint32_t lean_skip;
+  if (threadIdx.x == 0) lean_skip = P.sc.counters[15];
+  const bool try_lean = P.cfg.lean && P.plan && n_rings <= kLeanRings;
   if (try_lean && threadIdx.x < n_rings) {
     const uint32_t r = threadIdx.x;
     win_head[r] = P.rings.doorbell ? P.rings.doorbell[r] : P.rings.r[r].head;
@@ -71,7 +74,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
   }
   cta_barrier();
   FRONT_MARK(1);
-  if (try_lean) {
+  if (try_lean && lean_skip == 0) {
     const LeanMover mv{P.sc.scan_tmp + P.sc.max_jobs + 1, P.sc.counters};
     if (lean_step(ix, P.cfg, n_rings, [&](uint32_t r) { return P.rings.r[r]; },
                   [&](uint32_t r) { return P.send.r[r]; }, win_head, win_tail, send_off, P.region_base,
@@ -79,6 +82,9 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
       TL_END(P.cfg, TL_FUSED);
       return;
     }
+    if (threadIdx.x == 0) P.sc.counters[15] = P.cfg.lean_backoff;
+  } else if (try_lean && threadIdx.x == 0) {
+    P.sc.counters[15] = lean_skip - 1;
   }
   for (uint32_t i = threadIdx.x; i < sizeof(SchemaTable) / 4; i += blockDim.x)
     reinterpret_cast<uint32_t*>(&sch)[i] = reinterpret_cast<const uint32_t*>(P.schemas)[i];

@@ -26,6 +26,9 @@ constexpr uint32_t kLeanRecs = 32;          // records: one per lane of warp 0
 constexpr uint32_t kLeanRings = 8;
 constexpr uint64_t kLeanD2H = 64 * 1024;    // DtoH reply data the CTA encodes itself
 constexpr uint32_t kLeanFrags = 128;        // record-marking fragments of the step
+// After a step the lean path could not take, the next crk_config.lean_backoff steps go straight to the general
+// phases (a stream of control calls would otherwise pay the attempt -- the window copy and the warp's checks --
+// every step).
 
 struct LeanRec {
   uint64_t cur, ptr, n, off, c, size;  // header cursor; HtoD dst / DtoH src; bytes copied / DtoH size; reply cursor;

@@ -108,6 +108,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
   crk_server_bell* B = P.bell;
   const IndexDev& ix = P.ix;
   uint64_t seen = B->done_seq;
+  uint32_t lean_skip = 0;  // steps left before the lean path is tried again
   if (threadIdx.x == 0) seq_s = seen;
   cta_barrier();
   for (;;) {
@@ -149,9 +150,16 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (threadIdx.x == 0) B->t_phase_ns[0] = gtimer();
     STEP_MARK(threadIdx.x == 0, 0, 0);
     // ---- a lean step (well-formed memcpy CALLs only), else the general phases
-    if (lean_step(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
-                  [&](uint32_t r) { return P.send[r]; }, win_head, win_tail, send.off, P.region_base, P.region_bytes,
-                  lean_sh, lean_s, B, nullptr)) {
+    bool lean = false;  // (lean_skip is uniform across the CTA: lean_step's answer is)
+    if (P.cfg.lean && lean_skip == 0) {
+      lean = lean_step(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
+                       [&](uint32_t r) { return P.send[r]; }, win_head, win_tail, send.off, P.region_base,
+                       P.region_bytes, lean_sh, lean_s, B, nullptr);
+      if (!lean) lean_skip = P.cfg.lean_backoff;
+    } else if (lean_skip) {
+      --lean_skip;
+    }
+    if (lean) {
       if (threadIdx.x == 0) {
         const uint64_t t = gtimer();
         for (int k = 1; k < 5; ++k) B->t_phase_ns[k] = t;

@@ -190,7 +190,8 @@ def test_mutated_memcpy_streams_lean_boundary(strict, path):
     steps and must hand every mutated one (a flipped byte, a rewritten length, a truncation, garbage, a duplicate
     xid) to the general phases -- results, statuses, reply bytes and destination bytes equal or_serve's."""
     cfg = ocfg(strict=strict, F=1024)
-    ctx = ctx_for(cfg, max_record_bytes=1 << 14, fused_front_max_records=1024, fused_front_max_window=1 << 30)
+    ctx = ctx_for(cfg, max_record_bytes=1 << 14, fused_front_max_records=1024, fused_front_max_window=1 << 30,
+                  lean_backoff=0)  # every step tries the lean path
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
     g = gen.rng(7000 + 2 * strict + (path == "server"))

@@ -217,7 +217,7 @@ def test_lean_steps_match_oracle(mode, host, strict, F):
     the general phases would have written (fragment / record tables vs or_frame_scan, parsed CALLs vs
     or_parse_call, serve decisions vs or_serve)."""
     cfg = ocfg(strict=strict, F=F)
-    ctx = ctx_for(cfg, fused_front_max_records=1024, fused_front_max_window=1 << 30)
+    ctx = ctx_for(cfg, fused_front_max_records=1024, fused_front_max_window=1 << 30, lean_backoff=0)
     n_rings, cap, scap = 3, 1 << 16, 1 << 18
     region_bytes = 1 << 20
     region = torch.zeros(region_bytes, dtype=torch.uint8, device="cuda")
@@ -288,3 +288,35 @@ def test_lean_steps_match_oracle(mode, host, strict, F):
         if srv:
             srv.stop()
     assert lean >= 5, lean  # most steps took the lean path
+
+
+@pytest.mark.parametrize("lean_steps,backoff", [(0, 16), (1, 16)])
+def test_lean_switch_and_backoff(lean_steps, backoff):
+    """crk_config.lean_steps = 0 keeps every step on the general phases; with the back-off, a step the lean path
+    cannot take (a control call) makes the next `backoff` steps skip the attempt, after which it is tried again.
+    Results equal the oracle's either way."""
+    cfg = ocfg(F=4096, user={33: [O.K_U32]})
+    ctx = ctx_for(cfg, lean_steps=lean_steps, lean_backoff=backoff)
+    region = torch.zeros(1 << 16, dtype=torch.uint8, device="cuda")
+    base = region.data_ptr()
+    ring, send = crk.Ring.device(1 << 16), crk.Ring.device(1 << 16)
+    idx = ctx.index(1, 64, 16)
+    data = gen.random_bytes(5, 1000)
+    memcpy = O.encode_call(*h2d_call(1, data, base + 64), cfg)
+    control = O.encode_call(2, 33, [(O.K_U32, 7)], cfg)
+    took = []
+    head = 0
+    for step in range(2 + backoff + 1):
+        w = control if step == 1 else memcpy
+        ring.write(head, w)
+        idx.serve([(ring, head, head + len(w))], [send], [0], base, region.numel())
+        torch.cuda.synchronize()
+        res = idx.ring_results(1)[0]
+        assert res["status"] == O.OK and res["consumed"] == head + len(w)
+        took.append(ctx.debug_counters()[1] == 0)  # the lean path leaves the mover an empty plan
+        head += len(w)
+    assert np.array_equal(region[64:1064].cpu().numpy(), data)
+    if lean_steps == 0:
+        assert not any(took)
+    else:  # lean, the control call (general), `backoff` general steps, lean again
+        assert took == [True, False] + [False] * backoff + [True], took
