@@ -431,8 +431,10 @@ def main():
     runs = {
         "C1": lambda: c1(Ctx()),
         "C1_serve_one_record": lambda: serve_latency(Ctx()),
+        "C1_serve_one_record_general": lambda: serve_latency(crk.Context(0, **{**CTX_KW, "lean_steps": 0})),
         "C2_matrixMul": lambda: c2(Ctx()),
         "NEXT3_server": lambda: server_latency(Ctx()),
+        "NEXT3_server_general": lambda: server_latency(crk.Context(0, **{**CTX_KW, "lean_steps": 0}), reps=500),
         "C3_sweep": lambda: c3(Ctx()),
         "C4_typed_regular": lambda: c4(Ctx(), False),
         "C4_typed_irregular": lambda: c4(Ctx(), True),
