@@ -154,7 +154,11 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
           bool last = false;
 #pragma unroll 1
           while (!last) {
-            const uint32_t h = p + 4 <= tail[r] ? shadow_be32(sh, q.so_, q.sm_, p) : 0u, flen = h & 0x7fffffffu;
+            const uint32_t po = (uint32_t)(p & q.sm_);  // an aligned header is one shared-memory word
+            const uint32_t h = p + 4 > tail[r] ? 0u
+                               : !(po & 3) ? bswap32(*reinterpret_cast<const uint32_t*>(sh + q.so_ + po))
+                                           : shadow_be32(sh, q.so_, q.sm_, p);
+            const uint32_t flen = h & 0x7fffffffu;
             last = h >> 31;
             if (p + 4 > tail[r] || p + 4 + flen > tail[r] || sum + flen > cfg.max_record_bytes ||
                 nf >= ix.frags_per_ring || nfr >= kLeanFrags) { ok = 0; break; }
@@ -338,9 +342,12 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
         if (atomicCAS(ix.xid_hash + h, ~0ull, key) == ~0ull) break;
   }
   STEP_MARK(tid == 0, 26, 0);
-  // ---- HtoD payloads (shadow -> destination) and the framed replies (aligned words into the send rings)
+  // ---- HtoD payloads (shadow -> destination) and the framed replies (aligned words into the send rings): the
+  // CTA's warps split into N teams (one record each, in turn when N does not divide them)
+  const uint32_t nw = blockDim.x >> 5, wpt = N ? max(1u, nw / N) : nw, nteams = nw / wpt;
+  const uint32_t team = warp / wpt, ttid = tid - team * wpt * 32, tn = wpt * 32;
 #pragma unroll 1
-  for (uint32_t d = 0; d < N; ++d) {
+  for (uint32_t d = team; d < N && team < nteams; d += nteams) {
     const LeanRec& q = L.rec[d];
     if (!q.d2h) {  // logical [52, 52 + n) of the record, fragment by fragment
       uint8_t* dst = reinterpret_cast<uint8_t*>(q.ptr) - 52;
@@ -349,14 +356,14 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
         const LeanFrag& f = L.frag[q.f0 + j];
         const uint64_t a = max((uint64_t)f.lstart, (uint64_t)52), b = min((uint64_t)f.lstart + f.len, 52 + q.n);
 #pragma unroll 1
-        for (uint64_t o = a + tid; o < b; o += blockDim.x) dst[o] = sh[q.so_ + ((f.cur + 4 + o - f.lstart) & q.sm_)];
+        for (uint64_t o = a + ttid; o < b; o += tn) dst[o] = sh[q.so_ + ((f.cur + 4 + o - f.lstart) & q.sm_)];
       }
     }
     const RingDesc O = send_of(q.ring);
     const uint8_t* src = reinterpret_cast<const uint8_t*>(q.ptr);
     const uint32_t F = cfg.F;
 #pragma unroll 1
-    for (uint32_t k = tid; k < (q.w >> 2); k += blockDim.x) {
+    for (uint32_t k = ttid; k < (q.w >> 2); k += tn) {
       const uint32_t pos = 4 * k, f = pos / (F + 4), within = pos - f * (F + 4);
       uint32_t v;
       if (within == 0) {  // RFC 5531 §11 fragment header

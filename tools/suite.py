@@ -188,6 +188,12 @@ def server_latency(ctx, reps=2000):
     cur += ctx.encode_call(2, gen.PROC_H2D, [(crk.K_U64, base + MiB), (crk.K_OPAQUE_VAR, b), (crk.K_U64, b.numel())],
                            ring2, cur)
     cur += ctx.encode_call(3, gen.PROC_D2H, [(crk.K_U64, base + 3 * MiB), (crk.K_U64, Cm.nbytes)], ring2, cur)
+    # twelve 4 KiB HtoD CALLs in one step (a server collecting several clients' small calls)
+    ring3 = crk.Ring.device(1 << 16)
+    cur3 = 0
+    for i in range(12):
+        cur3 += ctx.encode_call(100 + i, gen.PROC_H2D, [(crk.K_U64, base + 2 * MiB + 4096 * i), (crk.K_OPAQUE_VAR, data),
+                                                        (crk.K_U64, 4096)], ring3, cur3)
     torch.cuda.synchronize()
     srv = crk.Server(idx, [ring], [send], base, region.numel())
     try:
@@ -223,6 +229,17 @@ def server_latency(ctx, reps=2000):
     finally:
         srv2.stop()
     ok2 &= bool(torch.equal(region[:a.numel()], a))
+    srv3 = crk.Server(ctx.index(1, 64, 16), [ring3], [send], base, region.numel())
+    try:
+        m12 = []
+        for i in range(200):
+            out3 = srv3.step([(0, cur3)], [0])
+            m12.append(out3["device_ns"])
+        ok3 = out3["results"][0]["status"] == 0 and out3["results"][0]["n_records"] == 12
+    finally:
+        srv3.stop()
+    ok3 &= all(bool(torch.equal(region[2 * MiB + 4096 * i:2 * MiB + 4096 * (i + 1)], data)) for i in range(12))
+    t12 = float(np.median(m12))
     return {"one_record_c_roundtrip_us_median": round(float(np.median(crt)) / 1e3, 2),
             "one_record_c_roundtrip_us_p99": round(float(np.percentile(crt, 99)) / 1e3, 2),
             "one_record_roundtrip_us_median": round(float(np.median(rt)) / 1e3, 2),
@@ -230,7 +247,9 @@ def server_latency(ctx, reps=2000):
             "one_record_roundtrip_us_p99": round(float(np.percentile(rt, 99)) / 1e3, 2), "ok": bool(ok),
             "one_record_phase_end_us_median": dict(zip(("setup", "scan", "parse", "plan", "move"),
                                                       [round(float(x) / 1e3, 2) for x in np.median(ph, axis=0)])),
-            "c2_batch_device_us_median": round(float(np.median(c2dv)) / 1e3, 2), "c2_ok": bool(ok2)}
+            "c2_batch_device_us_median": round(float(np.median(c2dv)) / 1e3, 2), "c2_ok": bool(ok2),
+            "twelve_4KiB_calls_device_us_median": round(t12 / 1e3, 2),
+            "twelve_4KiB_calls_gbs": round(12 * 4096 / t12, 2), "twelve_ok": bool(ok3)}
 
 
 def c2(ctx):
