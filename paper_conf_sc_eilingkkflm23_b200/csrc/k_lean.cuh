@@ -122,9 +122,18 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     const uint32_t nch = (uint32_t)((((tail[r] + 15) & ~15ull) - a) >> 4);
     const RingDesc R = ring_of(r);
 #pragma unroll 1
-    for (uint32_t i = tid; i < nch; i += blockDim.x) {
-      const uint64_t cur = a + 16ull * i;
-      *reinterpret_cast<uint4*>(sh + L.soff[r] + (uint32_t)(cur & L.smask[r])) = ld16_stream(R.base + (cur & R.mask));
+    for (uint32_t i0 = 0; i0 < nch; i0 += 4 * blockDim.x) {  // up to four loads in flight per thread
+      uint4 v[4];
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u) {
+        const uint32_t i = i0 + u * blockDim.x + tid;
+        if (i < nch) v[u] = ld16_stream(R.base + ((a + 16ull * i) & R.mask));
+      }
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u) {
+        const uint32_t i = i0 + u * blockDim.x + tid;
+        if (i < nch) *reinterpret_cast<uint4*>(sh + L.soff[r] + (uint32_t)((a + 16ull * i) & L.smask[r])) = v[u];
+      }
     }
   }
   cta_barrier();

@@ -27,8 +27,11 @@ ctx = crk.Context(0)
 region = torch.zeros(1 << 22, dtype=torch.uint8, device=dev)
 base = region.data_ptr()
 data = torch.from_numpy(gen.random_bytes(0xC1, 4096)).to(dev)
-ring = crk.Ring.device(1 << 14)
-w = ctx.encode_call(7, gen.PROC_H2D, [(crk.K_U64, base + 4096), (crk.K_OPAQUE_VAR, data), (crk.K_U64, 4096)], ring, 0)
+ring = crk.Ring.device(1 << 16)
+w = 0
+for i in range(int(os.environ.get("CALLS", "1"))):  # CALLS=12: a step of twelve 4 KiB HtoD calls
+    w += ctx.encode_call(7 + i, gen.PROC_H2D, [(crk.K_U64, base + 4096 * (i + 1)), (crk.K_OPAQUE_VAR, data),
+                                              (crk.K_U64, 4096)], ring, w)
 send = crk.Ring.device(1 << 16)
 idx = ctx.index(1, 64, 16)
 torch.cuda.synchronize()
