@@ -364,8 +364,21 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       for (uint32_t j = 0; j < q.nf; ++j) {
         const LeanFrag& f = L.frag[q.f0 + j];
         const uint64_t a = max((uint64_t)f.lstart, (uint64_t)52), b = min((uint64_t)f.lstart + f.len, 52 + q.n);
+        // whole destination words where the segment covers them (four shared-memory bytes gathered per word, any
+        // source alignment), single bytes at the two ends
+        const uint64_t sb = f.cur + 4 - f.lstart, da = q.ptr - 52;  // shadow cursor / address of logical offset 0
+        const uint64_t w0 = min(b, (da + a + 3) / 4 * 4 - da), w1 = max(w0, (da + b) / 4 * 4 - da);
 #pragma unroll 1
-        for (uint64_t o = a + ttid; o < b; o += tn) dst[o] = sh[q.so_ + ((f.cur + 4 + o - f.lstart) & q.sm_)];
+        for (uint64_t o = a + ttid; o < w0; o += tn) dst[o] = sh[q.so_ + ((sb + o) & q.sm_)];
+#pragma unroll 1
+        for (uint64_t o = w0 + 4 * ttid; o < w1; o += 4 * tn) {
+          uint32_t v = 0;
+#pragma unroll
+          for (uint32_t k = 0; k < 4; ++k) v |= (uint32_t)sh[q.so_ + ((sb + o + k) & q.sm_)] << (8 * k);
+          *reinterpret_cast<uint32_t*>(dst + o) = v;
+        }
+#pragma unroll 1
+        for (uint64_t o = w1 + ttid; o < b; o += tn) dst[o] = sh[q.so_ + ((sb + o) & q.sm_)];
       }
     }
     const RingDesc O = send_of(q.ring);
