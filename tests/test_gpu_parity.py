@@ -762,10 +762,13 @@ def test_staged_e2e_path_matches_oracle():
     assert np.array_equal(region.cpu().numpy(), host_region)
 
 
-def test_serve_graph_replays_with_doorbell_cursors():
-    """A captured serve step replayed over successive windows of the same ring == the oracle per window."""
+@pytest.mark.parametrize("shape,out0", [((4096, 256), 5), ((64, 16), 8)])
+def test_serve_graph_replays_with_doorbell_cursors(shape, out0):
+    """A captured serve step replayed over successive windows of the same ring == the oracle per window.  The
+    small index with an aligned send cursor takes the fused front end's lean path, its cursors read from the
+    doorbell at replay time (the mover then finds an empty plan)."""
     cfg = ocfg(F=4096)
-    ctx = ctx_for(cfg)
+    ctx = ctx_for(cfg, lean_backoff=0)
     region = torch.zeros(1 << 20, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
     host_region = np.zeros(1 << 20, np.uint8)
@@ -773,11 +776,11 @@ def test_serve_graph_replays_with_doorbell_cursors():
     region.copy_(torch.from_numpy(host_region))
     ring = make_ring(1 << 16)
     send = make_ring(1 << 17)
-    idx = ctx.index(1, 4096, 256)
+    idx = ctx.index(1, *shape)
     bell = crk.HostBuffer(3 * 8)
     cells = bell.np.view(np.uint64)
     graph = idx.serve_graph([ring], [send], base, region.numel(), bell)
-    head, out = 60000, 5
+    head, out = 60000, out0
     for batch in range(4):
         wires = []
         for i in range(3):
@@ -800,6 +803,8 @@ def test_serve_graph_replays_with_doorbell_cursors():
         n = want["reply_bytes"][0]
         assert send.read(out, n) == bytes(want["send"][0][out:out + n])
         assert np.array_equal(region.cpu().numpy(), host_region)
+        if out0 % 4 == 0:
+            assert ctx.debug_counters()[1] == 0  # the lean path served it
         head, out = tail, out + n
     cells[:] = [10, 5, 0]  # invalid window: E_ARG, nothing served
     graph.launch()
