@@ -385,26 +385,38 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     const uint8_t* src = reinterpret_cast<const uint8_t*>(q.ptr);
     const uint32_t F = cfg.F;
 #pragma unroll 1
-    for (uint32_t k = ttid; k < (q.w >> 2); k += tn) {
-      const uint32_t pos = 4 * k, f = pos / (F + 4), within = pos - f * (F + 4);
-      uint32_t v;
-      if (within == 0) {  // RFC 5531 §11 fragment header
-        const uint32_t flen = min(F, q.Ll - f * F);
-        v = flen | ((f * F + flen == q.Ll) ? 0x80000000u : 0u);
-      } else {  // REPLY: xid, REPLY 1, MSG_ACCEPTED 0, AUTH_NONE 0 / 0, SUCCESS 0, err 0, [DtoH: n, data, pad]
-        const uint32_t l0 = f * F + within - 4;
-        if (l0 < (q.d2h ? 32u : 28u)) {
-          v = l0 == 0 ? q.xid : l0 == 4 ? 1u : l0 == 28 ? (uint32_t)q.n : 0u;
-        } else {
-          v = 0;
+    // four words per thread per pass, every source load of the pass issued before any store (the send ring and
+    // the source may alias as far as the compiler knows, so it would not reorder them itself)
+    const uint32_t nwords = q.w >> 2;
 #pragma unroll 1
-          for (uint32_t j = 0; j < 4; ++j) {
-            const uint64_t di = l0 + j - 32;
-            v = (v << 8) | (di < q.n ? src[di] : 0u);
+    for (uint32_t k0 = ttid; k0 < nwords; k0 += 4 * tn) {
+      uint32_t v[4];
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u) {
+        const uint32_t k = k0 + u * tn, pos = 4 * k, f = pos / (F + 4), within = pos - f * (F + 4);
+        v[u] = 0;
+        if (k >= nwords) continue;
+        if (within == 0) {  // RFC 5531 §11 fragment header
+          const uint32_t flen = min(F, q.Ll - f * F);
+          v[u] = flen | ((f * F + flen == q.Ll) ? 0x80000000u : 0u);
+        } else {  // REPLY: xid, REPLY 1, MSG_ACCEPTED 0, AUTH_NONE 0 / 0, SUCCESS 0, err 0, [DtoH: n, data, pad]
+          const uint32_t l0 = f * F + within - 4;
+          if (l0 < (q.d2h ? 32u : 28u)) {
+            v[u] = l0 == 0 ? q.xid : l0 == 4 ? 1u : l0 == 28 ? (uint32_t)q.n : 0u;
+          } else {
+#pragma unroll
+            for (uint32_t j = 0; j < 4; ++j) {
+              const uint64_t di = l0 + j - 32;
+              v[u] = (v[u] << 8) | (di < q.n ? src[di] : 0u);
+            }
           }
         }
       }
-      *reinterpret_cast<uint32_t*>(O.base + ((q.off + pos) & O.mask)) = bswap32(v);
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u) {
+        const uint32_t k = k0 + u * tn;
+        if (k < nwords) *reinterpret_cast<uint32_t*>(O.base + ((q.off + 4 * k) & O.mask)) = bswap32(v[u]);
+      }
     }
   }
   STEP_MARK(tid == 0, 31, 0);
