@@ -93,7 +93,7 @@ struct LeanMover {
   uint64_t* total_tiles;  // the mover's plan (Scratch::scan_tmp[max_jobs + 1], counters)
   uint32_t* counters;
 };
-template <class RingOf, class SendOf>
+template <bool kRunWalk, class RingOf, class SendOf>
 __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& cfg, uint32_t n,
                                           RingOf ring_of, SendOf send_of, const uint64_t* head, const uint64_t* tail,
                                           const uint64_t* soff_bell, uint64_t region_base, uint64_t region_bytes,
@@ -141,55 +141,147 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
   // ---- warp 0: the chains, the records' checks and serve decisions, the reply offsets
   if (warp == 0) {
     uint32_t ok = 1, nrec = 0;
-    if (lane == 0) {  // RFC 5531 §11 chains: whole records (up to a last fragment) inside the window, in capacity
+    if constexpr (kRunWalk) {
+      // RFC 5531 §11 chains: whole records (up to a last fragment) inside the window, in capacity.  The warp walks
+      // them together: a run of identical single-fragment records is verified at once (lane k reads the header k
+      // records ahead; every header before the first mismatch is a true one), anything else -- a multi-fragment
+      // record, every failing check -- goes one record at a time through lane 0.  State is warp-uniform.
       uint32_t nfr = 0;
 #pragma unroll 1
       for (uint32_t r = 0; r < n && ok; ++r) {
-        L.prefix[r] = nrec;
+        if (lane == 0) L.prefix[r] = nrec;
+        const uint32_t so = L.soff[r], sm = L.smask[r];
+        auto hdr_at = [&](uint64_t c) -> uint32_t {  // an aligned header is one shared-memory word
+          const uint32_t po = (uint32_t)(c & sm);
+          return !(po & 3) ? bswap32(*reinterpret_cast<const uint32_t*>(sh + so + po)) : shadow_be32(sh, so, sm, c);
+        };
         uint64_t p = head[r];
         uint32_t nr = 0, nf = 0;
 #pragma unroll 1
         while (ok && p < tail[r]) {
-          if (nrec >= kLeanRecs || nr >= ix.recs_per_ring) { ok = 0; break; }
-          LeanRec& q = L.rec[nrec];
-          q.cur = p;
-          q.ring = r;
-          q.slot = nr;
-          q.so_ = L.soff[r];
-          q.sm_ = L.smask[r];
-          q.f0 = nfr;
-          q.fslot = nf;
-          uint64_t sum = 0;
-          bool last = false;
-#pragma unroll 1
-          while (!last) {
-            const uint32_t po = (uint32_t)(p & q.sm_);  // an aligned header is one shared-memory word
-            const uint32_t h = p + 4 > tail[r] ? 0u
-                               : !(po & 3) ? bswap32(*reinterpret_cast<const uint32_t*>(sh + q.so_ + po))
-                                           : shadow_be32(sh, q.so_, q.sm_, p);
-            const uint32_t flen = h & 0x7fffffffu;
-            last = h >> 31;
-            if (p + 4 > tail[r] || p + 4 + flen > tail[r] || sum + flen > cfg.max_record_bytes ||
-                nf >= ix.frags_per_ring || nfr >= kLeanFrags) { ok = 0; break; }
-            L.frag[nfr++] = LeanFrag{p, flen, (uint32_t)sum};
-            ++nf;
-            sum += flen;
-            p += 4 + flen;
+          const uint32_t h0 = p + 4 <= tail[r] ? hdr_at(p) : 0u, len0 = h0 & 0x7fffffffu;
+          uint32_t m = 0;
+          if ((h0 >> 31) && p + 4 + len0 < tail[r]) {  // (a window's last record takes the one-record path)
+            const uint64_t stride = 4 + (uint64_t)len0, qk = p + lane * stride;
+            const bool okk = qk + stride <= tail[r] && len0 <= cfg.max_record_bytes && nrec + lane < kLeanRecs &&
+                             nr + lane < ix.recs_per_ring && nf + lane < ix.frags_per_ring && nfr + lane < kLeanFrags &&
+                             (lane == 0 || hdr_at(qk) == h0);
+            const uint32_t bad = __ballot_sync(0xffffffffu, !okk);
+            m = bad ? __ffs(bad) - 1 : 32u;
+            if (lane < m) {
+              LeanRec& q = L.rec[nrec + lane];
+              q.cur = qk;
+              q.ring = r;
+              q.slot = nr + lane;
+              q.so_ = so;
+              q.sm_ = sm;
+              q.f0 = nfr + lane;
+              q.fslot = nf + lane;
+              q.len = len0;
+              q.nf = 1;
+              L.frag[nfr + lane] = LeanFrag{qk, len0, 0u};
+            }
+            p += m * stride;
+            nrec += m;
+            nr += m;
+            nf += m;
+            nfr += m;
           }
-          if (!ok) break;
-          q.len = (uint32_t)sum;
-          q.nf = nfr - q.f0;
-          ++nrec;
-          ++nr;
+          if (m) continue;
+          if (lane == 0) {  // one record, fragment by fragment
+            if (nrec >= kLeanRecs || nr >= ix.recs_per_ring) ok = 0;
+            LeanRec& q = L.rec[nrec < kLeanRecs ? nrec : 0];
+            const uint32_t f0 = nfr, fs0 = nf;
+            uint64_t sum = 0, p0 = p;
+            bool last = false;
+#pragma unroll 1
+            while (ok && !last) {
+              const uint32_t h = p + 4 <= tail[r] ? hdr_at(p) : 0u, flen = h & 0x7fffffffu;
+              last = h >> 31;
+              if (p + 4 > tail[r] || p + 4 + flen > tail[r] || sum + flen > cfg.max_record_bytes ||
+                  nf >= ix.frags_per_ring || nfr >= kLeanFrags) { ok = 0; break; }
+              L.frag[nfr++] = LeanFrag{p, flen, (uint32_t)sum};
+              ++nf;
+              sum += flen;
+              p += 4 + flen;
+            }
+            if (ok) {
+              q.cur = p0;
+              q.ring = r;
+              q.slot = nr;
+              q.so_ = so;
+              q.sm_ = sm;
+              q.f0 = f0;
+              q.fslot = fs0;
+              q.len = (uint32_t)sum;
+              q.nf = nfr - f0;
+              ++nrec;
+              ++nr;
+            }
+          }
+          ok = __shfl_sync(0xffffffffu, ok, 0);
+          p = __shfl_sync(0xffffffffu, p, 0);
+          nrec = __shfl_sync(0xffffffffu, nrec, 0);
+          nr = __shfl_sync(0xffffffffu, nr, 0);
+          nf = __shfl_sync(0xffffffffu, nf, 0);
+          nfr = __shfl_sync(0xffffffffu, nfr, 0);
         }
-        L.fcount[r] = nf;
+        if (lane == 0) L.fcount[r] = nf;
       }
-      L.prefix[n] = nrec;
-      STEP_MARK(true, 22, nrec);
+      if (lane == 0) L.prefix[n] = nrec;
+      STEP_MARK(lane == 0, 22, nrec);
+      __syncwarp();
+    } else {  // lane 0 alone, record by record (a single-call step's shortest path; the fused front end)
+      if (lane == 0) {  // RFC 5531 §11 chains: whole records (up to a last fragment) inside the window, in capacity
+        uint32_t nfr = 0;
+#pragma unroll 1
+        for (uint32_t r = 0; r < n && ok; ++r) {
+          L.prefix[r] = nrec;
+          uint64_t p = head[r];
+          uint32_t nr = 0, nf = 0;
+#pragma unroll 1
+          while (ok && p < tail[r]) {
+            if (nrec >= kLeanRecs || nr >= ix.recs_per_ring) { ok = 0; break; }
+            LeanRec& q = L.rec[nrec];
+            q.cur = p;
+            q.ring = r;
+            q.slot = nr;
+            q.so_ = L.soff[r];
+            q.sm_ = L.smask[r];
+            q.f0 = nfr;
+            q.fslot = nf;
+            uint64_t sum = 0;
+            bool last = false;
+#pragma unroll 1
+            while (!last) {
+              const uint32_t po = (uint32_t)(p & q.sm_);  // an aligned header is one shared-memory word
+              const uint32_t h = p + 4 > tail[r] ? 0u
+                                 : !(po & 3) ? bswap32(*reinterpret_cast<const uint32_t*>(sh + q.so_ + po))
+                                             : shadow_be32(sh, q.so_, q.sm_, p);
+              const uint32_t flen = h & 0x7fffffffu;
+              last = h >> 31;
+              if (p + 4 > tail[r] || p + 4 + flen > tail[r] || sum + flen > cfg.max_record_bytes ||
+                  nf >= ix.frags_per_ring || nfr >= kLeanFrags) { ok = 0; break; }
+              L.frag[nfr++] = LeanFrag{p, flen, (uint32_t)sum};
+              ++nf;
+              sum += flen;
+              p += 4 + flen;
+            }
+            if (!ok) break;
+            q.len = (uint32_t)sum;
+            q.nf = nfr - q.f0;
+            ++nrec;
+            ++nr;
+          }
+          L.fcount[r] = nf;
+        }
+        L.prefix[n] = nrec;
+        STEP_MARK(true, 22, nrec);
+      }
+      ok = __shfl_sync(0xffffffffu, ok, 0);
+      nrec = __shfl_sync(0xffffffffu, nrec, 0);
+      __syncwarp();
     }
-    ok = __shfl_sync(0xffffffffu, ok, 0);
-    nrec = __shfl_sync(0xffffffffu, nrec, 0);
-    __syncwarp();
     bool good = true;
     uint32_t xid = lane, ring = 0, w = 0;
     uint64_t d2h_bytes = 0;

@@ -152,7 +152,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     // ---- a lean step (well-formed memcpy CALLs only), else the general phases
     bool lean = false;  // (lean_skip is uniform across the CTA: lean_step's answer is)
     if (P.cfg.lean && lean_skip == 0) {
-      lean = lean_step(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
+      lean = lean_step<true>(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
                        [&](uint32_t r) { return P.send[r]; }, win_head, win_tail, send.off, P.region_base,
                        P.region_bytes, lean_sh, lean_s, B, nullptr);
       if (!lean) lean_skip = P.cfg.lean_backoff;
