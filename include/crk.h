@@ -173,7 +173,7 @@ typedef struct {
   uint64_t* p_value;      /* U32/U64 scalar value */
   int32_t* serve_status;  /* serve only: final per-record status (wire, E_XID, E_SIZE, E_PTR) */
   int32_t* serve_reply_err;/* serve only: -1 no reply, 0 / 1 the mem_result discriminant */
-  uint64_t* serve_reply_off;/* serve only: send-ring cursor of the reply */
+  uint64_t* serve_reply_off;/* serve only: send-ring cursor of the reply (0 when the record has none) */
   uint64_t* serve_reply_wire;
   crk_ring_result* ring_results; /* [max_rings] */
   uint32_t* total_records;       /* device scalar */

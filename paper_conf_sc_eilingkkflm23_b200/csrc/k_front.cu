@@ -78,7 +78,7 @@ __global__ void __launch_bounds__(kFrontThreads, 1) front_small_kernel(FrontPara
     const LeanMover mv{P.sc.scan_tmp + P.sc.max_jobs + 1, P.sc.counters};
     if (lean_step<false>(ix, P.cfg, n_rings, [&](uint32_t r) { return P.rings.r[r]; },
                   [&](uint32_t r) { return P.send.r[r]; }, win_head, win_tail, send_off, P.region_base,
-                  P.region_bytes, lean_sh, lean_s, nullptr, &mv)) {
+                  P.region_bytes, lean_sh, lean_s, nullptr, &mv, nullptr)) {
       TL_END(P.cfg, TL_FUSED);
       return;
     }

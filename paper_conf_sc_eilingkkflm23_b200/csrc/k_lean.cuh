@@ -35,6 +35,7 @@ struct LeanRec {
                                        // HtoD opaque count and size argument
   uint32_t len, ring, slot, xid, d2h, Ll, w, so_, sm_;  // len: the record's logical length
   uint32_t f0, nf, fslot;  // its fragments: first in the step's list, count, ring-local number of the first
+  uint32_t proc, ctrl;     // the procedure; ctrl: 1 + its schema entry for a registered (non-memcpy) procedure
 };
 struct LeanFrag {
   uint64_t cur;            // header cursor
@@ -81,6 +82,58 @@ __device__ __forceinline__ uint32_t lean_be32(const uint8_t* sh, const LeanState
   return v;
 }
 
+// The arguments of a registered procedure's CALL from offset 40 (after the fixed-layout head), item by item as the
+// schema lists them (RFC 4506 §4.1 int / unsigned, §4.5 hyper, §4.9-4.13 fixed and variable-length opaque and
+// arrays): true when every item fits in the record, its pad bytes are zero (strict) and nothing follows the last
+// one (strict) -- the parser's checks, all passing.  With `out.kind`, the parsed-item rows at b are written (kind,
+// offset, count, value as the parser writes them).
+struct ItemRows {  // the index's parsed-item columns (by value: no kernel parameter's address is taken)
+  uint32_t* kind;
+  uint64_t *off, *count, *value;
+};
+__device__ __noinline__ bool lean_items(const uint8_t* sh, const LeanState& L, const LeanRec& q, const Schema& s,
+                                        bool strict, ItemRows out, uint64_t b) {
+  uint64_t o = 40;
+#pragma unroll 1
+  for (uint32_t it = 0; it < s.n_items; ++it) {
+    const uint32_t code = s.items[it], kind = code & 0xff, fixed = code >> 8;
+    uint64_t off = o, cnt = 0, val = 0;
+    if (kind == CRK_K_U32) {
+      if (o + 4 > q.len) return false;
+      val = lean_be32(sh, L, q, o);
+      o += 4;
+    } else if (kind == CRK_K_U64) {
+      if (o + 8 > q.len) return false;
+      val = ((uint64_t)lean_be32(sh, L, q, o) << 32) | lean_be32(sh, L, q, o + 4);
+      o += 8;
+    } else {
+      const uint32_t es = elem_size_k(kind);
+      if (!es) return false;
+      uint64_t c = fixed;
+      if (kind == CRK_K_OPAQUE_VAR || (kind >= CRK_K_I32_VAR && kind <= CRK_K_F64_VAR)) {
+        if (o + 4 > q.len) return false;
+        c = lean_be32(sh, L, q, o);
+        o += 4;
+      }
+      const uint64_t bytes = c * es, pn = pad4(bytes);
+      if (o + bytes + pn > q.len) return false;
+#pragma unroll 1
+      for (uint64_t i = 0; strict && i < pn; ++i)
+        if (lean_byte(sh, L, q, o + bytes + i) != 0) return false;
+      off = o;
+      cnt = c;
+      o += bytes + pn;
+    }
+    if (out.kind) {
+      out.kind[b + it] = kind;
+      out.off[b + it] = off;
+      out.count[b + it] = cnt;
+      out.value[b + it] = val;
+    }
+  }
+  return !strict || o == q.len;
+}
+
 __device__ __noinline__ bool region_ok(uint64_t base, uint64_t bytes, uint64_t ptr, uint64_t n) {
   return ptr >= base && n <= bytes && ptr - base <= bytes - n;
 }
@@ -97,7 +150,8 @@ template <bool kRunWalk, class RingOf, class SendOf>
 __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& cfg, uint32_t n,
                                           RingOf ring_of, SendOf send_of, const uint64_t* head, const uint64_t* tail,
                                           const uint64_t* soff_bell, uint64_t region_base, uint64_t region_bytes,
-                                          uint8_t* sh, LeanState& L, crk_server_bell* B, const LeanMover* mover) {
+                                          uint8_t* sh, LeanState& L, crk_server_bell* B, const LeanMover* mover,
+                                          const SchemaTable* sch) {
   const uint32_t tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (n > kLeanRings || (cfg.F & 3) || cfg.F == 0) return false;
   // ---- the windows' shadow layout (thread 0) and their copy into shared memory (every thread)
@@ -291,7 +345,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       const uint64_t b0 = q.cur + 4;  // logical offset 0
       uint32_t wv[14];                // the fixed-layout head (and the DtoH arguments): in the first fragment
       const uint32_t o0 = (uint32_t)(b0 & q.sm_), flen0 = L.frag[q.f0].len;
-      if (flen0 < 52) good = false;
+      if (flen0 < 40) good = false;  // (the memcpy procedures need 52 / 56 bytes there, checked below)
       if (!(o0 & 3) && o0 + 56 <= q.sm_ + 1) {  // aligned and not across the shadow's wrap: 14 independent loads
         const uint32_t* wp = reinterpret_cast<const uint32_t*>(sh + q.so_ + o0);
 #pragma unroll
@@ -308,10 +362,21 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       const bool h2d = good && proc == cfg.proc_h2d, d2h = good && proc == cfg.proc_d2h;
       q.ptr = ((uint64_t)wv[10] << 32) | wv[11];
       q.d2h = d2h;
-      good = h2d || d2h;
+      q.proc = proc;
+      q.ctrl = 0;
+      // (with `sch`) a registered procedure -- a control call: served OK with no reply and nothing to move
+      if (good && !h2d && !d2h && sch && !(cfg.proc_stripe && proc == cfg.proc_stripe)) {
+        uint32_t e = 0;
+#pragma unroll 1
+        while (e < sch->n && sch->s[e].proc != proc) ++e;
+        if (e < sch->n && lean_items(sh, L, q, sch->s[e], cfg.strict, ItemRows{}, 0)) q.ctrl = e + 1;
+      }
+      good = h2d || d2h || q.ctrl;
+      q.Ll = 0;
+      q.n = 0;
       if (h2d) {  // RFC 4506 §4.10 opaque<>: count, bytes, zero pad; then the size hyper; nothing after it
         const uint64_t c = wv[12], pn = pad4(c), o2 = 52 + c + pn;
-        good = o2 + 8 == q.len;
+        good = flen0 >= 52 && o2 + 8 == q.len;
 #pragma unroll 1
         for (uint64_t i = 0; good && cfg.strict && i < pn; ++i) good = lean_byte(sh, L, q, 52 + c + i) == 0;
         const uint64_t size = good ? ((uint64_t)lean_be32(sh, L, q, o2) << 32) | lean_be32(sh, L, q, o2 + 4) : 0;
@@ -327,7 +392,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
         d2h_bytes = q.n;
         q.Ll = (uint32_t)(32 + q.n + pad4(q.n));
       }
-      w = good ? (uint32_t)wire_of(q.Ll, cfg.F) : 0;
+      w = good && !q.ctrl ? (uint32_t)wire_of(q.Ll, cfg.F) : 0;
       q.w = w;
       q.xid = xid;
       good = good && !(soff_bell[ring] & 3);  // replies are written as aligned words
@@ -346,6 +411,12 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
       const uint64_t y = __shfl_up_sync(0xffffffffu, incl, o);
       if (lane >= o) incl += y;
     }
+#ifdef CRK_LEAN_WHY  // diagnostic build only: why a step left the lean path (bell pad: walk ok | bad-lane mask | D2H)
+    if (B && lane == 0)
+      B->pad_ = (ok ? 1u : 0u) | (tot > kLeanD2H ? 2u : 0u) | (nrec << 2) |
+                (__ballot_sync(0xffffffffu, lane < nrec && !good) & 0xffffu) << 16;
+    else if (B) __ballot_sync(0xffffffffu, lane < nrec && !good);
+#endif
     ok = ok && !__any_sync(0xffffffffu, lane < nrec && !good) && tot <= kLeanD2H;
     // reply cursors: per ring, the exclusive prefix of the wire sizes in record order
     const uint64_t excl = incl - (lane < nrec ? w : 0);
@@ -407,31 +478,37 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     ix.p_slot[d] = rs;
     ix.p_ring[d] = q.ring;
     ix.p_xid[d] = q.xid;
-    ix.p_proc[d] = q.d2h ? cfg.proc_d2h : cfg.proc_h2d;
+    ix.p_proc[d] = q.proc;
     ix.p_status[d] = CRK_OK;
-    ix.p_nitems[d] = q.d2h ? 2 : 3;
+    ix.p_nitems[d] = q.ctrl ? sch->s[q.ctrl - 1].n_items : q.d2h ? 2 : 3;
     ix.p_frag0[d] = fs;
     ix.p_nfrags[d] = q.nf;
     ix.p_flen0[d] = L.frag[q.f0].len;
     // items: u64 ptr @40; then DtoH: u64 size @48; HtoD: opaque<> @52 (count c), u64 size after its pad
-    const uint64_t b = (uint64_t)d * kMaxItems, o2 = 52 + q.c + pad4(q.c), size = q.d2h ? q.n : q.size;
-    ix.p_kind[b] = CRK_K_U64;
-    ix.p_off[b] = 40;
-    ix.p_count[b] = 0;
-    ix.p_value[b] = q.ptr;
-    ix.p_kind[b + 1] = q.d2h ? CRK_K_U64 : CRK_K_OPAQUE_VAR;
-    ix.p_off[b + 1] = q.d2h ? 48 : 52;
-    ix.p_count[b + 1] = q.d2h ? 0 : q.c;
-    ix.p_value[b + 1] = q.d2h ? size : 0;
-    if (!q.d2h) {
-      ix.p_kind[b + 2] = CRK_K_U64;
-      ix.p_off[b + 2] = o2;
-      ix.p_count[b + 2] = 0;
-      ix.p_value[b + 2] = size;
+    const uint64_t b = (uint64_t)d * kMaxItems;
+    if (q.ctrl) {
+      const ItemRows rows{ix.p_kind, ix.p_off, ix.p_count, ix.p_value};
+      lean_items(sh, L, q, sch->s[q.ctrl - 1], cfg.strict, rows, b);
+    } else {
+      const uint64_t o2 = 52 + q.c + pad4(q.c), size = q.d2h ? q.n : q.size;
+      ix.p_kind[b] = CRK_K_U64;
+      ix.p_off[b] = 40;
+      ix.p_count[b] = 0;
+      ix.p_value[b] = q.ptr;
+      ix.p_kind[b + 1] = q.d2h ? CRK_K_U64 : CRK_K_OPAQUE_VAR;
+      ix.p_off[b + 1] = q.d2h ? 48 : 52;
+      ix.p_count[b + 1] = q.d2h ? 0 : q.c;
+      ix.p_value[b + 1] = q.d2h ? size : 0;
+      if (!q.d2h) {
+        ix.p_kind[b + 2] = CRK_K_U64;
+        ix.p_off[b + 2] = o2;
+        ix.p_count[b + 2] = 0;
+        ix.p_value[b + 2] = size;
+      }
     }
     ix.s_status[d] = CRK_OK;
-    ix.s_reply_err[d] = 0;
-    ix.s_reply_off[d] = q.off;
+    ix.s_reply_err[d] = q.ctrl ? -1 : 0;  // a control call has no reply
+    ix.s_reply_off[d] = q.ctrl ? 0 : q.off;  // (0 when the record has no reply, as the general phases write)
     ix.s_reply_wire[d] = q.w;
     // distinct xids into the cleared table: the first free slot (a lone record's is its home slot: a plain store)
     const unsigned long long key = ((unsigned long long)q.xid << 32) | d;
@@ -450,7 +527,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
 #pragma unroll 1
   for (uint32_t d = team; d < N && team < nteams; d += nteams) {
     const LeanRec& q = L.rec[d];
-    if (!q.d2h) {  // logical [52, 52 + n) of the record, fragment by fragment
+    if (!q.d2h && !q.ctrl) {  // logical [52, 52 + n) of the record, fragment by fragment
       uint8_t* dst = reinterpret_cast<uint8_t*>(q.ptr) - 52;
 #pragma unroll 1
       for (uint32_t j = 0; j < q.nf; ++j) {

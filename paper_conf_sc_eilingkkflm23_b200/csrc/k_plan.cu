@@ -145,8 +145,9 @@ __global__ void serve_plan2_kernel(IndexDev ix, ConfigDev cfg, Scratch sc, SendR
     const uint32_t first = ix.rec_prefix[ring], end = ix.rec_prefix[ring + 1];
     const uint64_t w = ix.s_reply_wire[d];
     const uint64_t off = (S.doorbell ? S.doorbell[2 * S.n_rings + ring] : S.off[ring]) + (pre[d] - pre[first]);
-    ix.s_reply_off[d] = off;
-    sc.jobs[total + d] = serve_reply_job(ix, cfg, sc, d, ring, ix.s_reply_err[d], off, w);
+    const int32_t err = ix.s_reply_err[d];
+    ix.s_reply_off[d] = err >= 0 ? off : 0;  // (the oracle's convention: 0 when the record has no reply)
+    sc.jobs[total + d] = serve_reply_job(ix, cfg, sc, d, ring, err, off, w);
     if (d + 1 == end) ix.res[ring].reply_bytes = pre[d] + w - pre[first];
   }
 }

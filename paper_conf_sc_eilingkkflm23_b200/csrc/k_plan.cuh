@@ -382,7 +382,7 @@ __device__ void plan_small_impl(const IndexDev& ix, const ConfigDev& cfg, const 
     ix.s_status[d] = st;
     ix.s_reply_err[d] = err;
     ix.s_reply_wire[d] = w;
-    ix.s_reply_off[d] = off;
+    ix.s_reply_off[d] = err >= 0 ? off : 0;  // (the oracle's convention: 0 when the record has no reply)
     enc = serve_reply_job(ix, cfg, sc, d, ring, err, off, w);
     sc.jobs[d] = dec;
     sc.jobs[total + d] = enc;

@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(kServerThreads, 1) server_kernel(ServerParams 
     if (P.cfg.lean && lean_skip == 0) {
       lean = lean_step<true>(ix, P.cfg, P.n_rings, [&](uint32_t r) { return P.rings[r]; },
                        [&](uint32_t r) { return P.send[r]; }, win_head, win_tail, send.off, P.region_base,
-                       P.region_bytes, lean_sh, lean_s, B, nullptr);
+                       P.region_bytes, lean_sh, lean_s, B, nullptr, &sch);
       if (!lean) lean_skip = P.cfg.lean_backoff;
     } else if (lean_skip) {
       --lean_skip;

@@ -122,3 +122,19 @@ def test_config_rejects_unknown_fields(L):
     with pytest.raises(KeyError):
         crk.config(mover_reserve=16)  # misspelt: the field is mover_reserve_ctas
     assert crk.config(mover_reserve_ctas=16).mover_reserve_ctas == 16
+
+
+def test_one_cta_kernels_keep_a_small_stack(L):
+    """The small-step kernels (persistent server, fused front end) run one CTA whose latency is the product: taking a
+    kernel parameter's address (or passing a big struct to an out-of-line helper) copies it to local memory in every
+    thread at entry, which cost the front end ~80 us per launch once.  Their frames stay under 1 KiB; no kernel
+    spills registers to local memory."""
+    import shutil
+    import subprocess
+    tool = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    out = subprocess.run([tool, "-res-usage", crk.LIBPATH], capture_output=True, text=True).stdout
+    usage = re.findall(r"Function (\S+):\s*\n\s*REG:(\d+) STACK:(\d+) SHARED:\d+ LOCAL:(\d+)", out)
+    assert len(usage) >= 10, out[:400]
+    small = {n: int(st) for n, _, st, _ in usage if "server_kernel" in n or "front_small_kernel" in n}
+    assert len(small) >= 2 and all(v < 1024 for v in small.values()), small
+    assert all(int(loc) == 0 for _, _, _, loc in usage), [u for u in usage if int(u[3])]

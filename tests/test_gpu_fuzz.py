@@ -189,7 +189,7 @@ def test_mutated_memcpy_streams_lean_boundary(strict, path):
     quarter of them unmutated: the lean path of the persistent server / the fused front end takes the well-formed
     steps and must hand every mutated one (a flipped byte, a rewritten length, a truncation, garbage, a duplicate
     xid) to the general phases -- results, statuses, reply bytes and destination bytes equal or_serve's."""
-    cfg = ocfg(strict=strict, F=1024)
+    cfg = ocfg(strict=strict, F=1024, user={40: [O.K_U32, O.K_OPAQUE_VAR]})
     ctx = ctx_for(cfg, max_record_bytes=1 << 14, fused_front_max_records=1024, fused_front_max_window=1 << 30,
                   lean_backoff=0)  # every step tries the lean path
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
@@ -212,8 +212,9 @@ def test_mutated_memcpy_streams_lean_boundary(strict, path):
             distinct = bool(g.integers(0, 8))
             clean = not g.integers(0, 4)
             for r in range(4):
-                w = stream(g, cfg, base, int(g.choice([64, 256, 1024, 1 << 16])), 8 * r, memcpy_only=True,
-                           distinct=distinct)
+                # (the persistent server's lean path also takes control calls of registered procedures)
+                w = stream(g, cfg, base, int(g.choice([64, 256, 1024, 1 << 16])), 8 * r,
+                           memcpy_only=path != "server", distinct=distinct)
                 wire = b"".join(bytes(x) for x in w) if clean else mutate(g, w)
                 rings[r].write(heads[r], wire)
                 tails[r] = heads[r] + len(wire)

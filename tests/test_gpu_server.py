@@ -216,7 +216,7 @@ def test_lean_steps_match_oracle(mode, host, strict, F):
     results, reply bytes (framed with F, here smaller than most replies), destination bytes, and the index tables
     the general phases would have written (fragment / record tables vs or_frame_scan, parsed CALLs vs
     or_parse_call, serve decisions vs or_serve)."""
-    cfg = ocfg(strict=strict, F=F)
+    cfg = ocfg(strict=strict, F=F, user={33: [O.K_U32, O.K_I32_VAR], 34: [O.K_U64, O.K_OPAQUE_FIX | (13 << 8)]})
     ctx = ctx_for(cfg, fused_front_max_records=1024, fused_front_max_window=1 << 30, lean_backoff=0)
     n_rings, cap, scap = 3, 1 << 16, 1 << 18
     region_bytes = 1 << 20
@@ -240,7 +240,15 @@ def test_lean_steps_match_oracle(mode, host, strict, F):
                 wire = b""
                 for i in range(int(g.integers(0, 5))):
                     xid = (step << 16) | (r << 8) | i
-                    if g.integers(0, 2):  # HtoD to a private slot of the lower half, any alignment
+                    k = int(g.integers(0, 5 if mode == "server" else 4))
+                    if k == 4:  # a control call (the server's lean path takes registered procedures too)
+                        if g.integers(0, 2):
+                            c = (xid, 33, [(O.K_U32, int(g.integers(0, 1 << 32))),
+                                           (O.K_I32_VAR, gen.random_elems(g, np.int32, int(g.integers(0, 40))))])
+                        else:
+                            c = (xid, 34, [(O.K_U64, int(g.integers(0, 1 << 62))),
+                                           (O.K_OPAQUE_FIX, gen.random_bytes(xid & 0xFFFF, 13).tobytes())])
+                    elif k < 2:  # HtoD to a private slot of the lower half, any alignment
                         data = gen.random_bytes((step * 7 + r * 3 + i) & 0xFFFF, int(g.integers(0, 2500)))
                         c = h2d_call(xid, data, base + (r * 4 + i) * 4096 + int(g.integers(0, 64)))
                     else:  # DtoH from the upper half

@@ -194,6 +194,12 @@ def server_latency(ctx, reps=2000):
     for i in range(12):
         cur3 += ctx.encode_call(100 + i, gen.PROC_H2D, [(crk.K_U64, base + 2 * MiB + 4096 * i), (crk.K_OPAQUE_VAR, data),
                                                         (crk.K_U64, 4096)], ring3, cur3)
+    # one control call of a registered procedure (a kernel launch's handle, grid size and a 64-byte parameter block)
+    ctx.register_schema(60, [crk.K_U64, crk.K_U32, crk.K_U32, crk.K_OPAQUE_VAR])
+    ring4 = crk.Ring.device(1 << 12)
+    params = torch.from_numpy(gen.random_bytes(0x60, 64)).to(dev)
+    cur4 = ctx.encode_call(9, 60, [(crk.K_U64, 0x7F00DEADBEEF), (crk.K_U32, 148), (crk.K_U32, 256),
+                                   (crk.K_OPAQUE_VAR, params)], ring4, 0)
     torch.cuda.synchronize()
     srv = crk.Server(idx, [ring], [send], base, region.numel())
     try:
@@ -239,6 +245,15 @@ def server_latency(ctx, reps=2000):
     finally:
         srv3.stop()
     ok3 &= all(bool(torch.equal(region[2 * MiB + 4096 * i:2 * MiB + 4096 * (i + 1)], data)) for i in range(12))
+    srv4 = crk.Server(ctx.index(1, 64, 16), [ring4], [send], base, region.numel())
+    try:
+        mc = []
+        for i in range(500):
+            out4 = srv4.step([(0, cur4)], [0])
+            mc.append(out4["device_ns"])
+        ok4 = out4["results"][0]["status"] == 0 and out4["results"][0]["n_records"] == 1
+    finally:
+        srv4.stop()
     t12 = float(np.median(m12))
     return {"one_record_c_roundtrip_us_median": round(float(np.median(crt)) / 1e3, 2),
             "one_record_c_roundtrip_us_p99": round(float(np.percentile(crt, 99)) / 1e3, 2),
@@ -249,7 +264,8 @@ def server_latency(ctx, reps=2000):
                                                       [round(float(x) / 1e3, 2) for x in np.median(ph, axis=0)])),
             "c2_batch_device_us_median": round(float(np.median(c2dv)) / 1e3, 2), "c2_ok": bool(ok2),
             "twelve_4KiB_calls_device_us_median": round(t12 / 1e3, 2),
-            "twelve_4KiB_calls_gbs": round(12 * 4096 / t12, 2), "twelve_ok": bool(ok3)}
+            "twelve_4KiB_calls_gbs": round(12 * 4096 / t12, 2), "twelve_ok": bool(ok3),
+            "control_call_device_us_median": round(float(np.median(mc)) / 1e3, 2), "control_ok": bool(ok4)}
 
 
 def c2(ctx):
