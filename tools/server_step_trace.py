@@ -29,7 +29,11 @@ base = region.data_ptr()
 data = torch.from_numpy(gen.random_bytes(0xC1, 4096)).to(dev)
 ring = crk.Ring.device(1 << 16)
 w = 0
-for i in range(int(os.environ.get("CALLS", "1"))):  # CALLS=12: a step of twelve 4 KiB HtoD calls
+if os.environ.get("CONTROL") == "1":  # one control call of a registered procedure instead (suite.py's)
+    ctx.register_schema(60, [crk.K_U64, crk.K_U32, crk.K_U32, crk.K_OPAQUE_VAR])
+    w = ctx.encode_call(9, 60, [(crk.K_U64, 0x7F00DEADBEEF), (crk.K_U32, 148), (crk.K_U32, 256),
+                                (crk.K_OPAQUE_VAR, data[:64])], ring, 0)
+for i in range(0 if w else int(os.environ.get("CALLS", "1"))):  # CALLS=12: a step of twelve 4 KiB HtoD calls
     w += ctx.encode_call(7 + i, gen.PROC_H2D, [(crk.K_U64, base + 4096 * (i + 1)), (crk.K_OPAQUE_VAR, data),
                                               (crk.K_U64, 4096)], ring, w)
 send = crk.Ring.device(1 << 16)
