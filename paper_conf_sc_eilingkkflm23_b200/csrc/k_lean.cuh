@@ -93,33 +93,40 @@ struct ItemRows {  // the index's parsed-item columns (by value: no kernel param
 };
 __device__ __noinline__ bool lean_items(const uint8_t* sh, const LeanState& L, const LeanRec& q, const Schema& s,
                                         bool strict, ItemRows out, uint64_t b) {
+  // the record's fields in registers; a single-fragment record at an aligned cursor reads its words directly
+  const uint32_t so = q.so_, sm = q.sm_, len = q.len;
+  const uint64_t c4 = q.cur + 4;
+  const bool direct = q.nf == 1 && !(c4 & 3);
+  auto word = [&](uint64_t at) {
+    return direct ? bswap32(*reinterpret_cast<const uint32_t*>(sh + so + ((c4 + at) & sm))) : lean_be32(sh, L, q, at);
+  };
   uint64_t o = 40;
 #pragma unroll 1
   for (uint32_t it = 0; it < s.n_items; ++it) {
     const uint32_t code = s.items[it], kind = code & 0xff, fixed = code >> 8;
     uint64_t off = o, cnt = 0, val = 0;
     if (kind == CRK_K_U32) {
-      if (o + 4 > q.len) return false;
-      val = lean_be32(sh, L, q, o);
+      if (o + 4 > len) return false;
+      val = word(o);
       o += 4;
     } else if (kind == CRK_K_U64) {
-      if (o + 8 > q.len) return false;
-      val = ((uint64_t)lean_be32(sh, L, q, o) << 32) | lean_be32(sh, L, q, o + 4);
+      if (o + 8 > len) return false;
+      val = ((uint64_t)word(o) << 32) | word(o + 4);
       o += 8;
     } else {
       const uint32_t es = elem_size_k(kind);
       if (!es) return false;
       uint64_t c = fixed;
       if (kind == CRK_K_OPAQUE_VAR || (kind >= CRK_K_I32_VAR && kind <= CRK_K_F64_VAR)) {
-        if (o + 4 > q.len) return false;
-        c = lean_be32(sh, L, q, o);
+        if (o + 4 > len) return false;
+        c = word(o);
         o += 4;
       }
       const uint64_t bytes = c * es, pn = pad4(bytes);
-      if (o + bytes + pn > q.len) return false;
+      if (o + bytes + pn > len) return false;
 #pragma unroll 1
       for (uint64_t i = 0; strict && i < pn; ++i)
-        if (lean_byte(sh, L, q, o + bytes + i) != 0) return false;
+        if ((direct ? sh[so + ((c4 + o + bytes + i) & sm)] : lean_byte(sh, L, q, o + bytes + i)) != 0) return false;
       off = o;
       cnt = c;
       o += bytes + pn;
@@ -131,7 +138,7 @@ __device__ __noinline__ bool lean_items(const uint8_t* sh, const LeanState& L, c
       out.value[b + it] = val;
     }
   }
-  return !strict || o == q.len;
+  return !strict || o == len;
 }
 
 __device__ __noinline__ bool region_ok(uint64_t base, uint64_t bytes, uint64_t ptr, uint64_t n) {
