@@ -417,8 +417,15 @@ def served(ctx, sizes_h2d, sizes_d2h, streams=1, reps=20):
                                                + 64 * len(per[s]) + 4096)))
     idx = ctx.index(streams, 1 << 20, 1 << 14)
     ms = timed(lambda _: idx.serve(rings, sends, [0] * streams, base, region.numel()), reps)
-    ok = all(r["status"] == 0 for r in idx.ring_results(streams))
-    ok &= all(bool(torch.equal(region[o:o + p.numel()], p)) for o, p in srcs[:4])
+    res = idx.ring_results(streams)
+    ok = all(r["status"] == 0 and r["n_records"] == len(per[s]) for s, r in enumerate(res))
+    # every destination; every ring's reply bytes (an HtoD reply carries a status, a DtoH one its data)
+    F = ctx.cfg.frag_payload
+    ok &= all(bool(torch.equal(region[o:o + p.numel()], p)) for o, p in srcs)
+    ok &= all(r["reply_bytes"] == sum(crk.wire_size_d2h(0, 1, F) if k == "h" else crk.wire_size_d2h(n, 0, F)
+                                      for k, _, n, _ in per[s]) for s, r in enumerate(res))
+    ok &= all(bool(torch.equal(region[o:o + n].cpu(), torch.from_numpy(gen.random_bytes(7000 + i, n))))
+              for s in range(streams) for k, i, n, o in per[s] if k == "d")  # DtoH sources untouched
     pay = total_h + sum(sizes_d2h)
     return {"ms": round(ms, 4), "payload_bytes": pay, "gbs": round(pay / ms / 1e6, 1), "ok": bool(ok)}
 
