@@ -163,7 +163,19 @@ def serve_latency(ctx):
     us_graph = timed(lambda _: g.launch(), 500) * 1e3
     ok = bool(torch.equal(region[4096:8192], data)) and idx.ring_results(1)[0]["reply_bytes"] == 32
     g.close()
-    return {"serve_launches_us": round(us_launch, 2), "serve_graph_us": round(us_graph, 2), "ok": ok}
+    # one control call of a registered procedure per step, graph replay (the server's NEXT3 control call)
+    ctx.register_schema(60, [crk.K_U64, crk.K_U32, crk.K_U32, crk.K_OPAQUE_VAR])
+    ring4 = crk.Ring.device(1 << 12)
+    w4 = ctx.encode_call(9, 60, [(crk.K_U64, 0x7F00DEADBEEF), (crk.K_U32, 148), (crk.K_U32, 256),
+                                 (crk.K_OPAQUE_VAR, data[:64])], ring4, 0)
+    bell4 = torch.tensor([0, w4, 0], dtype=torch.int64, device=dev)
+    g4 = idx.serve_graph([ring4], [send], base, region.numel(), bell4)
+    us_ctl = timed(lambda _: g4.launch(), 500) * 1e3
+    res4 = idx.ring_results(1)[0]
+    ok4 = res4["status"] == 0 and res4["n_records"] == 1 and res4["reply_bytes"] == 0
+    g4.close()
+    return {"serve_launches_us": round(us_launch, 2), "serve_graph_us": round(us_graph, 2), "ok": ok,
+            "control_call_graph_us": round(us_ctl, 2), "control_ok": bool(ok4)}
 
 
 def server_latency(ctx, reps=2000):
