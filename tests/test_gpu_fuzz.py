@@ -1,6 +1,8 @@
 """Mutation fuzzing of the whole server step against the oracle: valid CALL streams with seeded byte
 flips, header rewrites, truncations and spliced garbage.  Every ring status, consumed cursor, record
 status, reply byte and destination byte must match or_serve exactly (error paths included)."""
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -10,6 +12,8 @@ from paper_conf_sc_eilingkkflm23_b200 import crk, gen
 from tests.gpu_util import ctx_for, d2h_call, h2d_call, make_ring, ocfg, ring_np
 
 pytestmark = pytest.mark.gpu
+# CRK_FUZZ_SEED shifts every seed (longer fuzz campaigns: tools/gpu_tests.sh with the variable set)
+SEED = int(os.environ.get("CRK_FUZZ_SEED", "0"))
 
 if not torch.cuda.is_available():
     pytest.skip("needs a GPU", allow_module_level=True)
@@ -60,7 +64,7 @@ def test_mutated_streams_match_oracle(strict, fused):
                   fused_front_max_window=1 << 30)
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
-    g = gen.rng(2024 + strict)
+    g = gen.rng(2024 + strict + SEED)
     idx = ctx.index(4, 1 << 12, 256)
     skipped = 0
     for trial in range(250):
@@ -131,7 +135,7 @@ def test_mutated_streams_through_persistent_server(strict):
     ctx = ctx_for(cfg, max_record_bytes=1 << 14)
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
-    g = gen.rng(4048 + strict)
+    g = gen.rng(4048 + strict + SEED)
     idx = ctx.index(4, 1 << 12, 256)
     cap, scap = 1 << 16, 1 << 17
     rings = [make_ring(cap) for _ in range(4)]
@@ -194,7 +198,7 @@ def test_mutated_memcpy_streams_lean_boundary(strict, path):
                   lean_backoff=0)  # every step tries the lean path
     region = torch.zeros(1 << 17, dtype=torch.uint8, device="cuda")
     base = region.data_ptr()
-    g = gen.rng(7000 + 2 * strict + (path == "server"))
+    g = gen.rng(7000 + 2 * strict + (path == "server") + SEED)
     idx = ctx.index(4, 1 << 12, 256)
     cap, scap = 1 << 16, 1 << 17
     rings = [make_ring(cap) for _ in range(4)]
