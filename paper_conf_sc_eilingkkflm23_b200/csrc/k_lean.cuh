@@ -458,6 +458,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     if (B) B->res[tid] = rr;
     ix.rec_prefix[tid] = L.prefix[tid];
   }
+  STEP_MARK(tid == 0, 1, 0);
   if (tid == 0) {
     ix.rec_prefix[n] = N;
     *ix.total = N;
@@ -517,6 +518,7 @@ __device__ __forceinline__ bool lean_step(const IndexDev& ix, const ConfigDev& c
     ix.s_reply_err[d] = q.ctrl ? -1 : 0;  // a control call has no reply
     ix.s_reply_off[d] = q.ctrl ? 0 : q.off;  // (0 when the record has no reply, as the general phases write)
     ix.s_reply_wire[d] = q.w;
+    STEP_MARK(tid == 0, 2, 0);
     // distinct xids into the cleared table: the first free slot (a lone record's is its home slot: a plain store)
     const unsigned long long key = ((unsigned long long)q.xid << 32) | d;
     uint32_t h = (q.xid * 0x9E3779B1u) & ix.hash_mask;

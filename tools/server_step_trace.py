@@ -2,7 +2,9 @@
 build.build_variant) for one 4 KiB HtoD CALL per step: %globaltimer at numbered points (crk_device.cuh
 STEP_MARK), each taken once the value it depends on has arrived.  Points: 0 scan start; 8-13 inside
 parse_record (entry, record table, fragment table, ring bytes, lane-0 checks, tables written); 16 jobs staged;
-17 tiles moved; 18 after the move barrier; 19 results published; 20 done_seq released.  The trace is read
+17 tiles moved; 18 after the move barrier; 19 results published; 20 done_seq released.  Lean steps: 21 windows
+copied, 22 walked, 23 checked, 24 offsets, 25 decided, 1 ring results and 2 record rows written, 26 tables done,
+27-30 first warps' moves, 31 replies encoded.  The trace is read
 after each server stop (a device-wide copy would wait for the running server)."""
 import ctypes as C
 import zlib
